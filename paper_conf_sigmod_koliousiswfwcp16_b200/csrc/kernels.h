@@ -1,0 +1,47 @@
+// kernels.h -- host-side launchers of the sm_100a kernels (kernels.cu).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "plan.h"
+
+namespace sb {
+
+struct SlotDev {
+  unsigned char *rows;      // aggregation columns / IStream rows
+  void *hdr;                // saber_win_hdr[win_cap]
+  int64_t *counts;          // per (window, slab) row counts → offsets
+  SlotMeta *meta;
+};
+
+struct QueryDev {
+  State *st;
+  uint64_t *table;          // pane ring: R slots × slot_words
+  int64_t *pane_ts;         // R
+  uint64_t *tile_status;    // IStream look-back
+  int64_t tile_status_cap;
+  unsigned char *carry[2];  // IStream raw tail
+  int64_t carry_cap;        // tuples
+  int *tile_ctr;
+};
+
+// one task of an aggregation (RStream) query
+cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
+                            int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
+                            int p1_grid, int p2_grid, int win_chunk, cudaStream_t st);
+// one task of a σ/π (IStream) query
+cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
+                               int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
+                               int sel_grid, cudaStream_t st);
+cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, cudaStream_t st);
+cudaError_t launch_partition_plan(int ts_word, int tuple_words, int win_kind, int64_t s, int64_t l,
+                                  int64_t T0, const void *tuples, int64_t begin, int64_t n,
+                                  int64_t *dev_out2, cudaStream_t st);
+// occupancy helpers
+int p1_smem_bytes(const Plan &p);
+int p1_blocks_per_sm(const Plan &p);
+int p2_blocks_per_sm(const Plan &p);
+int sel_blocks_per_sm(const Plan &p);
+cudaError_t set_kernel_attributes(const Plan &p);
+
+}  // namespace sb

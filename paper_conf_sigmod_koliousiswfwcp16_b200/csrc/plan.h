@@ -1,0 +1,118 @@
+// plan.h -- query plan and per-query device state shared by the host runtime
+// (runtime.cu) and the kernels (kernels.cu).  Product code: nothing here is
+// shared with oracle/.
+//
+// A plan is derived once per query at saber_query_create from the paper's
+// query q = (ω, f^q, φ^q) (§2.4):
+//   pane length g = gcd(s, l), K = s/g panes per window, L = l/g panes per
+//   slide; window j covers panes [j·L, j·L+K)  (panes: L180-181, L1275-1280).
+// Pane partials (the window-fragment results f_f of §3) live in a
+// device ring of R pane slots indexed by pane id mod R; every slot holds a
+// table of C accumulator entries (C = 1 without GROUP BY, G for a declared
+// dense key domain, CAP for an open-addressing hash of arbitrary keys).
+#pragma once
+#include <stdint.h>
+
+namespace sb {
+
+constexpr int kMaxPred = 16, kMaxProj = 16, kMaxAgg = 8, kMaxKey = 4, kMaxField = 8, kMaxHave = 8;
+constexpr int kMaxCols = 12;
+constexpr int kMaxTupleWords = 64;      // tuples up to 256 bytes
+
+enum { T_I32 = 0, T_I64 = 1, T_F32 = 2, T_F64 = 3 };
+enum { OP_LT = 0, OP_LE, OP_GT, OP_GE, OP_EQ, OP_NE };
+enum { AG_SUM = 0, AG_COUNT, AG_AVG, AG_MIN, AG_MAX };
+enum { KM_GLOBAL = 0, KM_DENSE = 1, KM_HASH = 2 };
+enum { KP_RADIX = 0, KP_BIASED64 = 1, KP_BIASED32X2 = 2 };
+// accumulator fields (besides the count): fp64 sum, int64 sum, min, max.
+// min/max hold an order-preserving u64 encoding of int64 / double values.
+enum { FK_SUM_F = 0, FK_SUM_I = 1, FK_MIN = 2, FK_MAX = 3 };
+enum { WK_COUNT = 0, WK_TIME = 1 };
+
+// error bits in State::error (first one wins for the status)
+enum {
+  ERR_ORDER = 1, ERR_TS = 2, ERR_KEY = 4, ERR_CAPACITY = 8, ERR_RESULT = 16, ERR_CARRY = 32
+};
+
+struct Pred { int32_t word, type, op, pad; int64_t ival; double fval; };
+struct Key  { int32_t word, type, div, pad; int64_t domain, stride; };
+struct Field { int32_t kind, word, type, pad; };
+struct AggOut { int32_t fn, field, is_float_col, out_float; };
+struct Have { int32_t agg, op, pad0, pad1; int64_t ival; double fval; };
+
+struct Plan {
+  // schema
+  int32_t tuple_bytes, tuple_words, ts_word, chunk_mask;   // chunk = 16 bytes
+  // window ω(s,l), panes
+  int32_t win_kind, pad0;
+  int64_t s, l, T0, g, K, L;
+  // σ
+  int32_t npred, pad1;
+  Pred pred[kMaxPred];
+  // π (IStream): output word i of a row comes from tuple word proj_word[i]
+  int32_t nproj, out_row_words;
+  int32_t proj_word[2 * kMaxProj];
+  // α
+  int32_t nagg, nf;
+  AggOut agg[kMaxAgg];
+  Field field[kMaxField];
+  // γ
+  int32_t nkeys, key_mode, key_pack, pad2;
+  Key key[kMaxKey];
+  int64_t G;                      // dense key count (DENSE), 1 (GLOBAL)
+  int32_t nhave, pad3;
+  Have have[kMaxHave];
+  // pane ring geometry
+  int64_t C;                      // entries per pane slot
+  int64_t R;                      // ring slots (power of two)
+  int64_t slot_words;             // 8-byte words per slot
+  int32_t hash_bits, pad4;        // log2(C) in HASH mode
+  // phase-1 warp-private table
+  int32_t local_direct;           // 1: direct index (pl*C + key); 0: one-pane hash
+  int32_t local_entries;          // entries per warp
+  int32_t local_pl;               // panes per direct table
+  int32_t local_bytes;            // bytes per warp
+  // phase-2 window assembly
+  int32_t S, SB, GS, pad5;        // key slabs, slots per slab, threads per slab group
+  int32_t state_cap, p2_smem;     // hash state entries per CTA, dynamic smem bytes
+  int32_t has_minmax, has_inv;    // min/max fields present; invertible (count/sum) fields
+  // output
+  int32_t ncols, row_bytes;       // aggregation output columns, bytes per row
+  int32_t col_bytes[kMaxCols];
+  int64_t col_off[kMaxCols];      // byte offset of each column array in a result slot
+  int64_t rows_cap;               // rows per result slot
+  int64_t win_cap;                // windows per result slot
+  int64_t first_window;           // windows < first_window are not emitted
+  int64_t carry_cap;              // IStream: raw tail tuples kept between tasks
+};
+
+// Per-query device state, updated only by kernels on the query's stream.
+struct State {
+  int32_t error;                  // ERR_* bits, sticky
+  int32_t has_tau;
+  int64_t tau_last;               // time windows: last τ seen
+  int64_t pos_next;               // global position of the next tuple
+  int64_t J0;                     // first window not yet emitted
+  int64_t J1;                     // windows closed after the current task
+  int64_t zeroed_hi;              // pane slots for panes < zeroed_hi are initialised
+  int64_t zero_lo, zero_hi;       // pane range to initialise for the current task
+  int64_t pane_hi;                // highest pane touched so far
+  int64_t max_probe;              // longest pane-hash probe (HASH mode)
+  // current task
+  int64_t task_pos, task_n;
+  // IStream
+  int64_t cover_lo, cover_hi;     // emitted positions of the current task: [cover_lo, cover_hi)
+  int64_t carry_pos, carry_n;     // uncovered raw tail kept from earlier tasks
+  int32_t carry_sel, first_task;  // which carry buffer is current; first task flag
+  int64_t sel_rows;               // rows written by the compaction kernel
+  int64_t tile_epoch;             // look-back epoch
+};
+
+// Per result slot metadata, copied to the host after a task.
+struct SlotMeta {
+  int64_t first_window, nwindows, nrows, ntuples;
+  int32_t error, pad;
+  int64_t pos_end, tau_last;
+};
+
+}  // namespace sb

@@ -1,0 +1,794 @@
+// runtime.cu -- host runtime behind include/saber.h.
+//
+//   planner     query → Plan (pane length g = gcd(s,l), key regime, table sizes)
+//   dispatcher  cuts the submitted byte stream into φ-byte query tasks with
+//               monotone task ids (§4.1)
+//   ingest      pinned staging ring + H2D on a copy stream, event-chained to the
+//               compute stream (the paper's copyin/movein stages, §5.2)
+//   result ring result slot = task id mod slots; poll hands slices out in task
+//               order (the ordered output stream of §4.3)
+// Every step of a task executes in kernels.cu; nothing here touches tuple data.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/saber.h"
+#include "kernels.h"
+#include "plan.h"
+
+using namespace sb;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+enum SlotState { SLOT_FREE = 0, SLOT_BUSY = 1, SLOT_POLLED = 2 };
+
+struct Slot {
+  SlotDev dev{};
+  unsigned char *h_rows = nullptr;
+  saber_win_hdr *h_hdr = nullptr;
+  SlotMeta *h_meta = nullptr;
+  cudaEvent_t done = nullptr;
+  int64_t task_id = -1;
+  int state = SLOT_FREE;
+  SlotMeta meta{};
+};
+
+struct Stage {
+  unsigned char *h = nullptr;   // pinned
+  unsigned char *d = nullptr;   // device
+  cudaEvent_t free_ev = nullptr;
+  bool used = false;
+};
+
+int64_t gcd64(int64_t a, int64_t b) { while (b) { int64_t t = a % b; a = b; b = t; } return a; }
+int64_t next_pow2(int64_t x) { int64_t p = 1; while (p < x) p <<= 1; return p; }
+int64_t floor_pow2(int64_t x) { int64_t p = 1; while (p * 2 <= x) p <<= 1; return p; }
+int type_bytes(int t) { return (t == T_I32 || t == T_F32) ? 4 : 8; }
+bool is_float(int t) { return t == T_F32 || t == T_F64; }
+
+}  // namespace
+
+struct saber_query {
+  Plan plan{};
+  int ncols_schema = 0;
+  std::vector<int> col_type, col_off;
+  saber_window win{};
+  saber_config cfg{};
+  int device = 0, nsm = 148;
+  cudaStream_t cs = nullptr, h2d = nullptr, d2h = nullptr;
+  QueryDev qd{};
+  std::vector<Slot> slots;
+  std::vector<Stage> stages;
+  int cur_stage = 0;
+  int64_t stage_fill = 0;       // bytes in stages[cur_stage]
+  int64_t task_tuples = 0;
+  int64_t next_task = 0, next_poll = 0;
+  int p1_grid = 0, p2_grid = 0, sel_grid = 0, win_chunk = 32;
+  bool closed = false;
+  saber_status sticky = SABER_OK;
+  std::string err;
+  saber_stats stats{};
+  std::vector<std::pair<void *, size_t>> registered;
+  std::mutex mu;
+  int64_t *d_tmp = nullptr;
+};
+
+static saber_status fail(saber_query *q, saber_status s, const std::string &msg) {
+  if (q) q->err = msg;
+  g_last_error = msg;
+  return s;
+}
+
+#define CK(call)                                                                                 \
+  do {                                                                                           \
+    cudaError_t e_ = (call);                                                                     \
+    if (e_ != cudaSuccess) {                                                                     \
+      return fail(q, SABER_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_));          \
+    }                                                                                            \
+  } while (0)
+
+static saber_status status_from_err(int e) {
+  if (e & ERR_ORDER) return SABER_EORDER;
+  if (e & ERR_TS) return SABER_ETS;
+  if (e & ERR_KEY) return SABER_EKEY;
+  if (e & (ERR_CAPACITY | ERR_CARRY)) return SABER_ECAPACITY;
+  if (e & ERR_RESULT) return SABER_ENOMEM;
+  return SABER_OK;
+}
+static const char *err_text(int e) {
+  if (e & ERR_ORDER) return "timestamps are not non-decreasing (PAPER.md L347-349)";
+  if (e & ERR_TS) return "negative timestamp (time domain is {0,1,...}, L349-350)";
+  if (e & ERR_KEY) return "GROUP BY key outside its declared domain (or reserved key value)";
+  if (e & ERR_CAPACITY) return "pane hash table / pane ring / window state capacity exceeded";
+  if (e & ERR_CARRY) return "IStream carry (uncovered tail) exceeds its capacity";
+  if (e & ERR_RESULT) return "task output exceeds the result slot capacity (raise result_bytes or lower task_bytes)";
+  return "";
+}
+
+// ---------------------------------------------------------------------------
+// planner
+static saber_status build_plan(saber_query *q, const saber_schema *sc, const saber_operator *op,
+                               const saber_window *w) {
+  Plan &p = q->plan;
+  std::memset(&p, 0, sizeof(p));
+  if (!sc || !op || !w) return fail(q, SABER_EINVAL, "null argument");
+  if (sc->ncols < 1 || !sc->types || !sc->offsets) return fail(q, SABER_EINVAL, "schema needs columns");
+  if (sc->tuple_bytes % 16 || sc->tuple_bytes < 16 || sc->tuple_bytes > 64)
+    return fail(q, SABER_EINVAL, "tuple_bytes must be 16, 32, 48 or 64");
+  q->ncols_schema = sc->ncols;
+  for (int c = 0; c < sc->ncols; ++c) {
+    int t = sc->types[c], o = sc->offsets[c];
+    if (t < 0 || t > 3) return fail(q, SABER_EINVAL, "unknown column type");
+    int b = type_bytes(t);
+    if (o < 0 || o % b || o + b > sc->tuple_bytes) return fail(q, SABER_EINVAL, "misaligned or out-of-range column");
+    q->col_type.push_back(t);
+    q->col_off.push_back(o);
+  }
+  if (sc->ts_col < 0 || sc->ts_col >= sc->ncols || sc->types[sc->ts_col] != SABER_I64)
+    return fail(q, SABER_EINVAL, "ts_col must be an I64 column");
+  if (w->size < 1 || w->slide < 1) return fail(q, SABER_EINVAL, "window size and slide must be >= 1");
+  if (w->slide > w->size) return fail(q, SABER_EINVAL, "slide > size is not supported (PAPER.md L375)");
+  if (w->kind != SABER_WIN_COUNT && w->kind != SABER_WIN_TIME) return fail(q, SABER_EINVAL, "window kind");
+  if (w->kind == SABER_WIN_TIME && w->origin < 0) return fail(q, SABER_EINVAL, "negative origin");
+  if (op->npred < 0 || op->npred > kMaxPred || (op->npred && !op->where)) return fail(q, SABER_EINVAL, "where");
+  if (op->nagg < 0 || op->nagg > kMaxAgg || (op->nagg && !op->aggs)) return fail(q, SABER_EINVAL, "aggs");
+  if (op->nkeys < 0 || op->nkeys > kMaxKey || (op->nkeys && !op->group_by)) return fail(q, SABER_EINVAL, "group_by");
+  if (op->nproj < 0 || op->nproj > kMaxProj || (op->nproj && !op->proj)) return fail(q, SABER_EINVAL, "proj");
+  if (op->nhave < 0 || op->nhave > kMaxHave || (op->nhave && !op->having)) return fail(q, SABER_EINVAL, "having");
+  if (op->nagg == 0 && op->nproj == 0) return fail(q, SABER_EINVAL, "query needs aggregates or a projection");
+  if (op->nagg > 0 && op->nproj > 0) return fail(q, SABER_EINVAL, "projection and aggregation are exclusive");
+  if (op->nagg == 0 && (op->nkeys || op->nhave)) return fail(q, SABER_EINVAL, "GROUP BY / HAVING need aggregates");
+  if (op->nkeys + op->nagg > kMaxCols) return fail(q, SABER_EINVAL, "too many output columns");
+
+  auto colok = [&](int c) { return c >= 0 && c < sc->ncols; };
+  p.tuple_bytes = sc->tuple_bytes;
+  p.tuple_words = sc->tuple_bytes / 4;
+  p.ts_word = sc->offsets[sc->ts_col] / 4;
+  unsigned mask = 1u << (sc->offsets[sc->ts_col] / 16);
+  auto use = [&](int c) { mask |= 1u << (sc->offsets[c] / 16); };
+  p.win_kind = w->kind == SABER_WIN_TIME ? WK_TIME : WK_COUNT;
+  p.s = w->size; p.l = w->slide; p.T0 = w->kind == SABER_WIN_TIME ? w->origin : 0;
+  p.g = gcd64(p.s, p.l); p.K = p.s / p.g; p.L = p.l / p.g;
+
+  p.npred = op->npred;
+  for (int i = 0; i < op->npred; ++i) {
+    const saber_pred &pr = op->where[i];
+    if (!colok(pr.col) || pr.op < SABER_LT || pr.op > SABER_NE) return fail(q, SABER_EINVAL, "bad predicate");
+    p.pred[i].word = sc->offsets[pr.col] / 4;
+    p.pred[i].type = sc->types[pr.col];
+    p.pred[i].op = pr.op;
+    p.pred[i].ival = pr.ival;
+    p.pred[i].fval = pr.fval;
+    use(pr.col);
+  }
+  p.nproj = op->nproj;
+  int ow = 0;
+  for (int i = 0; i < op->nproj; ++i) {
+    int c = op->proj[i];
+    if (!colok(c)) return fail(q, SABER_EINVAL, "bad projection column");
+    int nw = type_bytes(sc->types[c]) / 4;
+    for (int k = 0; k < nw; ++k) p.proj_word[ow++] = sc->offsets[c] / 4 + k;
+    use(c);
+  }
+  p.out_row_words = ow;
+
+  // aggregates → accumulator fields (shared when equal)
+  p.nagg = op->nagg;
+  p.nf = 0;
+  for (int a = 0; a < op->nagg; ++a) {
+    const saber_agg &ag = op->aggs[a];
+    if (ag.fn < SABER_SUM || ag.fn > SABER_MAX) return fail(q, SABER_EINVAL, "bad aggregate");
+    AggOut &o = p.agg[a];
+    o.fn = ag.fn;
+    o.field = -1;
+    if (ag.fn == SABER_COUNT) { o.is_float_col = 0; o.out_float = 0; continue; }
+    if (!colok(ag.col)) return fail(q, SABER_EINVAL, "bad aggregate column");
+    int t = sc->types[ag.col];
+    use(ag.col);
+    int kind = (ag.fn == SABER_MIN) ? FK_MIN : (ag.fn == SABER_MAX) ? FK_MAX : (is_float(t) ? FK_SUM_F : FK_SUM_I);
+    int word = sc->offsets[ag.col] / 4;
+    int f = -1;
+    for (int i = 0; i < p.nf; ++i)
+      if (p.field[i].kind == kind && p.field[i].word == word) f = i;
+    if (f < 0) {
+      if (p.nf == kMaxField) return fail(q, SABER_EINVAL, "too many accumulator fields");
+      f = p.nf++;
+      p.field[f].kind = kind; p.field[f].word = word; p.field[f].type = t;
+    }
+    o.field = f;
+    o.is_float_col = is_float(t);
+    o.out_float = (ag.fn == SABER_AVG) || is_float(t);
+    if (kind == FK_MIN || kind == FK_MAX) p.has_minmax = 1;
+  }
+  // GROUP BY keys
+  p.nkeys = op->nkeys;
+  bool all_dom = op->nkeys > 0;
+  long double prod = 1;
+  for (int i = 0; i < op->nkeys; ++i) {
+    const saber_keyexpr &k = op->group_by[i];
+    if (!colok(k.col) || is_float(sc->types[k.col])) return fail(q, SABER_EINVAL, "GROUP BY needs integer columns");
+    if (k.div == 0) return fail(q, SABER_EINVAL, "key divisor is 0");
+    if (k.domain < 0) return fail(q, SABER_EINVAL, "negative key domain");
+    p.key[i].word = sc->offsets[k.col] / 4;
+    p.key[i].type = sc->types[k.col];
+    p.key[i].div = k.div;
+    p.key[i].domain = k.domain;
+    all_dom &= k.domain > 0;
+    prod *= (long double)(k.domain > 0 ? k.domain : 1);
+    use(k.col);
+  }
+  const int64_t kDenseMax = 8192;
+  if (op->nkeys == 0) {
+    p.key_mode = KM_GLOBAL; p.key_pack = KP_RADIX; p.G = 1;
+  } else if (all_dom && prod < 4.0e18L) {
+    p.key_pack = KP_RADIX;
+    int64_t stride = 1;
+    for (int i = op->nkeys - 1; i >= 0; --i) { p.key[i].stride = stride; stride *= p.key[i].domain; }
+    p.G = stride;
+    p.key_mode = (p.G <= kDenseMax) ? KM_DENSE : KM_HASH;
+  } else if (op->nkeys == 1) {
+    p.key_pack = KP_BIASED64; p.key_mode = KM_HASH; p.G = 0;
+  } else if (op->nkeys == 2) {
+    p.key_pack = KP_BIASED32X2; p.key_mode = KM_HASH; p.G = 0;
+  } else {
+    return fail(q, SABER_EINVAL, "more than two GROUP BY columns need declared domains");
+  }
+  p.nhave = op->nhave;
+  for (int h = 0; h < op->nhave; ++h) {
+    const saber_pred &hv = op->having[h];
+    if (hv.col < 0 || hv.col >= op->nagg || hv.op < SABER_LT || hv.op > SABER_NE)
+      return fail(q, SABER_EINVAL, "bad HAVING term");
+    p.have[h].agg = hv.col; p.have[h].op = hv.op; p.have[h].ival = hv.ival; p.have[h].fval = hv.fval;
+  }
+  p.chunk_mask = (int)mask;
+  p.first_window = q->cfg.first_window;
+  if (p.first_window < 0) return fail(q, SABER_EINVAL, "first_window < 0");
+  return SABER_OK;
+}
+
+static saber_status size_plan(saber_query *q) {
+  Plan &p = q->plan;
+  const saber_config &c = q->cfg;
+  q->task_tuples = c.task_bytes / p.tuple_bytes;
+  if (q->task_tuples < 1) return fail(q, SABER_EINVAL, "task_bytes smaller than one tuple");
+  if (q->task_tuples > (1ll << 31)) return fail(q, SABER_EINVAL, "task_bytes too large (max 2^31 tuples)");
+  const int64_t T = q->task_tuples;
+  if (p.nagg > 0) {
+    // entries per pane slot
+    if (p.key_mode == KM_GLOBAL) p.C = 1;
+    else if (p.key_mode == KM_DENSE) p.C = p.G;
+    else {
+      int64_t cap = c.hash_capacity;
+      if (cap <= 0) {
+        int64_t distinct = p.win_kind == WK_COUNT ? p.g : 4096;
+        if (p.key_pack == KP_RADIX && p.G < distinct) distinct = p.G;
+        cap = next_pow2(std::max<int64_t>(64, 2 * distinct));
+        cap = std::min<int64_t>(cap, 1 << 16);
+      }
+      if (cap & (cap - 1)) return fail(q, SABER_EINVAL, "hash_capacity must be a power of two");
+      p.C = cap;
+      int b = 0; while ((1ll << b) < cap) ++b;
+      p.hash_bits = b;
+    }
+    p.slot_words = (p.key_mode == KM_HASH ? p.C : 0) + p.C * (1 + p.nf);
+    const int64_t slot_bytes = p.slot_words * 8;
+    const int64_t budget = 2ll << 30;
+    int64_t need = p.K + p.L + 2;
+    int64_t R;
+    if (c.max_panes > 0) R = next_pow2(c.max_panes + need);
+    else if (p.win_kind == WK_COUNT) R = next_pow2(need + (T + p.g - 1) / p.g + 1);
+    else R = std::min(next_pow2(need + (1 << 20)), floor_pow2(std::max<int64_t>(budget / slot_bytes, 1)));
+    if (R < need + 16) R = next_pow2(need + 16);
+    p.R = R;
+    // phase-1 warp-private table (12 KiB per warp)
+    const int budget_w = 12 * 1024;
+    const int ed = 4 + 8 * p.nf, eh = 12 + 8 * p.nf;
+    if (p.key_mode != KM_HASH && p.C * 2 * ed <= budget_w) {
+      p.local_direct = 1;
+      int te = budget_w / ed;
+      p.local_pl = (int)(te / p.C);
+      p.local_entries = p.local_pl * (int)p.C;
+      p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
+    } else {
+      p.local_direct = 0;
+      p.local_entries = (int)floor_pow2(budget_w / eh);
+      p.local_pl = 1;
+      p.local_bytes = ((p.local_entries * eh) + 15) & ~15;
+    }
+    // phase-2 geometry
+    const int smem_budget = 96 * 1024;
+    if (p.key_mode != KM_HASH) {
+      p.GS = p.C <= 256 ? 32 : 256;
+      const int gpb = 256 / p.GS;
+      int sb = p.GS == 32 ? 256 : 2048;
+      while (sb > 1 && (int64_t)gpb * sb * 8 * (1 + p.nf) > smem_budget) sb >>= 1;
+      if (sb > p.C) sb = (int)p.C;
+      p.SB = sb;
+      p.S = (int)((p.C + sb - 1) / sb);
+      p.p2_smem = gpb * sb * 8 * (1 + p.nf);
+    } else {
+      p.GS = 256;
+      p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + p.nf)));
+      const double A = (double)(p.K + q->win_chunk * p.L) / 2.0;
+      const double B = p.key_pack == KP_RADIX ? (double)p.G / (double)p.C : 1e30;
+      const double per_slot = std::max(1e-9, std::min(A, B));
+      int64_t sb = floor_pow2(std::max<int64_t>(1, (int64_t)(p.state_cap / (2.0 * per_slot))));
+      if (sb > p.C) sb = p.C;
+      p.SB = (int)sb;
+      p.S = (int)(p.C / sb);
+      p.p2_smem = p.state_cap * 8 * (2 + p.nf);
+    }
+    // output columns (keys then aggregates)
+    p.ncols = p.nkeys + p.nagg;
+    p.row_bytes = 0;
+    for (int i = 0; i < p.nkeys; ++i) { p.col_bytes[i] = type_bytes(p.key[i].type); p.row_bytes += p.col_bytes[i]; }
+    for (int a = 0; a < p.nagg; ++a) { p.col_bytes[p.nkeys + a] = 8; p.row_bytes += 8; }
+    p.win_cap = p.win_kind == WK_COUNT ? T / p.l + 4 : p.R / p.L + 4;
+    int64_t rows_per_win = p.key_mode == KM_GLOBAL ? 1 : p.key_mode == KM_DENSE ? p.G
+                           : (p.win_kind == WK_COUNT ? std::min<int64_t>(p.s, p.C * p.K) : p.C * p.K);
+    int64_t rb = c.result_bytes;
+    if (rb <= 0) {
+      long double bound = (long double)p.win_cap * rows_per_win * p.row_bytes;
+      rb = (int64_t)std::min<long double>(std::max<long double>(bound, 1 << 20), 1ll << 30);
+    }
+    p.rows_cap = std::max<int64_t>(1, rb / p.row_bytes);
+    int64_t off = 0;
+    for (int i = 0; i < p.ncols; ++i) {
+      p.col_off[i] = off;
+      off += ((p.rows_cap * p.col_bytes[i]) + 255) & ~255ll;
+    }
+  } else {
+    p.carry_cap = p.win_kind == WK_COUNT ? p.s + p.l + 16 : T + 16;
+    p.rows_cap = T + p.carry_cap;
+    p.win_cap = p.win_kind == WK_COUNT ? T / p.l + 4 : T + 4;
+    p.S = 1;
+  }
+  return SABER_OK;
+}
+
+// ---------------------------------------------------------------------------
+static saber_status alloc_query(saber_query *q) {
+  Plan &p = q->plan;
+  CK(cudaSetDevice(q->device));
+  CK(cudaStreamCreateWithFlags(&q->cs, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&q->h2d, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&q->d2h, cudaStreamNonBlocking));
+  CK(cudaMalloc(&q->qd.st, sizeof(State)));
+  CK(cudaMalloc(&q->qd.tile_ctr, 64));
+  CK(cudaMalloc(&q->d_tmp, 64));
+  if (p.nagg > 0) {
+    CK(cudaMalloc(&q->qd.table, (size_t)p.R * p.slot_words * 8));
+    CK(cudaMalloc(&q->qd.pane_ts, (size_t)p.R * 8));
+  } else {
+    q->qd.carry_cap = p.carry_cap;
+    CK(cudaMalloc(&q->qd.carry[0], (size_t)p.carry_cap * p.tuple_bytes));
+    CK(cudaMalloc(&q->qd.carry[1], (size_t)p.carry_cap * p.tuple_bytes));
+    q->qd.tile_status_cap = (q->task_tuples + p.carry_cap) / 2048 + 4;
+    CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
+    CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
+  }
+  const int nslots = q->cfg.result_slots > 0 ? q->cfg.result_slots : 8;
+  q->slots.resize(nslots);
+  const size_t rows_bytes = p.nagg > 0 ? (size_t)p.col_off[p.ncols - 1] + (((p.rows_cap * p.col_bytes[p.ncols - 1]) + 255) & ~255ll)
+                                       : (size_t)p.rows_cap * p.out_row_words * 4;
+  for (auto &s : q->slots) {
+    CK(cudaMalloc(&s.dev.rows, rows_bytes ? rows_bytes : 16));
+    CK(cudaMalloc(&s.dev.hdr, (size_t)p.win_cap * sizeof(saber_win_hdr)));
+    CK(cudaMalloc(&s.dev.counts, (size_t)p.win_cap * std::max(1, p.S) * 8));
+    CK(cudaMalloc(&s.dev.meta, sizeof(SlotMeta)));
+    CK(cudaMallocHost(&s.h_meta, sizeof(SlotMeta)));
+    if (q->cfg.result_mode == SABER_RESULTS_HOST) {
+      CK(cudaMallocHost(&s.h_rows, rows_bytes ? rows_bytes : 16));
+      CK(cudaMallocHost(&s.h_hdr, (size_t)p.win_cap * sizeof(saber_win_hdr)));
+    }
+    CK(cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
+  }
+  CK(set_kernel_attributes(p));
+  CK(cudaDeviceGetAttribute(&q->nsm, cudaDevAttrMultiProcessorCount, q->device));
+  if (p.nagg > 0) {
+    q->p1_grid = p1_blocks_per_sm(p) * q->nsm;
+    q->p2_grid = p2_blocks_per_sm(p) * q->nsm * 2;
+  } else {
+    q->sel_grid = sel_blocks_per_sm(p) * q->nsm;
+  }
+  CK(launch_init_state(p, q->qd, q->cfg.base_index, q->cs));
+  CK(cudaStreamSynchronize(q->cs));
+  return SABER_OK;
+}
+
+static saber_status check_sticky(saber_query *q) {
+  if (q->sticky != SABER_OK) return fail(q, q->sticky, q->err);
+  return SABER_OK;
+}
+
+static int free_slots(saber_query *q) {
+  int n = 0;
+  for (auto &s : q->slots) n += s.state == SLOT_FREE;
+  return n;
+}
+
+// enqueue one task (device-resident tuples) on the compute stream
+static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuples, int final_, int has_wm, int64_t wm) {
+  Slot &s = q->slots[q->next_task % (int64_t)q->slots.size()];
+  if (s.state != SLOT_FREE) return fail(q, SABER_EAGAIN, "no free result slot");
+  const Plan &p = q->plan;
+  cudaError_t e;
+  if (p.nagg > 0)
+    e = launch_agg_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish, q->p1_grid,
+                        q->p2_grid, q->win_chunk, q->cs);
+  else
+    e = launch_select_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish, q->sel_grid, q->cs);
+  if (e != cudaSuccess) return fail(q, SABER_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e));
+  CK(cudaMemcpyAsync(s.h_meta, s.dev.meta, sizeof(SlotMeta), cudaMemcpyDeviceToHost, q->cs));
+  CK(cudaEventRecord(s.done, q->cs));
+  s.state = SLOT_BUSY;
+  s.task_id = q->next_task++;
+  q->stats.tasks += 1;
+  q->stats.tuples += ntuples;
+  q->stats.bytes_in += ntuples * p.tuple_bytes;
+  // window-fragment classes of this task (count windows, host closed form)
+  if (p.win_kind == WK_COUNT && ntuples > 0) {
+    const int64_t b = q->stats.tuples - ntuples + q->cfg.base_index, e2 = b + ntuples;
+    int64_t c = 0, o = 0, cl = 0, pe = 0;
+    // windows with start in [b, e2) or end-1 in [b, e2) or spanning
+    int64_t jlo = (b - p.s + 1) > 0 ? (b - p.s + 1 + p.l - 1) / p.l : 0;   // first window ending >= b
+    int64_t jhi = (e2 - 1) / p.l;                                          // last window starting < e2
+    for (int64_t j = std::max(jlo, p.first_window); j <= jhi && j - jlo < (1 << 20); ++j) {
+      int64_t a = j * p.l, z = a + p.s - 1;
+      bool si = a >= b && a < e2, ei = z >= b && z < e2;
+      if (si && ei) ++c; else if (si) ++o; else if (ei) ++cl; else ++pe;
+    }
+    q->stats.last_complete = c; q->stats.last_opening = o; q->stats.last_closing = cl; q->stats.last_pending = pe;
+  }
+  return SABER_OK;
+}
+
+// ---------------------------------------------------------------------------
+extern "C" {
+
+const char *saber_version(void) { return "saber-b200 0.1 (sm_100a)"; }
+
+const char *saber_last_error(const saber_query *q) {
+  if (q) return q->err.c_str();
+  return g_last_error.c_str();
+}
+
+saber_status saber_query_create(const saber_schema *schema, const saber_operator *op, const saber_window *window,
+                                const saber_config *cfg, saber_query **out) {
+  saber_query *q = nullptr;
+  if (!out) return fail(nullptr, SABER_EINVAL, "out is NULL");
+  *out = nullptr;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+    cudaGetLastError();
+    return fail(nullptr, SABER_ECUDA, "no CUDA device (there is no CPU path)");
+  }
+  q = new saber_query();
+  if (cfg) q->cfg = *cfg;
+  if (q->cfg.task_bytes <= 0) q->cfg.task_bytes = 64ll << 20;
+  if (q->cfg.pipeline_depth <= 0) q->cfg.pipeline_depth = 3;
+  if (!cfg) q->cfg.emit_on_finish = 1;
+  if (q->cfg.result_mode != SABER_RESULTS_HOST && q->cfg.result_mode != SABER_RESULTS_DEVICE) {
+    delete q;
+    return fail(nullptr, SABER_EINVAL, "result_mode");
+  }
+  if (cfg && cfg->device >= 0) q->device = cfg->device;
+  else cudaGetDevice(&q->device);
+  if (q->device >= ndev) { delete q; return fail(nullptr, SABER_EINVAL, "device ordinal"); }
+  q->win = *window;
+  saber_status st = build_plan(q, schema, op, window);
+  if (st == SABER_OK) st = size_plan(q);
+  if (st == SABER_OK) st = alloc_query(q);
+  if (st != SABER_OK) {
+    g_last_error = q->err;
+    saber_query_destroy(q);
+    return st;
+  }
+  *out = q;
+  return SABER_OK;
+}
+
+void saber_query_destroy(saber_query *q) {
+  if (!q) return;
+  cudaSetDevice(q->device);
+  if (q->cs) cudaStreamSynchronize(q->cs);
+  if (q->h2d) cudaStreamSynchronize(q->h2d);
+  for (auto &s : q->slots) {
+    cudaFree(s.dev.rows); cudaFree(s.dev.hdr); cudaFree(s.dev.counts); cudaFree(s.dev.meta);
+    cudaFreeHost(s.h_meta); cudaFreeHost(s.h_rows); cudaFreeHost(s.h_hdr);
+    if (s.done) cudaEventDestroy(s.done);
+  }
+  for (auto &g : q->stages) {
+    cudaFreeHost(g.h); cudaFree(g.d);
+    if (g.free_ev) cudaEventDestroy(g.free_ev);
+  }
+  for (auto &r : q->registered) cudaHostUnregister(r.first);
+  cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
+  cudaFree(q->qd.carry[0]); cudaFree(q->qd.carry[1]); cudaFree(q->qd.tile_ctr); cudaFree(q->d_tmp);
+  if (q->cs) cudaStreamDestroy(q->cs);
+  if (q->h2d) cudaStreamDestroy(q->h2d);
+  if (q->d2h) cudaStreamDestroy(q->d2h);
+  cudaGetLastError();
+  delete q;
+}
+
+saber_status saber_task_submit_device(saber_query *q, const void *dev_tuples, size_t nbytes, void *cuda_stream) {
+  if (!q) return fail(nullptr, SABER_EINVAL, "null query");
+  std::lock_guard<std::mutex> lk(q->mu);
+  if (saber_status s = check_sticky(q)) return s;
+  if (q->closed) return fail(q, SABER_ECLOSED, "submit after finish");
+  const Plan &p = q->plan;
+  if (nbytes % p.tuple_bytes) return fail(q, SABER_EINVAL, "nbytes is not a multiple of tuple_bytes");
+  if (q->stage_fill) return fail(q, SABER_EINVAL, "device submit while host bytes of a partial task are staged");
+  const int64_t n = (int64_t)(nbytes / p.tuple_bytes);
+  if (n == 0) return SABER_OK;
+  if (((uintptr_t)dev_tuples) & 15) return fail(q, SABER_EINVAL, "device tuples must be 16-byte aligned");
+  const int64_t ntasks = (n + q->task_tuples - 1) / q->task_tuples;
+  if (ntasks > (int64_t)q->slots.size()) return fail(q, SABER_EINVAL, "submit at most result_slots * task_bytes per call");
+  if (ntasks > free_slots(q)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
+  CK(cudaSetDevice(q->device));
+  cudaStream_t us = (cudaStream_t)cuda_stream;
+  cudaEvent_t ev;
+  CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+  CK(cudaEventRecord(ev, us));
+  CK(cudaStreamWaitEvent(q->cs, ev, 0));
+  for (int64_t t = 0; t < ntasks; ++t) {
+    const int64_t off = t * q->task_tuples;
+    const int64_t cnt = std::min(q->task_tuples, n - off);
+    saber_status s = enqueue_task(q, (const unsigned char *)dev_tuples + off * p.tuple_bytes, cnt, 0, 0, 0);
+    if (s) { cudaEventDestroy(ev); return s; }
+  }
+  CK(cudaEventRecord(ev, q->cs));
+  CK(cudaStreamWaitEvent(us, ev, 0));
+  CK(cudaEventDestroy(ev));
+  return SABER_OK;
+}
+
+static bool is_registered(saber_query *q, const void *p, size_t n) {
+  for (auto &r : q->registered)
+    if ((const char *)p >= (const char *)r.first && (const char *)p + n <= (const char *)r.first + r.second) return true;
+  return false;
+}
+
+static saber_status ensure_stages(saber_query *q) {
+  if (!q->stages.empty()) return SABER_OK;
+  q->stages.resize(q->cfg.pipeline_depth);
+  const size_t tb = (size_t)q->task_tuples * q->plan.tuple_bytes;
+  for (auto &g : q->stages) {
+    CK(cudaMallocHost(&g.h, tb));
+    CK(cudaMalloc(&g.d, tb));
+    CK(cudaEventCreateWithFlags(&g.free_ev, cudaEventDisableTiming));
+  }
+  return SABER_OK;
+}
+
+// H2D of one task from pinned memory `src` into stage g, then the task itself
+static saber_status dispatch_host_task(saber_query *q, Stage &g, const void *src, int64_t ntuples, int final_,
+                                       int has_wm, int64_t wm) {
+  const size_t bytes = (size_t)ntuples * q->plan.tuple_bytes;
+  if (bytes) {
+    CK(cudaMemcpyAsync(g.d, src, bytes, cudaMemcpyHostToDevice, q->h2d));
+    cudaEvent_t ev;
+    CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    CK(cudaEventRecord(ev, q->h2d));
+    CK(cudaStreamWaitEvent(q->cs, ev, 0));
+    CK(cudaEventDestroy(ev));
+  }
+  saber_status s = enqueue_task(q, g.d, ntuples, final_, has_wm, wm);
+  if (s) return s;
+  CK(cudaEventRecord(g.free_ev, q->cs));   // stage reusable once the task's kernels are done
+  // the H2D copy of the next task may start now; the copy stream waits for the stage to be free
+  g.used = true;
+  return SABER_OK;
+}
+
+saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t nbytes) {
+  if (!q) return fail(nullptr, SABER_EINVAL, "null query");
+  std::lock_guard<std::mutex> lk(q->mu);
+  if (saber_status s = check_sticky(q)) return s;
+  if (q->closed) return fail(q, SABER_ECLOSED, "submit after finish");
+  const Plan &p = q->plan;
+  if (nbytes % p.tuple_bytes) return fail(q, SABER_EINVAL, "nbytes is not a multiple of tuple_bytes");
+  if (nbytes == 0) return SABER_OK;
+  if (saber_status s = ensure_stages(q)) return s;
+  CK(cudaSetDevice(q->device));
+  const int64_t tbytes = q->task_tuples * p.tuple_bytes;
+  const int64_t whole = ((int64_t)nbytes + q->stage_fill) / tbytes;
+  if (whole > free_slots(q)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
+  const bool reg = is_registered(q, host_tuples, nbytes);
+  const unsigned char *src = (const unsigned char *)host_tuples;
+  int64_t left = (int64_t)nbytes;
+  cudaEvent_t last_h2d = nullptr;
+  while (left > 0) {
+    Stage &g = q->stages[q->cur_stage];
+    if (q->stage_fill == 0 && g.used) CK(cudaEventSynchronize(g.free_ev));
+    if (reg && q->stage_fill == 0 && left >= tbytes) {
+      // registered caller memory: DMA straight from it (no copyin stage)
+      CK(cudaStreamWaitEvent(q->h2d, g.free_ev, 0));
+      saber_status s = dispatch_host_task(q, g, src, q->task_tuples, 0, 0, 0);
+      if (s) return s;
+      if (!last_h2d) CK(cudaEventCreateWithFlags(&last_h2d, cudaEventDisableTiming));
+      CK(cudaEventRecord(last_h2d, q->h2d));
+      src += tbytes; left -= tbytes;
+      q->cur_stage = (q->cur_stage + 1) % (int)q->stages.size();
+      continue;
+    }
+    const int64_t take = std::min(left, tbytes - q->stage_fill);
+    std::memcpy(g.h + q->stage_fill, src, (size_t)take);   // copyin (pageable → pinned)
+    q->stage_fill += take; src += take; left -= take;
+    if (q->stage_fill == tbytes) {
+      saber_status s = dispatch_host_task(q, g, g.h, q->task_tuples, 0, 0, 0);
+      if (s) return s;
+      q->stage_fill = 0;
+      q->cur_stage = (q->cur_stage + 1) % (int)q->stages.size();
+    }
+  }
+  if (last_h2d) {
+    CK(cudaEventSynchronize(last_h2d));   // the caller's registered bytes are free again
+    CK(cudaEventDestroy(last_h2d));
+  }
+  return SABER_OK;
+}
+
+saber_status saber_register_host(saber_query *q, void *ptr, size_t nbytes) {
+  if (!q || !ptr || !nbytes) return fail(q, SABER_EINVAL, "register_host arguments");
+  std::lock_guard<std::mutex> lk(q->mu);
+  CK(cudaSetDevice(q->device));
+  cudaError_t e = cudaHostRegister(ptr, nbytes, cudaHostRegisterDefault);
+  if (e == cudaErrorHostMemoryAlreadyRegistered) { cudaGetLastError(); return SABER_OK; }
+  if (e != cudaSuccess) return fail(q, SABER_ECUDA, std::string("cudaHostRegister: ") + cudaGetErrorString(e));
+  q->registered.emplace_back(ptr, nbytes);
+  return SABER_OK;
+}
+
+saber_status saber_query_finish(saber_query *q, int64_t watermark) {
+  if (!q) return fail(nullptr, SABER_EINVAL, "null query");
+  std::lock_guard<std::mutex> lk(q->mu);
+  if (saber_status s = check_sticky(q)) return s;
+  if (q->closed) return fail(q, SABER_ECLOSED, "finish called twice");
+  CK(cudaSetDevice(q->device));
+  const int need = 1 + (q->stage_fill > 0);
+  if (free_slots(q) < need) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
+  const int has_wm = watermark != INT64_MIN;
+  if (q->stage_fill > 0) {
+    Stage &g = q->stages[q->cur_stage];
+    saber_status s = dispatch_host_task(q, g, g.h, q->stage_fill / q->plan.tuple_bytes, 0, 0, 0);
+    if (s) return s;
+    q->stage_fill = 0;
+    q->cur_stage = (q->cur_stage + 1) % (int)q->stages.size();
+  }
+  saber_status s = enqueue_task(q, nullptr, 0, 1, has_wm, watermark);
+  if (s) return s;
+  q->closed = true;
+  return SABER_OK;
+}
+
+saber_status saber_results_poll(saber_query *q, saber_results *out, int32_t timeout_us) {
+  if (!q || !out) return fail(q, SABER_EINVAL, "poll arguments");
+  std::lock_guard<std::mutex> lk(q->mu);
+  std::memset(out, 0, sizeof(*out));
+  if (q->next_poll >= q->next_task) return fail(q, SABER_EAGAIN, "no pending task");
+  Slot &s = q->slots[q->next_poll % (int64_t)q->slots.size()];
+  if (s.state != SLOT_BUSY || s.task_id != q->next_poll) return fail(q, SABER_EINVAL, "result ring out of order");
+  CK(cudaSetDevice(q->device));
+  if (timeout_us < 0) {
+    CK(cudaEventSynchronize(s.done));
+  } else {
+    auto t0 = std::chrono::steady_clock::now();
+    for (;;) {
+      cudaError_t e = cudaEventQuery(s.done);
+      if (e == cudaSuccess) break;
+      if (e != cudaErrorNotReady) CK(e);
+      cudaGetLastError();
+      auto us = std::chrono::duration_cast<std::chrono::microseconds>(std::chrono::steady_clock::now() - t0).count();
+      if (us >= timeout_us) return fail(q, SABER_EAGAIN, "poll timeout");
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+    }
+  }
+  s.meta = *s.h_meta;
+  const Plan &p = q->plan;
+  if (s.meta.error) {
+    q->sticky = status_from_err(s.meta.error);
+    return fail(q, q->sticky, err_text(s.meta.error));
+  }
+  out->task_id = s.task_id;
+  out->first_window = s.meta.first_window;
+  out->nwindows = s.meta.nwindows;
+  out->nrows = s.meta.nrows;
+  out->ntuples = s.meta.ntuples;
+  const bool host = q->cfg.result_mode == SABER_RESULTS_HOST;
+  out->on_device = !host;
+  if (p.nagg > 0) {
+    out->ncols = p.ncols;
+    for (int c = 0; c < p.ncols; ++c) out->col_bytes[c] = p.col_bytes[c];
+    if (host) {
+      if (s.meta.nwindows)
+        CK(cudaMemcpyAsync(s.h_hdr, s.dev.hdr, (size_t)s.meta.nwindows * sizeof(saber_win_hdr), cudaMemcpyDeviceToHost, q->d2h));
+      for (int c = 0; c < p.ncols && s.meta.nrows; ++c)
+        CK(cudaMemcpyAsync(s.h_rows + p.col_off[c], s.dev.rows + p.col_off[c], (size_t)s.meta.nrows * p.col_bytes[c],
+                           cudaMemcpyDeviceToHost, q->d2h));
+      CK(cudaStreamSynchronize(q->d2h));
+    }
+    unsigned char *rows = host ? s.h_rows : s.dev.rows;
+    out->hdr = host ? s.h_hdr : (const saber_win_hdr *)s.dev.hdr;
+    for (int c = 0; c < p.ncols; ++c) out->cols[c] = rows + p.col_off[c];
+  } else {
+    out->tuple_bytes = p.out_row_words * 4;
+    if (host && s.meta.ntuples) {
+      CK(cudaMemcpyAsync(s.h_rows, s.dev.rows, (size_t)s.meta.ntuples * out->tuple_bytes, cudaMemcpyDeviceToHost, q->d2h));
+      CK(cudaStreamSynchronize(q->d2h));
+    }
+    out->tuples = host ? (const void *)s.h_rows : (const void *)s.dev.rows;
+    out->hdr = nullptr;
+  }
+  q->stats.windows += s.meta.nwindows;
+  q->stats.rows += s.meta.nrows;
+  q->stats.out_tuples += s.meta.ntuples;
+  s.state = SLOT_POLLED;
+  q->next_poll++;
+  return SABER_OK;
+}
+
+saber_status saber_results_release(saber_query *q, const saber_results *r) {
+  if (!q || !r) return fail(q, SABER_EINVAL, "release arguments");
+  std::lock_guard<std::mutex> lk(q->mu);
+  Slot &s = q->slots[r->task_id % (int64_t)q->slots.size()];
+  if (s.task_id != r->task_id || s.state != SLOT_POLLED) return fail(q, SABER_EINVAL, "slice not polled or released twice");
+  s.state = SLOT_FREE;
+  return SABER_OK;
+}
+
+saber_status saber_query_stats(const saber_query *q, saber_stats *out) {
+  if (!q || !out) return SABER_EINVAL;
+  *out = q->stats;
+  out->tasks_pending = q->next_task - q->next_poll;
+  return SABER_OK;
+}
+
+saber_status saber_query_sync(saber_query *q) {
+  if (!q) return SABER_EINVAL;
+  CK(cudaSetDevice(q->device));
+  CK(cudaStreamSynchronize(q->cs));
+  return SABER_OK;
+}
+
+saber_status saber_partition_plan(const saber_schema *schema, const saber_window *window, const void *dev_tuples,
+                                  int64_t begin, int64_t n, int64_t *closed_windows, int64_t *halo_first) {
+  saber_query *q = nullptr;
+  if (!schema || !window || !closed_windows || !halo_first || n < 0 || begin < 0)
+    return fail(nullptr, SABER_EINVAL, "partition_plan arguments");
+  if (window->size < 1 || window->slide < 1 || window->slide > window->size)
+    return fail(nullptr, SABER_EINVAL, "window");
+  if (schema->ts_col < 0 || schema->ts_col >= schema->ncols) return fail(nullptr, SABER_EINVAL, "ts_col");
+  const int ts_word = schema->offsets[schema->ts_col] / 4;
+  if (window->kind == SABER_WIN_COUNT) {
+    int64_t total = begin + n;
+    *closed_windows = total >= window->size ? (total - window->size) / window->slide + 1 : 0;
+    *halo_first = *closed_windows * window->slide;
+    return SABER_OK;
+  }
+  if (n == 0) { *closed_windows = 0; *halo_first = begin; return SABER_OK; }
+  if (!dev_tuples) return fail(nullptr, SABER_EINVAL, "time windows need the partition's tuples");
+  int64_t *d = nullptr;
+  CK(cudaMalloc(&d, 16));
+  CK(launch_partition_plan(ts_word, schema->tuple_bytes / 4, 1, window->size, window->slide, window->origin,
+                           dev_tuples, begin, n, d, 0));
+  int64_t h[2];
+  CK(cudaMemcpy(h, d, 16, cudaMemcpyDeviceToHost));
+  cudaFree(d);
+  if (h[0] < 0) return fail(nullptr, SABER_EINVAL, "partition is shorter than the window span");
+  *closed_windows = h[0];
+  *halo_first = h[1];
+  return SABER_OK;
+}
+
+}  // extern "C"

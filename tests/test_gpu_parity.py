@@ -1,0 +1,268 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by
+element on the same seeded inputs (run with -m gpu on a B200)."""
+import numpy as np
+import pytest
+
+from parity import compare
+from saber_inputs import gen, workloads
+from tiny import TINY, golden, spec as tspec, stream
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def saber():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_sigmod_koliousiswfwcp16_b200 import saber as S
+    return S
+
+
+def run_product(S, spec, data, task_bytes=1 << 20, watermark=None, chunk_bytes=None, **kw):
+    q = S.Query(spec, task_bytes=task_bytes, **kw)
+    try:
+        return q.run(data, chunk_bytes=chunk_bytes, watermark=watermark)
+    finally:
+        q.close()
+
+
+def check(S, oracle_lib, spec, data, watermark=None, **kw):
+    exp = oracle_lib.run(spec, data, watermark=watermark, nthreads=8)
+    got = run_product(S, spec, data, watermark=watermark, **kw)
+    compare(spec, got, exp)
+    return got, exp
+
+
+# ------------------------------------------------------------------ goldens --
+@pytest.mark.parametrize("gid", ["G1", "G2", "G3"])
+@pytest.mark.parametrize("task_tuples", [1, 3, 5, 64])
+def test_golden_count(saber, oracle_lib, gid, task_tuples):
+    g = golden(gid)
+    sp = tspec(g["window"], aggs=[("sum", "v"), ("count", None), ("min", "v"), ("max", "x")])
+    got, _ = check(saber, oracle_lib, sp, stream(v=g["tuples_v"], x=np.arange(10) / 4.0),
+                   task_bytes=32 * task_tuples)
+    assert list(got["vals"][0]) == g["expect_sum"]
+
+
+def test_golden_fragment_classes(saber):
+    """Fig. 2 prose (L508-517): per-task window-fragment classes for 5-tuple tasks."""
+    for gid in ("G1", "G2"):
+        g = golden(gid)
+        sp = tspec(g["window"], aggs=[("sum", "v")])
+        q = saber.Query(sp, task_bytes=32 * g["task_tuples"])
+        d = stream(v=g["tuples_v"])
+        for t, cls in enumerate(g["expect_task_classes"]):
+            assert q.submit(d[t * 160:(t + 1) * 160]) == 0
+            st = q.stats()
+            assert (st["last_complete"], st["last_opening"], st["last_closing"], st["last_pending"]) == \
+                (len(cls["complete"]), len(cls["opening"]), len(cls["closing"]), len(cls["pending"])), (gid, t)
+        q.close()
+
+
+@pytest.mark.parametrize("task_tuples", [1, 2, 4, 10])
+def test_golden_time(saber, oracle_lib, task_tuples):
+    g = golden("G4")
+    d = stream(v=g["tuples_v"], tau=g["tau"])
+    for w in ({"kind": "time", "size": 3, "slide": 1}, {"kind": "time", "size": 1, "slide": 1},
+              {"kind": "time", "size": 2, "slide": 2}):
+        sp = tspec(w, aggs=[("count", None), ("sum", "v")])
+        check(saber, oracle_lib, sp, d, task_bytes=32 * task_tuples)
+
+
+def test_golden_groupby_having_istream(saber, oracle_lib):
+    g6 = golden("G6")
+    d = stream(x=g6["x"], k=g6["key"])
+    for dom in (0, 3):
+        sp = tspec(g6["window"], aggs=[("sum", "x"), ("count", None), ("avg", "x")], group_by=[("k", 1, dom)])
+        check(saber, oracle_lib, sp, d, task_bytes=64)
+        sp = tspec(g6["window"], aggs=[("avg", "x")], group_by=[("k", 1, dom)], having=[(0, "<", 1.0)])
+        check(saber, oracle_lib, sp, d, task_bytes=96)
+    g7 = golden("G7")
+    sp = tspec(g7["window"], where=[("o", "==", 1)], project=["v"])
+    got, _ = check(saber, oracle_lib, sp, stream(v=g7["tuples_v"]), task_bytes=64)
+    assert list(np.frombuffer(got["tuples"], np.int32)) == g7["expect_v"]
+
+
+# -------------------------------------------------------------- configs -------
+@pytest.mark.parametrize("fn", ["sum", "count", "avg", "min", "max"])
+def test_c1_full_size(saber, oracle_lib, fn):
+    """configs[0] at its full size (1M tuples), one task and many tasks."""
+    spec, g = workloads.c1(fn)
+    data = gen.generate("syn", g["n"], g["seed"], rate=g["rate"], groups=g["groups"])
+    check(saber, oracle_lib, spec, data, task_bytes=32 << 20)
+    check(saber, oracle_lib, spec, data, task_bytes=(1 << 20) + 4096)
+
+
+@pytest.mark.parametrize("sel", [0.0, 0.01, 0.5, 1.0])
+def test_c2_select_project(saber, oracle_lib, sel):
+    spec, g = workloads.c2(sel=sel, npred=4 if sel == 0.5 else 1)
+    n = 1 << 20
+    data = gen.generate("syn", n, g["seed"], rate=1)
+    check(saber, oracle_lib, spec, data, task_bytes=(4 << 20) + 32 * 77)
+
+
+@pytest.mark.parametrize("groups,dom", [(64, True), (64, False), (1024, True), (16384, True), (65536, False)])
+def test_c3_groupby(saber, oracle_lib, groups, dom):
+    spec, g = workloads.c3(groups=groups, declare_domain=dom)
+    n = 1 << 19
+    data = gen.generate("syn", n, g["seed"], rate=1, groups=groups)
+    check(saber, oracle_lib, spec, data, task_bytes=(4 << 20))
+
+
+@pytest.mark.parametrize("rate", [64, 4096])
+def test_c4_cm1(saber, oracle_lib, rate):
+    spec, g = workloads.c4(rate=rate)
+    n = 1 << 18
+    data = gen.generate("cm", n, g["seed"], rate=rate, groups=g["groups"])
+    check(saber, oracle_lib, spec, data, task_bytes=(2 << 20))
+
+
+def test_c5a_sg2_and_sg1(saber, oracle_lib):
+    for spec, g in (workloads.c5a(), workloads.sg1()):
+        spec["window"]["size"] = 60          # shorter window so the oracle stays fast
+        n = 1 << 19
+        data = gen.generate("sg", n, g["seed"], rate=1024)
+        check(saber, oracle_lib, spec, data, task_bytes=(2 << 20))
+
+
+def test_c5b_lrb3(saber, oracle_lib):
+    spec, g = workloads.c5b()
+    spec["window"]["size"] = 30
+    n = 1 << 19
+    data = gen.generate("lrb", n, g["seed"], rate=2048)
+    check(saber, oracle_lib, spec, data, task_bytes=(2 << 20))
+
+
+def test_cm2_int64_key_hash(saber, oracle_lib):
+    spec, g = workloads.cm2(rate=64)
+    n = 1 << 17
+    data = gen.generate("cm", n, g["seed"], rate=64, groups=4)
+    check(saber, oracle_lib, spec, data, task_bytes=(1 << 20))
+
+
+# ----------------------------------------------------- random small streams --
+def _random_case(rng):
+    n = int(rng.integers(0, 3000))
+    s = int(rng.integers(1, 200))
+    l = int(rng.integers(1, s + 1))
+    kind = "count" if rng.random() < 0.5 else "time"
+    tau = np.cumsum(rng.choice([0, 0, 1, 1, 2, 5], size=n)) if kind == "time" else np.arange(n)
+    v = rng.integers(-1000, 1000, size=n)
+    x = rng.integers(0, 1 << 12, size=n) / 64.0
+    k = rng.integers(0, int(rng.choice([1, 3, 17, 300])), size=n)
+    w = {"kind": kind, "size": s, "slide": l, "origin": int(rng.integers(0, 3)) if kind == "time" else 0}
+    where = [("v", "<", int(rng.integers(-500, 1000)))] if rng.random() < 0.4 else []
+    if rng.random() < 0.2:
+        sp = tspec(w, where=where, project=list(rng.choice(["ts", "v", "x", "k", "m"], size=int(rng.integers(1, 4)))))
+    else:
+        fns = ["sum", "count", "avg", "min", "max"]
+        aggs = []
+        for _ in range(int(rng.integers(1, 4))):
+            fn = str(rng.choice(fns))
+            aggs.append((fn, None) if fn == "count" else (fn, str(rng.choice(["v", "x"]))))
+        gb = []
+        r = rng.random()
+        if r < 0.35:
+            gb = [("k", 1, 300 if rng.random() < 0.5 else 0)]
+        elif r < 0.5:
+            gb = [("k", 1, 0), ("v", 7, 0)]
+        elif r < 0.6:
+            gb = [("k", 1, 300), ("o", 1, 2)]
+        having = [(0, ">=", 0.0)] if rng.random() < 0.2 else []
+        sp = tspec(w, where=where, aggs=aggs, group_by=gb, having=having)
+    return sp, stream(v=v, tau=tau, x=x, k=k, n=n)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_streams(saber, oracle_lib, seed):
+    rng = np.random.default_rng(77 + seed)
+    for _ in range(12):
+        sp, d = _random_case(rng)
+        tt = int(rng.choice([1, 7, 100, 1000, 5000]))
+        wm = None
+        if sp["window"]["kind"] == "time" and rng.random() < 0.3 and len(d):
+            wm = int(np.frombuffer(d, np.int64).reshape(-1, 4)[-1, 0] + rng.integers(0, 50))
+        chunk = int(rng.choice([32, 32 * 13, 32 * 1000])) if rng.random() < 0.5 else None
+        check(saber, oracle_lib, sp, d, watermark=wm, task_bytes=32 * tt, chunk_bytes=chunk)
+
+
+# --------------------------------------------------------------- invariants --
+def test_task_size_invariance(saber, oracle_lib):
+    """A22 / Fig. 13: results do not depend on the task size φ (ints bit-exact)."""
+    spec, g = workloads.c3(groups=256)
+    spec["aggs"] = [("count", None), ("sum", "a3"), ("max", "a1"), ("avg", "a1")]
+    spec["window"] = workloads.count_window(4096, 512)
+    data = gen.generate("syn", 1 << 18, 9, groups=256)
+    exp = oracle_lib.run(spec, data, nthreads=8)
+    for tb in (32 * 999, 1 << 20, 3 << 20, 8 << 20):
+        compare(spec, run_product(saber, spec, data, task_bytes=tb), exp)
+
+
+def test_device_submit_matches_host(saber, oracle_lib):
+    import torch
+    spec, g = workloads.c4(rate=64)
+    n = 1 << 17
+    data = gen.generate("cm", n, g["seed"], rate=64, groups=4)
+    exp = oracle_lib.run(spec, data, nthreads=8)
+    dev = torch.from_numpy(np.frombuffer(data, np.uint8).copy()).cuda()
+    q = saber.Query(spec, task_bytes=1 << 20)
+    slices = []
+    off, tb = 0, 1 << 20
+    while off < dev.numel():
+        nb = min(tb * 2, dev.numel() - off)
+        st = q.submit_device(dev.data_ptr() + off, nb, torch.cuda.current_stream().cuda_stream)
+        if st == saber.EAGAIN:
+            slices.append(q.poll())
+            continue
+        assert st == 0, q.last_error()
+        off += nb
+    assert q.finish() == 0
+    while (s := q.poll()) is not None:
+        slices.append(s)
+    compare(spec, saber.merge_slices(slices, q.m), exp)
+    q.close()
+
+
+# ------------------------------------------------------------------- errors --
+def test_errors_are_sticky(saber):
+    sp = tspec({"kind": "time", "size": 2, "slide": 1}, aggs=[("count", None)])
+    q = saber.Query(sp, task_bytes=32 * 4)
+    q.submit(stream(tau=[0, 1, 2, 1, 3, 4, 5, 6]))
+    q.finish()
+    with pytest.raises(saber.SaberError) as e:
+        while q.poll() is not None:
+            pass
+    assert e.value.status == saber.EORDER
+    q.close()
+    sp = tspec({"kind": "count", "size": 2, "slide": 1}, aggs=[("count", None)], group_by=[("k", 1, 2)])
+    q = saber.Query(sp, task_bytes=32 * 4)
+    q.submit(stream(k=[0, 1, 5, 1]))
+    q.finish()
+    with pytest.raises(saber.SaberError) as e:
+        while q.poll() is not None:
+            pass
+    assert e.value.status == saber.EKEY
+    q.close()
+
+
+def test_invalid_queries_rejected(saber):
+    with pytest.raises(saber.SaberError) as e:
+        saber.Query(tspec({"kind": "count", "size": 2, "slide": 3}, aggs=[("count", None)]))
+    assert e.value.status == saber.EINVAL
+    with pytest.raises(saber.SaberError):
+        saber.Query(tspec({"kind": "count", "size": 2, "slide": 1}, aggs=[("sum", "x")], group_by=[("x", 1, 0)]))
+
+
+def test_device_generator_matches_numpy(saber):
+    import ctypes as C
+    import os
+    import torch
+    L = C.CDLL(os.path.join(os.path.dirname(gen.__file__), "libsaber_gen.so"))
+    for kind, tb in (("syn", 32), ("cm", 64), ("sg", 32), ("lrb", 32)):
+        n, i0 = 5000, 123456789
+        buf = torch.empty(n * tb, dtype=torch.uint8, device="cuda")
+        L.saber_gen(gen.KIND_ID[kind], C.c_uint64(7), C.c_int64(i0), C.c_int64(n), C.c_int64(3), C.c_int64(64),
+                    C.c_void_p(buf.data_ptr()), None)
+        torch.cuda.synchronize()
+        assert buf.cpu().numpy().tobytes() == gen.generate(kind, n, 7, i0=i0, rate=3, groups=64), kind
