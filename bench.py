@@ -1,0 +1,439 @@
+#!/usr/bin/env python
+"""Benchmark: one windowed query over a synthetic stream on 1..8 B200s.
+
+Default workload (BASELINE.json configs[2], SURVEY.md §8 "C3"): Syn 32-byte
+tuples, ``SELECT AVG(a1) FROM Syn [ROWS 32768 SLIDE 1024] GROUP BY a2`` with
+G = 64 groups, 2^28 tuples (8 GiB) per GPU.  A step is one pass of the whole
+hot path -- task dispatch, K1 boundary/pane assignment + σ + pane partial
+aggregation, window assembly and the result stage -- over the GPU's stream
+partition (plus the halo exchange when N > 1).  Multi-GPU is weak scaling:
+rank r owns tuples [r·2^28, (r+1)·2^28) of one global stream of N·2^28 tuples
+and emits the windows closed inside its partition; only the halo (< s tuples)
+crosses NVLink, once per step.
+
+``value``  tuples/s, device-resident (inputs already in HBM), whole job / max rank time
+``e2e``    the same metric through the C ABI from pinned HOST buffers, H2D of the
+           inputs and D2H of every result slice inside the timed region
+``--impl reference``  the CPU oracle (oracle/) timed on this host's cores on a
+           bounded sample of the same workload (the reference arm of this tier)
+"""
+from __future__ import annotations
+
+import argparse
+import ctypes as C
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from saber_inputs import gen, workloads  # noqa: E402
+
+METRIC = "tuples/s & GB/s per windowed query at 1/2/4/8 B200; % of HBM roofline"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="saber", choices=["saber", "reference"])
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "C5a", "C5b", "SG1"])
+    ap.add_argument("--groups", type=int, default=64)
+    ap.add_argument("--sel", type=float, default=0.5)
+    ap.add_argument("--rate", type=int, default=0)
+    ap.add_argument("--tuples-log2", type=int, default=0, help="tuples per GPU (default: the config's)")
+    ap.add_argument("--task-mb", type=int, default=256)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    return ap.parse_args()
+
+
+def workload(args):
+    c = args.config
+    if c == "C1":
+        spec, g = workloads.c1()
+    elif c == "C2":
+        spec, g = workloads.c2(sel=args.sel)
+    elif c == "C3":
+        spec, g = workloads.c3(groups=args.groups)
+    elif c == "C4":
+        spec, g = workloads.c4(rate=args.rate or 64)
+    elif c == "C5a":
+        spec, g = workloads.c5a(rate=args.rate or 4096)
+    elif c == "C5b":
+        spec, g = workloads.c5b(rate=args.rate or 8192)
+    else:
+        spec, g = workloads.sg1(rate=args.rate or 4096)
+    if args.tuples_log2:
+        g["n"] = 1 << args.tuples_log2
+    w = spec["window"]
+    desc = {
+        "C1": "Syn 32-B, SUM(a1), count w(1024,1024)",
+        "C2": f"Syn 32-B, SELECT ts,a1,a2 WHERE a3<sel*2^31 (sel={args.sel}), count w(1024,64), IStream",
+        "C3": f"Syn 32-B, AVG(a1) GROUP BY a2 (G={args.groups}), count w(32768,1024)",
+        "C4": f"CM 64-B, SUM(cpu) GROUP BY category, time w(60,1), R={g['rate']}/s",
+        "C5a": f"SG 32-B, AVG(value) GROUP BY plug,household,house, time w(3600,1), R={g['rate']}/s",
+        "C5b": f"LRB 32-B, AVG(speed) GROUP BY highway,direction,position/5280 HAVING avg<40, time w(300,1), R={g['rate']}/s",
+        "SG1": f"SG 32-B, AVG(value), time w(3600,1), R={g['rate']}/s",
+    }[c]
+    name = f"{c}: {desc}, 2^{int(np.log2(g['n']))} tuples ({g['n'] * spec['schema']['tuple_bytes'] >> 20} MiB) per GPU"
+    return spec, g, name, w
+
+
+# --------------------------------------------------------------------------- utils
+class Clocks:
+    """nvidia-smi sampling during the timed region (the recipe's clocks line)."""
+
+    def __init__(self, index, path):
+        self.path = path
+        self.proc = None
+        self.index = index
+
+    def __enter__(self):
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=index,clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            self.f.close()
+
+    def summary(self):
+        try:
+            rows = [r.split(", ") for r in open(self.path).read().strip().splitlines() if r.strip()]
+        except Exception:
+            rows = []
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if len(r) > 5 + i and r[5 + i].strip() == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic(config_key):
+    """Per-launch DRAM bytes of the dominant kernel from a committed ncu --set full capture."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get(config_key)
+    except Exception:
+        return None
+
+
+def gen_device(lib_gen, kind, seed, i0, n, rate, groups, out, stream):
+    rc = lib_gen.saber_gen(gen.KIND_ID[kind], C.c_uint64(seed), C.c_int64(i0), C.c_int64(n), C.c_int64(rate),
+                           C.c_int64(groups), C.c_void_p(out.data_ptr()), C.c_void_p(stream))
+    assert rc == 0, rc
+
+
+# --------------------------------------------------------------------------- reference arm
+def cpu_oracle_sample(spec, g, budget_s, threads):
+    """Time the oracle (as it stands) on a bounded prefix of the same workload.
+    Returns (tuples/s of stream covered, sample description)."""
+    import oracle
+    oracle.build()
+    w = spec["window"]
+    tb = spec["schema"]["tuple_bytes"]
+    rate = g.get("rate", 1)
+    unit = w["slide"] if w["kind"] == "count" else w["slide"] * rate     # tuples per window step
+
+    def run(nw):
+        if w["kind"] == "count":
+            ntup = (nw - 1) * w["slide"] + w["size"]
+        else:
+            ntup = ((nw - 1) * w["slide"] + w["size"] + 1) * rate
+        data = gen.generate(g["kind"], ntup, g["seed"], rate=rate, groups=g["groups"])
+        t0 = time.perf_counter()
+        r = oracle.run(spec, data, windows=list(range(nw)), nthreads=threads)
+        dt = time.perf_counter() - t0
+        assert len(r["win_id"]) == nw
+        return dt, ntup
+
+    nw = 16
+    dt, _ = run(nw)
+    while dt < 0.5 and nw < (1 << 22):
+        nw *= 4
+        dt, _ = run(nw)
+    nw = max(16, int(nw * budget_s / max(dt, 1e-3)))
+    dt, ntup = run(nw)
+    value = nw * unit / dt
+    sample = (f"first {nw} windows of the workload's stream ({ntup} tuples read, {nw * unit} tuples of stream "
+              f"advanced), oracle recomputes every window from scratch; value = stream tuples advanced / wall s")
+    return value, sample, dt
+
+
+def run_reference(args, spec, g, name, rank, world):
+    if rank != 0:
+        return
+    threads = len(os.sched_getaffinity(0))
+    vals = []
+    for i in range(args.warmup + args.steps):
+        v, sample, dt = cpu_oracle_sample(spec, g, max(2.0, args.cpu_seconds / max(1, args.steps)), threads)
+        if i >= args.warmup:
+            vals.append(v)
+    value = statistics.median(vals)
+    line = {"metric": METRIC, "value": value, "unit": "tuples/s", "impl": "reference", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": None, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": name, "groups": args.groups},
+            "cpu_baseline": {"value": value, "unit": "tuples/s", "cores": threads, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": "tuples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------------------- product arm
+def main():
+    args = parse()
+    spec, g, name, w = workload(args)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    import torch
+    import torch.distributed as dist
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.impl == "reference":
+        run_reference(args, spec, g, name, rank, world)
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    from paper_conf_sigmod_koliousiswfwcp16_b200 import saber
+    from paper_conf_sigmod_koliousiswfwcp16_b200.parallel import exchange_halo
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    lib_gen = C.CDLL(os.path.join(ROOT, "saber_inputs", "libsaber_gen.so"))
+    tb = spec["schema"]["tuple_bytes"]
+    n = g["n"]                                   # tuples per GPU (weak scaling)
+    begin = rank * n
+    part = torch.empty(n * tb, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+    gen_device(lib_gen, g["kind"], g["seed"], begin, n, g["rate"], g["groups"], part, stream.cuda_stream)
+    torch.cuda.synchronize()
+    task_bytes = args.task_mb << 20
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def drive(q, pieces, s):
+        """Submit device pieces (ptr, nbytes) in task-sized chunks; poll+release
+        whenever all result slots are busy.  Returns (windows, rows, tuples out)."""
+        nw = nr = nt = 0
+
+        def drain_one():
+            nonlocal nw, nr, nt
+            st, r = q.poll_raw(-1)
+            if st != 0:
+                raise saber.SaberError(st, q.last_error())
+            nw += r.nwindows; nr += r.nrows; nt += r.ntuples
+            q.release(r)
+        for ptr, nbytes in pieces:
+            off = 0
+            while off < nbytes:
+                nb = min(task_bytes, nbytes - off)
+                st = q.submit_device(ptr + off, nb, s)
+                if st == saber.EAGAIN:
+                    drain_one()
+                    continue
+                if st != 0:
+                    raise saber.SaberError(st, q.last_error())
+                off += nb
+        while (st := q.finish()) == saber.EAGAIN:
+            drain_one()
+        if st != 0:
+            raise saber.SaberError(st, q.last_error())
+        q.record(s)
+        return drain_one, (lambda: (nw, nr, nt))
+
+    # ---------------- device-resident timed loop
+    # partition planning metadata (first window / base index) is fixed by the data;
+    # the query objects are created outside the timed region, the halo bytes are
+    # exchanged inside it every step.
+    if world > 1:
+        _, first_window, base_index = exchange_halo(spec, part, begin, n, rank, world)
+    else:
+        first_window, base_index = 0, begin
+    times, stats_acc = [], []
+    out_rows = out_tuples = out_windows = 0
+    clk_dir = os.path.join(ROOT, "gpurun_out") if os.path.isdir(os.path.join(ROOT, "gpurun_out")) else "/tmp"
+    with Clocks(local, os.path.join(clk_dir, f"clocks_rank{rank}.csv")) as clk:
+        for it in range(args.warmup + args.steps):
+            q = saber.Query(spec, base_index=base_index, first_window=first_window,
+                            emit_on_finish=(rank == world - 1), task_bytes=task_bytes,
+                            result_mode=saber.RESULTS_DEVICE, profile=True, result_slots=8, device=local)
+            barrier()
+            torch.cuda.synchronize()
+            ev0 = torch.cuda.Event(enable_timing=True)
+            ev1 = torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            pieces = []
+            if world > 1:
+                halo, fw, bi = exchange_halo(spec, part, begin, n, rank, world)
+                assert (fw, bi) == (first_window, base_index)
+                if halo.numel():
+                    pieces.append((halo.data_ptr(), halo.numel()))
+            pieces.append((part.data_ptr(), part.numel()))
+            drain_one, counts = drive(q, pieces, stream.cuda_stream)
+            ev1.record(stream)
+            while q.stats()["tasks_pending"] > 0:     # already complete once ev1 is
+                drain_one()
+            torch.cuda.synchronize()
+            ms = ev0.elapsed_time(ev1)
+            st = q.stats()
+            q.close()
+            if it >= args.warmup:
+                times.append(ms)
+                stats_acc.append(st)
+                out_windows, out_rows, out_tuples = counts()
+    clocks = clk.summary()
+    ms_rank = statistics.median(times)
+    print(f"[bench rank {rank}] device-resident step ms: {[round(t, 3) for t in times]}", file=sys.stderr)
+    ms_step = max_over_ranks(ms_rank)
+    total_tuples = n * world
+    value = total_tuples / (ms_step / 1e3)
+
+    # roofline of the dominant kernel (the fused K1+σ+pane-aggregation scan, or K1+K3 for σ/π)
+    scan_ms = sum(s["scan_ms"] for s in stats_acc)
+    scan_launches = sum(s["scan_launches"] for s in stats_acc)
+    launches = sum(s["kernel_launches"] for s in stats_acc)
+    bytes_scanned = sum(s["bytes_in"] for s in stats_acc)        # 1 x 32-B sector per 32-B tuple read
+    peak, peak_src = measured_peaks()
+    per_launch_bytes = bytes_scanned / max(1, scan_launches)
+    per_launch_ms = scan_ms / max(1, scan_launches)
+    achieved = per_launch_bytes / (per_launch_ms / 1e3) / 1e9 if per_launch_ms > 0 else None
+    key = f"{args.config}_G{args.groups}" if args.config == "C3" else args.config
+    traffic = ncu_traffic(key)
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+                "kernel": "k_select" if not spec["aggs"] else "k_pane_agg",
+                "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,
+                "launches_per_step": scan_launches / max(1, len(stats_acc)), "peak_source": peak_src,
+                "share_of_step": (scan_ms / max(1, len(stats_acc))) / ms_rank if ms_rank else None}
+
+    # ---------------- end-to-end through the C ABI from pinned host memory
+    e2e = None
+    if not args.no_e2e:
+        host = torch.empty(n * tb, dtype=torch.uint8, pin_memory=True)
+        host.copy_(part)
+        torch.cuda.synchronize()
+        host_np = host.numpy()
+        e_times = []
+        d2h_bytes = 0
+        for it in range(args.warmup + min(args.steps, 3)):
+            q = saber.Query(spec, task_bytes=task_bytes, result_mode=saber.RESULTS_HOST, device=local,
+                            base_index=base_index, first_window=first_window, emit_on_finish=(rank == world - 1))
+            q.register_host(host_np)
+            barrier()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            halo_np = None
+            if world > 1:
+                halo, _, _ = exchange_halo(spec, part, begin, n, rank, world)
+                halo_np = halo.cpu().numpy() if halo.numel() else None
+            got_bytes = 0
+            chunks = []
+            if halo_np is not None:
+                chunks.append(halo_np)
+            chunks.append(host_np)
+            per = task_bytes * 7
+            for arr in chunks:
+                off = 0
+                while off < arr.size:
+                    part_np = arr[off:off + per]
+                    st = q.submit(part_np)
+                    if st == saber.EAGAIN:
+                        s = q.poll()
+                        got_bytes += sum(k.nbytes for k in s.keys) + sum(v.nbytes for v in s.vals) + \
+                            len(s.tuples) + s.nwindows * 32
+                        continue
+                    if st != 0:
+                        raise saber.SaberError(st, q.last_error())
+                    off += part_np.size
+            while (st := q.finish()) == saber.EAGAIN:
+                s = q.poll()
+                got_bytes += sum(k.nbytes for k in s.keys) + sum(v.nbytes for v in s.vals) + len(s.tuples) + s.nwindows * 32
+            while (s := q.poll()) is not None:
+                got_bytes += sum(k.nbytes for k in s.keys) + sum(v.nbytes for v in s.vals) + len(s.tuples) + s.nwindows * 32
+            torch.cuda.synchronize()
+            dt = time.perf_counter() - t0
+            q.close()
+            if it >= args.warmup:
+                e_times.append(dt)
+                d2h_bytes = got_bytes
+        e_s = max_over_ranks(statistics.median(e_times))
+        e2e = {"value": total_tuples / e_s, "unit": "tuples/s", "h2d_bytes_per_step": n * tb,
+               "d2h_bytes_per_step": d2h_bytes, "s_per_step": e_s,
+               "input_gbs": total_tuples * tb / e_s / 1e9}
+
+    # ---------------- CPU oracle baseline (rank 0, N = 1)
+    cpu = None
+    if not args.no_cpu and world == 1 and rank == 0:
+        threads = len(os.sched_getaffinity(0))
+        v, sample, dt = cpu_oracle_sample(spec, g, args.cpu_seconds, threads)
+        cpu = {"value": v, "unit": "tuples/s", "cores": threads, "kind": "oracle", "sample": sample,
+               "seconds": dt}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "tuples/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "input_gbs": total_tuples * tb / (ms_step / 1e3) / 1e9,
+                "config": {"workload": name, "groups": args.groups if args.config == "C3" else None,
+                           "task_bytes": task_bytes, "tuples_per_gpu": n,
+                           "l2": "inputs (>= 1 GiB per GPU) exceed the 126 MB L2: no flush needed",
+                           "windows_per_step": out_windows, "rows_per_step": out_rows,
+                           "out_tuples_per_step": out_tuples, "parallelism": f"dp{world} (stream partitions + halo)"},
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "gpu_launches": launches}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -116,7 +116,10 @@ typedef enum { SABER_RESULTS_HOST = 0, SABER_RESULTS_DEVICE = 1 } saber_result_m
  *                   partition's tail windows are left to its successor [1]
  *  result_slots     result slices held until released (the paper's circular
  *                   result buffer, L1044-1058); a submit that needs more free
- *                   slots than exist returns SABER_EAGAIN without consuming [8] */
+ *                   slots than exist returns SABER_EAGAIN without consuming [8]
+ *  profile          1: bracket each task's kernels with CUDA events on the
+ *                   query's stream and accumulate per-phase device time in
+ *                   saber_stats (read at poll)                  [0] */
 typedef struct {
   int32_t device;
   int64_t task_bytes;
@@ -129,7 +132,8 @@ typedef struct {
   int64_t first_window;
   int32_t emit_on_finish;
   int32_t result_slots;
-  int32_t reserved[6];
+  int32_t profile;
+  int32_t reserved[5];
 } saber_config;
 
 typedef struct saber_query saber_query;
@@ -216,11 +220,21 @@ typedef struct {
   int64_t tasks_pending;
   /* window-fragment classes of the last task */
   int64_t last_complete, last_opening, last_closing, last_pending;
+  /* device work: kernels launched, and (profile = 1) accumulated device time of
+   * the pane/selection pass (K1+σ+K2/K4 or K1+K3) and of window assembly +
+   * result stage (K5/K6), over the tasks polled so far */
+  int64_t kernel_launches;
+  int64_t scan_launches;        /* launches of the fused scan kernel (pane or select) */
+  double scan_ms, assemble_ms;
 } saber_stats;
 saber_status saber_query_stats(const saber_query *q, saber_stats *out);
 
 /* Block until all enqueued work of q is complete (results stay pending). */
 saber_status saber_query_sync(saber_query *q);
+/* Make `cuda_stream` (a cudaStream_t; NULL = legacy default stream) wait for
+ * all work enqueued on q so far, without blocking the host (stream-ordered
+ * completion, e.g. for CUDA-event timing around a whole query). */
+saber_status saber_query_record(saber_query *q, void *cuda_stream);
 
 void saber_query_destroy(saber_query *q);
 /* Human-readable reason for the last error of q (q may be NULL: global). */

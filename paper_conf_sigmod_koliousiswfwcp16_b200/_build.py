@@ -40,11 +40,22 @@ def _sources():
 def build(force: bool = False, verbose: bool = False) -> str:
     srcs = _sources()
     if force or _stale(LIB, srcs):
-        cu = [os.path.join(CSRC, f) for f in ("kernels.cu", "runtime.cu")]
-        cmd = [NVCC, *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), *cu, "-o", LIB + ".tmp"]
-        if verbose:
-            print(" ".join(cmd))
-        subprocess.check_call(cmd)
+        cus = [f for f in sorted(os.listdir(CSRC)) if f.endswith(".cu")]
+        objdir = os.path.join(CSRC, "..", "build")
+        os.makedirs(objdir, exist_ok=True)
+        objs, procs = [], []
+        for f in cus:     # one nvcc per translation unit, in parallel
+            o = os.path.join(objdir, f[:-3] + ".o")
+            objs.append(o)
+            cmd = [NVCC, *ARCH, *[x for x in FLAGS if x != "-shared"], "-c", "-I", os.path.join(ROOT, "include"),
+                   os.path.join(CSRC, f), "-o", o]
+            if verbose:
+                print(" ".join(cmd))
+            procs.append((f, subprocess.Popen(cmd)))
+        for f, pr in procs:
+            if pr.wait() != 0:
+                raise RuntimeError(f"nvcc failed on {f}")
+        subprocess.check_call([NVCC, *ARCH, "-shared", *objs, "-o", LIB + ".tmp"])
         os.replace(LIB + ".tmp", LIB)
     if force or _stale(GEN_LIB, [GEN_SRC]):
         cmd = [NVCC, *ARCH, *FLAGS, GEN_SRC, "-o", GEN_LIB + ".tmp"]

@@ -1,0 +1,229 @@
+// common.cuh -- device helpers shared by the kernel translation units.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "device_util.cuh"
+#include "plan.h"
+
+namespace sb {
+
+struct WinHdr { int64_t window_id, ts, row_offset; int32_t nrows, flags; };
+
+// --------------------------------------------------------------------------
+// generic tuple access
+template <int NW>
+__device__ __forceinline__ void load_tuple(const uint4 *t, unsigned mask, uint32_t (&w)[NW]) {
+#pragma unroll
+  for (int c = 0; c < NW / 4; ++c) {
+    uint4 v = make_uint4(0, 0, 0, 0);
+    if (mask & (1u << c)) v = ld_stream(t + c);
+    w[4 * c + 0] = v.x; w[4 * c + 1] = v.y; w[4 * c + 2] = v.z; w[4 * c + 3] = v.w;
+  }
+}
+
+template <int NW>
+__device__ __forceinline__ bool eval_preds(const Plan &p, const uint32_t (&w)[NW]) {
+  bool ok = true;
+  for (int i = 0; i < p.npred; ++i) {
+    const Pred &pr = p.pred[i];
+    if (pr.type == T_F32 || pr.type == T_F64) ok &= cmp_op(get_float<NW>(w, pr.word, pr.type), pr.op, pr.fval);
+    else ok &= cmp_op(get_int<NW>(w, pr.word, pr.type), pr.op, pr.ival);
+  }
+  return ok;
+}
+
+// GROUP BY key of a tuple (reading A17); flags ERR_KEY.
+template <int NW>
+__device__ __forceinline__ uint64_t make_key(const Plan &p, const uint32_t (&w)[NW], bool &valid, int &err) {
+  if (p.key_mode == KM_GLOBAL) return 0;
+  int64_t v[kMaxKey];
+#pragma unroll
+  for (int i = 0; i < kMaxKey; ++i) {
+    v[i] = 0;
+    if (i < p.nkeys) {
+      v[i] = get_int<NW>(w, p.key[i].word, p.key[i].type);
+      if (p.key[i].div != 1) v[i] /= p.key[i].div;
+    }
+  }
+  uint64_t k = 0;
+  bool bad = false;
+  if (p.key_pack == KP_RADIX) {
+#pragma unroll
+    for (int i = 0; i < kMaxKey; ++i)
+      if (i < p.nkeys) {
+        bad |= (v[i] < 0) | (v[i] >= p.key[i].domain);
+        k += (uint64_t)v[i] * (uint64_t)p.key[i].stride;
+      }
+  } else if (p.key_pack == KP_BIASED64) {
+    k = (uint64_t)v[0] ^ 0x8000000000000000ull;
+    bad = (k == kEmpty);
+  } else {
+    bad = (v[0] != (int32_t)v[0]) | (v[1] != (int32_t)v[1]);
+    k = ((uint64_t)((uint32_t)v[0] ^ 0x80000000u) << 32) | (uint64_t)((uint32_t)v[1] ^ 0x80000000u);
+    bad |= (k == kEmpty);
+  }
+  if (valid && bad) { err |= ERR_KEY; valid = false; }
+  return k;
+}
+
+template <int NW>
+__device__ __forceinline__ uint64_t field_value(const Field &f, const uint32_t (&w)[NW]) {
+  bool fl = (f.type == T_F32 || f.type == T_F64);
+  switch (f.kind) {
+    case FK_SUM_F: return (uint64_t)__double_as_longlong(get_float<NW>(w, f.word, f.type));
+    case FK_SUM_I: return (uint64_t)get_int<NW>(w, f.word, f.type);
+    default: return fl ? enc_dbl(get_float<NW>(w, f.word, f.type)) : enc_int(get_int<NW>(w, f.word, f.type));
+  }
+}
+
+__device__ __forceinline__ int64_t cnt_off(const Plan &p) { return p.key_mode == KM_HASH ? p.C : 0; }
+__device__ __forceinline__ int64_t fld_off(const Plan &p, int f) { return cnt_off(p) + (int64_t)(1 + f) * p.C; }
+
+// --------------------------------------------------------------------------
+// task prologue (one warp)
+__device__ __forceinline__ int64_t tau_at(const Plan &p, const unsigned char *t, int64_t i) {
+  return *(const int64_t *)(t + i * p.tuple_bytes + 4 * p.ts_word);
+}
+
+// lower_bound over the concatenation [a (na tuples) ++ b (nb tuples)] of τ < key (warp-cooperative)
+static __device__ int64_t warp_lower_bound(const Plan &p, const unsigned char *a, int64_t na,
+                                    const unsigned char *b, int64_t nb, int64_t key) {
+  const int lane = threadIdx.x & 31;
+  int64_t lo = 0, hi = na + nb;
+  while (lo < hi) {
+    int64_t span = hi - lo;
+    int64_t idx = (span <= 32) ? lo + lane : lo + (span * lane) / 32;
+    bool inb = idx < hi;
+    int64_t t = 0;
+    if (inb) t = idx < na ? tau_at(p, a, idx) : tau_at(p, b, idx - na);
+    bool pred = inb && t < key;
+    unsigned bal = __ballot_sync(kFull, pred);
+    int c = __popc(bal);
+    if (span <= 32) { lo = lo + c; break; }
+    if (c == 0) { hi = lo; break; }
+    int64_t prev = lo + (span * (c - 1)) / 32;
+    int64_t next = (c < 32) ? lo + (span * c) / 32 : hi;
+    lo = prev + 1;
+    hi = next;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ int64_t global_insert(const Plan &p, State *st, uint64_t *gkeys, uint64_t k, int &err) {
+  const uint32_t mask = (uint32_t)p.C - 1;
+  uint32_t h = (uint32_t)fmix64(k) & mask;
+  for (int64_t probe = 0; probe < p.C; ++probe) {
+    uint64_t cur = __ldcg((const unsigned long long *)&gkeys[h]);
+    if (cur == k) return h;
+    if (cur == kEmpty) {
+      uint64_t old = atomicCAS((unsigned long long *)&gkeys[h], kEmpty, k);
+      if (old == kEmpty || old == k) {
+        if (probe > 0) atomicMax((unsigned long long *)&st->max_probe, (unsigned long long)probe);
+        return h;
+      }
+    }
+    h = (h + 1) & mask;
+  }
+  err |= ERR_CAPACITY;
+  return -1;
+}
+
+
+// --------------------------------------------------------------------------
+// window assembly helpers
+struct AggVal { uint64_t bits; bool isf; };
+
+__device__ __forceinline__ AggVal finalize(const Plan &p, int a, int64_t cnt, const uint64_t *fv) {
+  const AggOut &o = p.agg[a];
+  AggVal r;
+  r.isf = o.out_float;
+  switch (o.fn) {
+    case AG_COUNT: r.bits = (uint64_t)cnt; break;
+    case AG_SUM: r.bits = fv[o.field]; break;
+    case AG_AVG: {
+      double sum = (p.field[o.field].kind == FK_SUM_F) ? __longlong_as_double((long long)fv[o.field])
+                                                      : (double)(int64_t)fv[o.field];
+      r.bits = (uint64_t)__double_as_longlong(sum / (double)cnt);   // reading A11
+      break;
+    }
+    default: {
+      uint64_t u = fv[o.field];
+      r.bits = o.is_float_col ? (uint64_t)__double_as_longlong(dec_dbl(u)) : (uint64_t)dec_int(u);
+    }
+  }
+  return r;
+}
+
+__device__ __forceinline__ bool having_ok(const Plan &p, int64_t cnt, const uint64_t *fv) {
+  for (int h = 0; h < p.nhave; ++h) {
+    const Have &hv = p.have[h];
+    AggVal v = finalize(p, hv.agg, cnt, fv);
+    bool ok = v.isf ? cmp_op(__longlong_as_double((long long)v.bits), hv.op, hv.fval)
+                    : cmp_op((int64_t)v.bits, hv.op, hv.ival);
+    if (!ok) return false;
+  }
+  return true;
+}
+
+__device__ __forceinline__ void write_row(const Plan &p, unsigned char *rows, int64_t r, const int64_t *kv,
+                                          int64_t cnt, const uint64_t *fv) {
+  if (r >= p.rows_cap) return;
+  for (int i = 0; i < p.nkeys; ++i) {
+    unsigned char *c = rows + p.col_off[i];
+    if (p.col_bytes[i] == 4) ((int32_t *)c)[r] = (int32_t)kv[i];
+    else ((int64_t *)c)[r] = kv[i];
+  }
+  for (int a = 0; a < p.nagg; ++a) {
+    AggVal v = finalize(p, a, cnt, fv);
+    ((uint64_t *)(rows + p.col_off[p.nkeys + a]))[r] = v.bits;
+  }
+}
+
+__device__ __forceinline__ void decode_key(const Plan &p, uint64_t k, int64_t *kv) {
+  if (p.key_pack == KP_RADIX) {
+    for (int i = 0; i < p.nkeys; ++i) kv[i] = (int64_t)((k / (uint64_t)p.key[i].stride) % (uint64_t)p.key[i].domain);
+  } else if (p.key_pack == KP_BIASED64) {
+    kv[0] = (int64_t)(k ^ 0x8000000000000000ull);
+  } else {
+    kv[0] = (int32_t)((uint32_t)(k >> 32) ^ 0x80000000u);
+    kv[1] = (int32_t)((uint32_t)k ^ 0x80000000u);
+  }
+}
+
+// exclusive scan over the threads of a group (GS = 32: warp; GS = 256: block)
+__device__ __forceinline__ int group_excl_scan(int v, int GS, int *sm, int &total) {
+  const int lane = threadIdx.x & 31;
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int y = __shfl_up_sync(kFull, x, o);
+    if (lane >= o) x += y;
+  }
+  if (GS == 32) {
+    total = __shfl_sync(kFull, x, 31);
+    return x - v;
+  }
+  const int wid = threadIdx.x >> 5;
+  if (lane == 31) sm[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    int w = lane < (GS >> 5) ? sm[lane] : 0;
+    int s = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int y = __shfl_up_sync(kFull, s, o);
+      if (lane >= o) s += y;
+    }
+    if (lane < (GS >> 5)) sm[lane] = s - w;
+    if (lane == (GS >> 5) - 1) sm[32] = s;
+  }
+  __syncthreads();
+  int r = sm[wid] + x - v;
+  total = sm[32];
+  __syncthreads();
+  return r;
+}
+
+
+}  // namespace sb

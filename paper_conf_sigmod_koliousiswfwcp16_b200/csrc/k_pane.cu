@@ -1,0 +1,461 @@
+// k_pane.cu -- K1 + σ + K2/K4 fused: the one HBM pass of an aggregation task.
+//
+// Each CTA owns a contiguous range of the task's tuples (row-major byte records,
+// PAPER.md L744-745) and streams it through shared memory with 1-D TMA bulk
+// copies (cp.async.bulk + mbarrier transaction counts), kStages deep, so the
+// HBM stream never waits on compute.  Per tuple, in shared memory:
+//   K1  pane id: count windows position/g, time windows (τ-T0)/g (panes are
+//       the window fragments of length g = gcd(s,l), L180-181, L1275-1280);
+//       τ non-decreasing (L347-349) and non-negative are checked here
+//   σ   conjunction of `col op const` (L1320-1322)
+//   γ   GROUP BY key (dense radix index or packed 64-bit key)
+//   α   fields of the accumulator (count, fp64/int64 sums, min/max)
+// and is folded into a warp-private shared-memory table after warp-level
+// de-duplication (__match_any_sync + shuffles; no shared-memory atomics).  The
+// CTA advances over a pane window [pbase, pbase+PL) that is uniform across its
+// warps; leaving it flushes the tables into the device pane ring with L2
+// atomics (RED), after summing the eight warp tables (DIRECT mode) so each
+// (pane, key) costs one set of REDs per CTA.
+#include <cuda_runtime.h>
+#include <climits>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "launch_internal.h"
+
+namespace sb {
+
+constexpr int kP1Threads = 256, kP1Warps = kP1Threads / 32;
+constexpr int kStageBytes = 16384;
+constexpr int kStages = 3;
+
+// ---------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase) {
+  asm volatile(
+      "{\n .reg .pred P1;\n"
+      "WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      " @!P1 bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+      "r"(phase)
+      : "memory");
+}
+// 1-D TMA bulk copy global → shared, completion counted on `bar` (SASS: UBLKCP)
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+// x / d for x >= 0 via a double reciprocal and exact integer correction
+__device__ __forceinline__ int64_t fdiv(int64_t x, int64_t d, double inv) {
+  if (d == 1) return x;
+  if (x < (1ll << 52)) {
+    int64_t q = (int64_t)((double)x * inv);
+    int64_t r = x - q * d;
+    while (r < 0) { --q; r += d; }
+    while (r >= d) { ++q; r -= d; }
+    return q;
+  }
+  return x / d;
+}
+
+// field access straight from the shared-memory tuple (runtime byte offsets)
+__device__ __forceinline__ int64_t s_int(const unsigned char *t, int word, int type) {
+  return type == T_I32 ? (int64_t) * (const int32_t *)(t + 4 * word) : *(const int64_t *)(t + 4 * word);
+}
+__device__ __forceinline__ double s_flt(const unsigned char *t, int word, int type) {
+  return type == T_F32 ? (double)*(const float *)(t + 4 * word) : *(const double *)(t + 4 * word);
+}
+
+__device__ __forceinline__ bool s_preds(const Plan &p, const unsigned char *t) {
+  bool ok = true;
+  for (int i = 0; i < p.npred; ++i) {
+    const Pred &pr = p.pred[i];
+    if (pr.type == T_F32 || pr.type == T_F64) ok &= cmp_op(s_flt(t, pr.word, pr.type), pr.op, pr.fval);
+    else ok &= cmp_op(s_int(t, pr.word, pr.type), pr.op, pr.ival);
+  }
+  return ok;
+}
+
+__device__ __forceinline__ uint64_t s_key(const Plan &p, const unsigned char *t, bool &valid, int &err) {
+  if (p.key_mode == KM_GLOBAL) return 0;
+  uint64_t k = 0;
+  bool bad = false;
+  if (p.key_pack == KP_RADIX) {
+    for (int i = 0; i < p.nkeys; ++i) {
+      int64_t v = s_int(t, p.key[i].word, p.key[i].type);
+      if (p.key[i].div != 1) v /= p.key[i].div;
+      bad |= (v < 0) | (v >= p.key[i].domain);
+      k += (uint64_t)v * (uint64_t)p.key[i].stride;
+    }
+  } else if (p.key_pack == KP_BIASED64) {
+    int64_t v = s_int(t, p.key[0].word, p.key[0].type);
+    if (p.key[0].div != 1) v /= p.key[0].div;
+    k = (uint64_t)v ^ 0x8000000000000000ull;
+    bad = (k == kEmpty);
+  } else {
+    int64_t v0 = s_int(t, p.key[0].word, p.key[0].type), v1 = s_int(t, p.key[1].word, p.key[1].type);
+    if (p.key[0].div != 1) v0 /= p.key[0].div;
+    if (p.key[1].div != 1) v1 /= p.key[1].div;
+    bad = (v0 != (int32_t)v0) | (v1 != (int32_t)v1);
+    k = ((uint64_t)((uint32_t)v0 ^ 0x80000000u) << 32) | (uint64_t)((uint32_t)v1 ^ 0x80000000u);
+    bad |= (k == kEmpty);
+  }
+  if (valid && bad) { err |= ERR_KEY; valid = false; }
+  return k;
+}
+
+__device__ __forceinline__ uint64_t s_field(const Field &f, const unsigned char *t) {
+  const bool fl = (f.type == T_F32 || f.type == T_F64);
+  switch (f.kind) {
+    case FK_SUM_F: return (uint64_t)__double_as_longlong(s_flt(t, f.word, f.type));
+    case FK_SUM_I: return (uint64_t)s_int(t, f.word, f.type);
+    default: return fl ? enc_dbl(s_flt(t, f.word, f.type)) : enc_int(s_int(t, f.word, f.type));
+  }
+}
+
+// leaders of each equal-key lane group receive the group's combined fields
+template <int NF>
+__device__ __forceinline__ void warp_combine(const Plan &p, bool act, unsigned m, uint64_t (&fv)[NF]) {
+  const int lane = threadIdx.x & 31;
+  const int leader = m ? __ffs(m) - 1 : -1;
+  const int npeer = __popc(m);
+  const int maxn = (int)__reduce_max_sync(kFull, act ? (unsigned)npeer : 0u);
+  if (maxn <= 1) return;
+  const unsigned lmask = __ballot_sync(kFull, act && leader == lane);
+  const int ng = __popc(lmask);
+  if (ng * 5 < maxn - 1) {
+    // few groups with many members (no GROUP BY, tiny G): one butterfly per group
+    unsigned rem = lmask;
+    while (rem) {
+      const int L = __ffs(rem) - 1;
+      rem &= rem - 1;
+      const bool mine = act && leader == L;
+#pragma unroll
+      for (int i = 0; i < NF; ++i) {
+        if (i >= p.nf) break;
+        const int kind = p.field[i].kind;
+        uint64_t v = mine ? fv[i] : field_identity(kind);
+#pragma unroll
+        for (int x = 16; x; x >>= 1) v = field_combine(kind, v, shfl_xor64(v, x));
+        if (lane == L) fv[i] = v;
+      }
+    }
+  } else {
+    unsigned rest = act ? (m & (m - 1)) : 0u;   // peers after the leader
+    uint64_t acc[NF];
+#pragma unroll
+    for (int i = 0; i < NF; ++i) acc[i] = fv[i];
+    for (int k = 1; k < maxn; ++k) {
+      const bool ok = rest != 0u;
+      const int s = ok ? __ffs(rest) - 1 : lane;
+      rest &= rest - 1;
+#pragma unroll
+      for (int i = 0; i < NF; ++i) {
+        if (i >= p.nf) break;
+        const uint64_t o = shfl64(fv[i], s);
+        if (ok) acc[i] = field_combine(p.field[i].kind, acc[i], o);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < NF; ++i) fv[i] = acc[i];
+  }
+}
+
+// add one pre-aggregated (pane, key) entry into the device pane ring
+template <int NF>
+__device__ __forceinline__ void flush_entry(const Plan &p, State *st, uint64_t *table, int64_t pane, uint64_t key,
+                                            uint32_t c, const uint64_t (&fv)[NF], int &err) {
+  uint64_t *base = table + (pane & (p.R - 1)) * p.slot_words;
+  int64_t idx;
+  if (p.key_mode == KM_HASH) {
+    idx = global_insert(p, st, base, key, err);
+    if (idx < 0) return;
+  } else {
+    idx = (int64_t)key;
+  }
+  atomicAdd((unsigned long long *)&base[cnt_off(p) + idx], (unsigned long long)c);
+#pragma unroll
+  for (int i = 0; i < NF; ++i)
+    if (i < p.nf) red_field(p.field[i].kind, &base[fld_off(p, i) + idx], fv[i]);
+}
+
+template <bool HASHED, int WK, int NF>
+__global__ void __launch_bounds__(kP1Threads, 2)
+k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
+           uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ long long s_next;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int tb = p.tuple_bytes;
+  const int ST = kStageBytes / tb;                       // tuples per stage
+  unsigned char *stages = smem;
+  uint64_t *full = (uint64_t *)(smem + kStages * kStageBytes);
+  uint64_t *empty = full + kStages;
+  unsigned char *tabs = (unsigned char *)(empty + kStages);
+  const int TE = p.local_entries;
+  unsigned char *wt = tabs + (size_t)wid * p.local_bytes;
+  uint64_t *tkeys = (uint64_t *)wt;
+  uint64_t *tf = (uint64_t *)(wt + (HASHED ? 8 * TE : 0));
+  uint32_t *tcnt = (uint32_t *)(wt + (HASHED ? 8 * TE : 0) + (size_t)8 * TE * NF);
+  for (int e = lane; e < TE; e += 32) {
+    if (HASHED) tkeys[e] = kEmpty;
+    tcnt[e] = 0;
+#pragma unroll
+    for (int f = 0; f < NF; ++f) tf[f * TE + e] = f < p.nf ? field_identity(p.field[f].kind) : 0;
+  }
+
+  // contiguous, stage-aligned range of this CTA
+  const int64_t per = ((n + gridDim.x - 1) / gridDim.x + ST - 1) / ST * ST;
+  const int64_t lo = (int64_t)blockIdx.x * per;
+  const int64_t hi = lo + per < n ? lo + per : n;
+  const int64_t nst = hi > lo ? (hi - lo + ST - 1) / ST : 0;
+  if (tid == 0) {
+    for (int i = 0; i < kStages; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], kP1Warps); }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  auto issue = [&](int64_t k) {
+    const int slot = (int)(k % kStages);
+    const int64_t cnt = (hi - lo - k * ST) < ST ? (hi - lo - k * ST) : ST;
+    const uint32_t bytes = (uint32_t)(cnt * tb);
+    mbar_expect_tx(&full[slot], bytes);
+    bulk_g2s(stages + slot * kStageBytes, tup + (lo + k * ST) * tb, bytes, &full[slot]);
+  };
+  if (tid == 0)
+    for (int64_t k = 0; k < kStages && k < nst; ++k) issue(k);
+
+  const int64_t pos0 = st->task_pos;
+  const int64_t min_pane = st->J0 * p.L;
+  const int PL = HASHED ? 1 : p.local_pl;
+  const int C = (int)p.C;
+  const int tsw = p.ts_word;
+  int err = 0;
+  int occ = 0;
+  int64_t pbase = -1;      // CTA-uniform pane window [pbase, pbase + PL)
+  int64_t prev_last = (lo > 0 && lo < hi) ? *(const int64_t *)(tup + (lo - 1) * tb + 4 * tsw) : INT64_MIN;
+  const int per_warp = (ST + kP1Warps - 1) / kP1Warps;
+
+  auto flush_direct = [&]() {
+    __syncthreads();
+    for (int e = tid; e < TE; e += kP1Threads) {
+      uint32_t c = 0;
+      uint64_t fv[NF];
+#pragma unroll
+      for (int f = 0; f < NF; ++f) fv[f] = f < p.nf ? field_identity(p.field[f].kind) : 0;
+      for (int w = 0; w < kP1Warps; ++w) {
+        unsigned char *ow = tabs + (size_t)w * p.local_bytes;
+        uint64_t *of = (uint64_t *)ow;
+        uint32_t *oc = (uint32_t *)(ow + (size_t)8 * TE * NF);
+        const uint32_t cw = oc[e];
+        if (!cw) continue;
+        c += cw;
+        oc[e] = 0;
+#pragma unroll
+        for (int f = 0; f < NF; ++f)
+          if (f < p.nf) {
+            fv[f] = field_combine(p.field[f].kind, fv[f], of[f * TE + e]);
+            of[f * TE + e] = field_identity(p.field[f].kind);
+          }
+      }
+      if (c) flush_entry<NF>(p, st, table, pbase + e / C, (uint64_t)(e % C), c, fv, err);
+    }
+    __syncthreads();
+  };
+  auto flush_hashed = [&]() {      // warp-private table of one pane
+    __syncwarp();
+    for (int e = lane; e < TE; e += 32) {
+      const uint64_t k = tkeys[e];
+      if (k == kEmpty) continue;
+      uint64_t fv[NF];
+#pragma unroll
+      for (int f = 0; f < NF; ++f) {
+        fv[f] = tf[f * TE + e];
+        if (f < p.nf) tf[f * TE + e] = field_identity(p.field[f].kind);
+      }
+      flush_entry<NF>(p, st, table, pbase, k, tcnt[e], fv, err);
+      tkeys[e] = kEmpty;
+      tcnt[e] = 0;
+    }
+    __syncwarp();
+    occ = 0;
+  };
+
+  for (int64_t k = 0; k < nst; ++k) {
+    const int slot = (int)(k % kStages);
+    const uint32_t phase = (uint32_t)((k / kStages) & 1);
+    mbar_wait(&full[slot], phase);
+    const unsigned char *sb = stages + slot * kStageBytes;
+    const int ntup = (int)((hi - lo - k * ST) < ST ? (hi - lo - k * ST) : ST);
+    const int64_t spos = pos0 + lo + k * ST;             // global position of stage tuple 0
+    int64_t pf, pl;                                      // stage pane range (CTA-uniform)
+    if (WK == WK_COUNT) {
+      pf = fdiv(spos, p.g, p.g_inv);
+      pl = fdiv(spos + ntup - 1, p.g, p.g_inv);
+    } else {
+      const int64_t t0 = *(const int64_t *)(sb + 4 * tsw), t1 = *(const int64_t *)(sb + (ntup - 1) * tb + 4 * tsw);
+      pf = t0 >= p.T0 ? fdiv(t0 - p.T0, p.g, p.g_inv) : 0;
+      pl = t1 >= p.T0 ? fdiv(t1 - p.T0, p.g, p.g_inv) : -1;
+    }
+    if (pf < min_pane) pf = min_pane;
+    const int ib = wid * per_warp;
+    const int ie = ib + per_warp < ntup ? ib + per_warp : ntup;
+    // K1 order check, once per tuple
+    for (int i = ib + lane; i < ie; i += 32) {
+      const int64_t tau = *(const int64_t *)(sb + i * tb + 4 * tsw);
+      const int64_t up = i > 0 ? *(const int64_t *)(sb + (i - 1) * tb + 4 * tsw) : prev_last;
+      if (tau < up) err |= ERR_ORDER;
+      if (tau < 0) err |= ERR_TS;
+    }
+    int64_t cur = pf;
+    bool first_round = true;
+    while (cur <= pl) {
+      if (pbase < 0 || cur < pbase || cur >= pbase + PL) {
+        if (pbase >= 0) {
+          if (HASHED) flush_hashed(); else flush_direct();
+        }
+        pbase = cur;
+      }
+      const int64_t wend = pbase + PL;
+      for (int i0 = ib; i0 < ie; i0 += 32) {
+        const int i = i0 + lane;
+        bool valid = i < ie;
+        const unsigned char *t = sb + (valid ? i : ib) * tb;
+        int64_t pane;
+        if (WK == WK_COUNT) {
+          const int64_t pos = spos + i;
+          pane = fdiv(pos, p.g, p.g_inv);
+          if (valid && first_round && pos == pane * p.g && pane >= min_pane)
+            pane_ts[pane & (p.R - 1)] = *(const int64_t *)(t + 4 * tsw);
+        } else {
+          const int64_t tau = *(const int64_t *)(t + 4 * tsw);
+          valid &= tau >= p.T0;
+          pane = tau >= p.T0 ? fdiv(tau - p.T0, p.g, p.g_inv) : -1;
+        }
+        valid &= (pane >= pbase) & (pane < wend) & (pane >= min_pane);
+        if (p.npred && valid) valid &= s_preds(p, t);
+        const uint64_t key = s_key(p, t, valid, err);
+        uint64_t fv[NF];
+#pragma unroll
+        for (int f = 0; f < NF; ++f) fv[f] = (f < p.nf) ? s_field(p.field[f], t) : 0;
+        const unsigned actm = __ballot_sync(kFull, valid);
+        if (!actm) continue;
+        if (!HASHED) {
+          const int e = valid ? (int)(pane - pbase) * C + (int)key : -1 - lane;
+          const unsigned m = __match_any_sync(kFull, e) & actm;
+          warp_combine<NF>(p, valid, m, fv);
+          if (valid && (__ffs(m) - 1) == lane) {
+            tcnt[e] += (uint32_t)__popc(m);
+#pragma unroll
+            for (int f = 0; f < NF; ++f)
+              if (f < p.nf) tf[f * TE + e] = field_combine(p.field[f].kind, tf[f * TE + e], fv[f]);
+          }
+        } else {
+          if (occ + 32 > TE / 2) flush_hashed();
+          const unsigned m = __match_any_sync(kFull, (unsigned long long)key) & actm;
+          warp_combine<NF>(p, valid, m, fv);
+          bool ins = false;
+          if (valid && (__ffs(m) - 1) == lane) {
+            uint32_t h = (uint32_t)fmix64(key) & (uint32_t)(TE - 1);
+            volatile uint64_t *vk = tkeys;
+            for (;;) {
+              const uint64_t kk = vk[h];
+              if (kk == key) break;
+              if (kk == kEmpty) {
+                const uint64_t old = atomicCAS((unsigned long long *)&tkeys[h], kEmpty, key);
+                if (old == kEmpty) { ins = true; break; }
+                if (old == key) break;
+              }
+              h = (h + 1) & (uint32_t)(TE - 1);
+            }
+            tcnt[h] += (uint32_t)__popc(m);
+#pragma unroll
+            for (int f = 0; f < NF; ++f)
+              if (f < p.nf) tf[f * TE + h] = field_combine(p.field[f].kind, tf[f * TE + h], fv[f]);
+          }
+          occ += __popc(__ballot_sync(kFull, ins));
+        }
+        __syncwarp();
+      }
+      first_round = false;
+      if (pl < wend) break;
+      // next non-empty pane >= wend in this stage (time gaps, tiny panes)
+      if (tid == 0) s_next = LLONG_MAX;
+      __syncthreads();
+      for (int i = ib + lane; i < ie; i += 32) {
+        const unsigned char *t = sb + i * tb;
+        int64_t pane;
+        if (WK == WK_COUNT) pane = fdiv(spos + i, p.g, p.g_inv);
+        else {
+          const int64_t tau = *(const int64_t *)(t + 4 * tsw);
+          pane = tau >= p.T0 ? fdiv(tau - p.T0, p.g, p.g_inv) : -1;
+        }
+        if (pane >= wend) atomicMin(&s_next, (long long)pane);
+      }
+      __syncthreads();
+      cur = s_next;
+      __syncthreads();
+    }
+    prev_last = *(const int64_t *)(sb + (ntup - 1) * tb + 4 * tsw);
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[slot]);
+    if (tid == 0 && k + kStages < nst) {
+      mbar_wait(&empty[slot], phase);
+      issue(k + kStages);
+    }
+  }
+  if (pbase >= 0) {
+    if (HASHED) flush_hashed(); else flush_direct();
+  }
+  if (err) atomicOr(&st->error, err);
+}
+
+// ---------------------------------------------------------------- host side
+int p1_nf_template(int nf) { return nf <= 1 ? 1 : nf <= 2 ? 2 : nf <= 4 ? 4 : 8; }
+
+int p1_smem_bytes(const Plan &p) { return kStages * kStageBytes + 2 * kStages * 8 + kP1Warps * p.local_bytes; }
+
+template <bool H, int WK>
+static void *p1_nf(int nf) {
+  switch (p1_nf_template(nf)) {
+    case 1: return (void *)k_pane_agg<H, WK, 1>;
+    case 2: return (void *)k_pane_agg<H, WK, 2>;
+    case 4: return (void *)k_pane_agg<H, WK, 4>;
+    default: return (void *)k_pane_agg<H, WK, 8>;
+  }
+}
+void *p1_kernel(const Plan &p) {
+  const bool h = !p.local_direct;
+  if (p.win_kind == WK_COUNT) return h ? p1_nf<true, WK_COUNT>(p.nf) : p1_nf<false, WK_COUNT>(p.nf);
+  return h ? p1_nf<true, WK_TIME>(p.nf) : p1_nf<false, WK_TIME>(p.nf);
+}
+
+int p1_blocks_per_sm(const Plan &p) {
+  int b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, p1_kernel(p), kP1Threads, p1_smem_bytes(p));
+  return b > 0 ? b : 1;
+}
+
+cudaError_t launch_pane_agg(const Plan &p, const QueryDev &q, const void *tuples, int64_t n, int grid,
+                            cudaStream_t st) {
+  if (n <= 0) return cudaSuccess;
+  const int64_t stage_t = kStageBytes / p.tuple_bytes;
+  int64_t need = (n + stage_t - 1) / stage_t;     // at least one stage per CTA
+  int g = (int)(need < grid ? need : grid);
+  void *args[] = {(void *)&p, (void *)&q.st, (void *)&tuples, (void *)&n, (void *)&q.table, (void *)&q.pane_ts};
+  return cudaLaunchKernel(p1_kernel(p), dim3(g), dim3(kP1Threads), args, (size_t)p1_smem_bytes(p), st);
+}
+
+}  // namespace sb

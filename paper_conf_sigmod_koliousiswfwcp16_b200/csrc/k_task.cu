@@ -1,0 +1,296 @@
+// k_task.cu -- scalar task prologue/epilogue, pane-ring initialisation, window headers, IStream carry, partition planning.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "launch_internal.h"
+
+namespace sb {
+
+__global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, int64_t n, int final_,
+                             int has_wm, int64_t wm, int emit_on_finish, SlotMeta *meta,
+                             const unsigned char *carry0, const unsigned char *carry1, int *tile_ctr) {
+  const int lane = threadIdx.x;
+  __shared__ int64_t sh[8];
+  if (lane == 0) {
+    int err = 0;
+    const int64_t pos0 = st->pos_next;
+    st->task_pos = pos0;
+    st->task_n = n;
+    int64_t J0 = st->J0, J1 = J0;
+    int64_t plo = 0, phi = -1;
+    if (n > 0) {
+      int64_t tf = tau_at(p, tup, 0), tl = tau_at(p, tup, n - 1);
+      if (tf < 0) err |= ERR_TS;
+      if (st->has_tau && tf < st->tau_last) err |= ERR_ORDER;
+      if (!st->has_tau || tl > st->tau_last) st->tau_last = tl;
+      st->has_tau = 1;
+    }
+    if (p.win_kind == WK_TIME) {
+      if (n > 0) {
+        int64_t tf = tau_at(p, tup, 0), tl = tau_at(p, tup, n - 1);
+        if (tl >= p.T0) {
+          plo = tf >= p.T0 ? (tf - p.T0) / p.g : 0;
+          phi = (tl - p.T0) / p.g;
+        }
+      }
+      // window j = [T0+j·l, T0+j·l+s) is closed once a tuple with τ >= its end has
+      // arrived (τ non-decreasing, L347-349) or the watermark passed it (reading A3)
+      bool use_wm = final_ && emit_on_finish;
+      int64_t B;
+      bool haveB = true;
+      if (use_wm && has_wm) B = wm;
+      else if (use_wm) { B = st->tau_last + 1; haveB = st->has_tau; }
+      else { B = st->tau_last; haveB = st->has_tau; }
+      if (haveB && B - p.T0 - p.s >= 0) J1 = (B - p.T0 - p.s) / p.l + 1;
+    } else {
+      int64_t total = pos0 + n;   // count: W_j = [j·l, j·l+s) closes with position j·l+s-1
+      if (total >= p.s) J1 = (total - p.s) / p.l + 1;
+      if (n > 0) { plo = pos0 / p.g; phi = (total - 1) / p.g; }
+    }
+    if (J1 < J0) J1 = J0;
+    st->pos_next = pos0 + n;
+    st->J1 = J1;
+    // pane ring: slots of panes [J0·L, phi] must coexist during this task
+    int64_t live_lo = J0 * p.L;
+    int64_t zlo = st->zeroed_hi > live_lo ? st->zeroed_hi : live_lo;
+    int64_t zhi = zlo;
+    if (phi >= 0 && p.nagg > 0) {
+      if (phi - live_lo + 1 > p.R) err |= ERR_CAPACITY;
+      else if (phi + 1 > zlo) zhi = phi + 1;
+    }
+    st->zero_lo = zlo;
+    st->zero_hi = zhi;
+    if (zhi > st->zeroed_hi) st->zeroed_hi = zhi;
+    if (phi > st->pane_hi) st->pane_hi = phi;
+    (void)plo;
+    if (J1 - J0 > p.win_cap) err |= ERR_RESULT;
+    meta->first_window = J0;
+    meta->nwindows = J1 - J0;
+    if (err) st->error |= err;
+    st->tile_epoch += 1;
+    st->sel_rows = 0;
+    *tile_ctr = 0;
+    sh[0] = J0; sh[1] = J1; sh[2] = pos0;
+  }
+  __syncwarp();
+  if (p.nagg > 0) return;
+  // ---- IStream cover (L395-400): emit selected tuples of window positions not
+  // emitted before; the virtual input is [carry ++ task]
+  const int64_t J0 = sh[0], J1 = sh[1], pos0 = sh[2];
+  const unsigned char *carry = st->carry_sel ? carry1 : carry0;
+  const int64_t cpos = st->carry_pos, cn = st->carry_n;
+  int64_t cover_lo = st->cover_hi;
+  int64_t cover_hi;
+  if (p.win_kind == WK_COUNT) {
+    if (st->first_task) cover_lo = J0 > 0 ? (J0 - 1) * p.l + p.s : 0;
+    cover_hi = J1 > 0 ? (J1 - 1) * p.l + p.s : cover_lo;
+  } else {
+    if (st->first_task) {
+      int64_t B = J0 > 0 ? p.T0 + (J0 - 1) * p.l + p.s : p.T0;
+      cover_lo = cpos + warp_lower_bound(p, carry, cn, tup, n, B);
+    }
+    if (J1 > 0) {
+      int64_t B = p.T0 + (J1 - 1) * p.l + p.s;
+      cover_hi = cpos + warp_lower_bound(p, carry, cn, tup, n, B);
+    } else {
+      cover_hi = cover_lo;
+    }
+  }
+  if (lane == 0) {
+    if (cover_hi < cover_lo) cover_hi = cover_lo;
+    const int64_t end = pos0 + n;
+    if (cover_lo < cpos) cover_lo = cpos;
+    if (cover_hi > end) cover_hi = end;
+    st->cover_lo = cover_lo;
+    st->cover_hi = cover_hi;
+    st->first_task = 0;
+    // the uncovered tail [max(cover_hi, cpos), end) is carried to the next task
+    int64_t ncp = cover_hi > cpos ? cover_hi : cpos;
+    st->zero_lo = ncp;            // reused: new carry position
+    st->zero_hi = end - ncp;      // reused: new carry length
+    if (end - ncp > p.carry_cap) st->error |= ERR_CARRY;
+  }
+}
+
+// --------------------------------------------------------------------------
+__global__ void k_zero_panes(const Plan p, const State *st, uint64_t *table) {
+  const int64_t lo = st->zero_lo, hi = st->zero_hi;
+  if (hi <= lo) return;
+  const int64_t words = (hi - lo) * p.slot_words;
+  const int64_t co = cnt_off(p);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < words;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t pane = lo + i / p.slot_words;
+    int64_t w = i % p.slot_words;
+    uint64_t v;
+    if (w < co) v = kEmpty;                               // hash keys
+    else if (w < co + p.C) v = 0;                         // counts
+    else v = field_identity(p.field[(w - co - p.C) / p.C].kind);
+    table[(pane & (p.R - 1)) * p.slot_words + w] = v;
+  }
+}
+
+__global__ void __launch_bounds__(1024)
+k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t *__restrict__ counts,
+           WinHdr *__restrict__ hdr, SlotMeta *meta) {
+  __shared__ int64_t wsum[32];
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  const int S = p.S;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int64_t per = (nw + blockDim.x - 1) / blockDim.x;
+  const int64_t a = (int64_t)tid * per, b = (a + per < nw) ? a + per : nw;
+  int64_t local = 0;
+  for (int64_t j = a; j < b; ++j)
+    for (int s = 0; s < S; ++s) local += counts[j * S + s];
+  int64_t x = local;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int64_t y = (int64_t)__shfl_up_sync(kFull, (unsigned long long)x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    int64_t w = wsum[lane], s = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int64_t y = (int64_t)__shfl_up_sync(kFull, (unsigned long long)s, o);
+      if (lane >= o) s += y;
+    }
+    wsum[lane] = s - w;
+  }
+  __syncthreads();
+  int64_t run = wsum[wid] + x - local;
+  for (int64_t j = a; j < b; ++j) {
+    WinHdr h;
+    h.window_id = J0 + j;
+    h.ts = (p.win_kind == WK_TIME) ? p.T0 + (J0 + j) * p.l : pane_ts[((J0 + j) * p.L) & (p.R - 1)];
+    h.row_offset = run;
+    int64_t nr = 0;
+    for (int s = 0; s < S; ++s) {
+      int64_t c = counts[j * S + s];
+      counts[j * S + s] = run;
+      run += c;
+      nr += c;
+    }
+    h.nrows = (int32_t)nr;
+    h.flags = 0;
+    hdr[j] = h;
+  }
+  if (tid == blockDim.x - 1) {
+    meta->nrows = run;
+    if (run > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+  }
+}
+
+__global__ void k_task_end(const Plan p, State *st, SlotMeta *meta) {
+  if (threadIdx.x) return;
+  meta->first_window = st->J0;
+  meta->nwindows = st->J1 - st->J0;
+  meta->error = st->error;
+  meta->pos_end = st->pos_next;
+  meta->tau_last = st->tau_last;
+  if (p.nagg == 0) {
+    meta->nrows = 0;
+    meta->ntuples = st->sel_rows;
+    st->carry_pos = st->zero_lo;
+    st->carry_n = st->zero_hi;
+    st->carry_sel ^= 1;
+    st->zero_lo = st->zero_hi = 0;
+  } else {
+    meta->ntuples = 0;
+  }
+  st->J0 = st->J1;
+}
+
+__global__ void k_carry(const Plan p, const State *st, const uint4 *task, const uint4 *carry0,
+                        const uint4 *carry1, uint4 *dst0, uint4 *dst1) {
+  const int64_t ncp = st->zero_lo, nn = st->zero_hi;
+  if (nn <= 0 || nn > p.carry_cap) return;
+  const int64_t tpos = st->task_pos, cpos = st->carry_pos;
+  const uint4 *carry = st->carry_sel ? carry1 : carry0;
+  uint4 *dst = st->carry_sel ? dst0 : dst1;
+  const int CW = p.tuple_bytes / 16;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nn * CW; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t pos = ncp + i / CW;
+    const int c = (int)(i % CW);
+    dst[i] = pos < tpos ? carry[(pos - cpos) * CW + c] : task[(pos - tpos) * CW + c];
+  }
+}
+
+__global__ void k_init_state(State *st, int64_t base_index, int64_t first_window, int64_t L) {
+  if (threadIdx.x) return;
+  State s = {};
+  s.pos_next = base_index;
+  s.J0 = first_window;
+  s.J1 = first_window;
+  s.zeroed_hi = first_window * L;
+  s.pane_hi = -1;
+  s.first_task = 1;
+  s.carry_pos = base_index;
+  *st = s;
+}
+
+__global__ void k_partition_plan(int ts_word, int tuple_bytes, int win_kind, int64_t s, int64_t l, int64_t T0,
+                                 const unsigned char *tup, int64_t begin, int64_t n, int64_t *out) {
+  Plan p;
+  p.ts_word = ts_word;
+  p.tuple_bytes = tuple_bytes;
+  int64_t closed = 0, halo = begin;
+  if (win_kind == WK_COUNT) {
+    const int64_t total = begin + n;
+    closed = total >= s ? (total - s) / l + 1 : 0;
+    halo = closed * l;
+  } else if (n > 0) {
+    const int64_t tl = tau_at(p, tup, n - 1);
+    closed = (tl - T0 - s >= 0) ? (tl - T0 - s) / l + 1 : 0;
+    const int64_t B = T0 + closed * l;
+    const int64_t idx = warp_lower_bound(p, tup, n, tup, 0, B);
+    halo = begin + idx;
+    if (idx == 0 && begin > 0 && tau_at(p, tup, 0) > B) closed = -1;   // window spans > partition
+  }
+  if (threadIdx.x == 0) { out[0] = closed; out[1] = halo; }
+}
+
+// ==========================================================================
+
+}  // namespace sb
+
+namespace sb {
+
+cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
+                              int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st) {
+  k_task_begin<<<1, 32, 0, st>>>(p, q.st, (const unsigned char *)tuples, n, final_, has_wm, wm, emit_on_finish,
+                                 s.meta, q.carry[0], q.carry[1], q.tile_ctr);
+  return cudaGetLastError();
+}
+cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st) {
+  k_zero_panes<<<148 * 4, 256, 0, st>>>(p, q.st, q.table);
+  return cudaGetLastError();
+}
+cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st) {
+  k_win_scan<<<1, 1024, 0, st>>>(p, q.st, q.pane_ts, s.counts, (WinHdr *)s.hdr, s.meta);
+  return cudaGetLastError();
+}
+cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st) {
+  k_task_end<<<1, 32, 0, st>>>(p, q.st, s.meta);
+  return cudaGetLastError();
+}
+cudaError_t launch_carry(const Plan &p, const QueryDev &q, const void *tuples, cudaStream_t st) {
+  k_carry<<<148, 256, 0, st>>>(p, q.st, (const uint4 *)tuples, (const uint4 *)q.carry[0], (const uint4 *)q.carry[1],
+                               (uint4 *)q.carry[0], (uint4 *)q.carry[1]);
+  return cudaGetLastError();
+}
+cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, cudaStream_t s) {
+  k_init_state<<<1, 32, 0, s>>>(q.st, base_index, p.first_window, p.L);
+  return cudaGetLastError();
+}
+cudaError_t launch_partition_plan(int ts_word, int tuple_words, int win_kind, int64_t s, int64_t l, int64_t T0,
+                                  const void *tuples, int64_t begin, int64_t n, int64_t *dev_out2, cudaStream_t st) {
+  k_partition_plan<<<1, 32, 0, st>>>(ts_word, tuple_words * 4, win_kind, s, l, T0, (const unsigned char *)tuples,
+                                     begin, n, dev_out2);
+  return cudaGetLastError();
+}
+
+}  // namespace sb

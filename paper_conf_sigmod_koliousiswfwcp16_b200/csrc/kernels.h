@@ -17,6 +17,8 @@ struct SlotDev {
 struct QueryDev {
   State *st;
   uint64_t *table;          // pane ring: R slots × slot_words
+  uint64_t *vh_pre;         // van Herk block-prefix arrays (DENSE/GLOBAL), same geometry
+  uint64_t *vh_suf;         // van Herk block-suffix arrays
   int64_t *pane_ts;         // R
   uint64_t *tile_status;    // IStream look-back
   int64_t tile_status_cap;
@@ -28,11 +30,12 @@ struct QueryDev {
 // one task of an aggregation (RStream) query
 cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
                             int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
-                            int p1_grid, int p2_grid, int win_chunk, cudaStream_t st);
+                            int p1_grid, int p2_grid, int win_chunk, cudaStream_t st,
+                            cudaEvent_t *evs /* 3 events or nullptr */, int *launches);
 // one task of a σ/π (IStream) query
 cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
                                int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
-                               int sel_grid, cudaStream_t st);
+                               int sel_grid, cudaStream_t st, cudaEvent_t *evs, int *launches);
 cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, cudaStream_t st);
 cudaError_t launch_partition_plan(int ts_word, int tuple_words, int win_kind, int64_t s, int64_t l,
                                   int64_t T0, const void *tuples, int64_t begin, int64_t n,

@@ -1,0 +1,71 @@
+// launch.cu -- the kernel sequence of one query task (host side).
+#include <cuda_runtime.h>
+
+#include "kernels.h"
+#include "launch_internal.h"
+
+namespace sb {
+
+cudaError_t set_kernel_attributes(const Plan &p) {
+  cudaError_t e = cudaSuccess;
+  if (p.nagg > 0) {
+    e = cudaFuncSetAttribute(p1_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p1_smem_bytes(p));
+    if (e) return e;
+    if (p.p2_smem > 0) e = cudaFuncSetAttribute(p2_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
+    if (e) return e;
+    if (p.key_mode == KM_HASH) {
+      e = cudaFuncSetAttribute(p2_kernel_count(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
+    }
+  }
+  return e;
+}
+
+int p2_blocks_per_sm(const Plan &p) {
+  int b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, p2_kernel(p), 256, p.p2_smem);
+  return b > 0 ? b : 1;
+}
+int sel_blocks_per_sm(const Plan &p) {
+  int b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sel_kernel(p), 256, 0);
+  return b > 0 ? b : 1;
+}
+
+cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
+                            int final_, int has_wm, int64_t wm, int emit_on_finish, int p1_grid, int p2_grid,
+                            int win_chunk, cudaStream_t st, cudaEvent_t *evs, int *launches) {
+  cudaError_t e;
+  if ((e = launch_task_begin(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, st))) return e;
+  if ((e = launch_zero_panes(p, q, st))) return e;
+  *launches = 2;
+  if (evs) cudaEventRecord(evs[0], st);
+  if (n > 0) {
+    if ((e = launch_pane_agg(p, q, tuples, n, p1_grid, st))) return e;
+    *launches += 1;
+  }
+  if (evs) cudaEventRecord(evs[1], st);
+  if ((e = launch_windows(p, q, s, false, p2_grid, win_chunk, st))) return e;
+  if ((e = launch_win_scan(p, q, s, st))) return e;
+  if ((e = launch_windows(p, q, s, true, p2_grid, win_chunk, st))) return e;
+  if ((e = launch_task_end(p, q, s, st))) return e;
+  *launches += p.key_mode == KM_HASH ? 4 : 5;
+  if (evs) cudaEventRecord(evs[2], st);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
+                               int final_, int has_wm, int64_t wm, int emit_on_finish, int sel_grid, cudaStream_t st,
+                               cudaEvent_t *evs, int *launches) {
+  cudaError_t e;
+  if ((e = launch_task_begin(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, st))) return e;
+  if (evs) cudaEventRecord(evs[0], st);
+  if ((e = launch_select(p, q, s, tuples, sel_grid, st))) return e;
+  if (evs) cudaEventRecord(evs[1], st);
+  if ((e = launch_carry(p, q, tuples, st))) return e;
+  if ((e = launch_task_end(p, q, s, st))) return e;
+  *launches = 4;
+  if (evs) cudaEventRecord(evs[2], st);
+  return cudaGetLastError();
+}
+
+}  // namespace sb

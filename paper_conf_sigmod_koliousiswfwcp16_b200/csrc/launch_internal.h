@@ -1,0 +1,30 @@
+// launch_internal.h -- per-translation-unit launchers (host side), used by launch.cu.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "kernels.h"
+#include "plan.h"
+
+namespace sb {
+// k_task.cu
+cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
+                              int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st);
+cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st);
+cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);
+cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);
+cudaError_t launch_carry(const Plan &p, const QueryDev &q, const void *tuples, cudaStream_t st);
+// k_pane.cu
+void *p1_kernel(const Plan &p);
+cudaError_t launch_pane_agg(const Plan &p, const QueryDev &q, const void *tuples, int64_t n, int grid,
+                            cudaStream_t st);
+// k_window.cu
+void *p2_kernel(const Plan &p);
+void *p2_kernel_count(const Plan &p);
+cudaError_t launch_windows(const Plan &p, const QueryDev &q, const SlotDev &s, bool emit, int grid, int win_chunk,
+                           cudaStream_t st);
+// k_select.cu
+void *sel_kernel(const Plan &p);
+cudaError_t launch_select(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int grid,
+                          cudaStream_t st);
+}  // namespace sb

@@ -46,6 +46,7 @@ struct Plan {
   // window ω(s,l), panes
   int32_t win_kind, pad0;
   int64_t s, l, T0, g, K, L;
+  double g_inv;                   // 1/g for the reciprocal division in K1
   // σ
   int32_t npred, pad1;
   Pred pred[kMaxPred];

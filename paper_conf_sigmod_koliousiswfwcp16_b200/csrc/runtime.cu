@@ -37,6 +37,8 @@ struct Slot {
   saber_win_hdr *h_hdr = nullptr;
   SlotMeta *h_meta = nullptr;
   cudaEvent_t done = nullptr;
+  cudaEvent_t prof[3] = {nullptr, nullptr, nullptr};
+  bool profiled = false, scanned = false;
   int64_t task_id = -1;
   int state = SLOT_FREE;
   SlotMeta meta{};
@@ -78,6 +80,7 @@ struct saber_query {
   std::string err;
   saber_stats stats{};
   std::vector<std::pair<void *, size_t>> registered;
+  std::vector<void *> prereg;   // registered by someone else: never unregistered here
   std::mutex mu;
   int64_t *d_tmp = nullptr;
 };
@@ -158,6 +161,7 @@ static saber_status build_plan(saber_query *q, const saber_schema *sc, const sab
   p.win_kind = w->kind == SABER_WIN_TIME ? WK_TIME : WK_COUNT;
   p.s = w->size; p.l = w->slide; p.T0 = w->kind == SABER_WIN_TIME ? w->origin : 0;
   p.g = gcd64(p.s, p.l); p.K = p.s / p.g; p.L = p.l / p.g;
+  p.g_inv = 1.0 / (double)p.g;
 
   p.npred = op->npred;
   for (int i = 0; i < op->npred; ++i) {
@@ -289,13 +293,13 @@ static saber_status size_plan(saber_query *q) {
     else R = std::min(next_pow2(need + (1 << 20)), floor_pow2(std::max<int64_t>(budget / slot_bytes, 1)));
     if (R < need + 16) R = next_pow2(need + 16);
     p.R = R;
-    // phase-1 warp-private table (12 KiB per warp)
-    const int budget_w = 12 * 1024;
-    const int ed = 4 + 8 * p.nf, eh = 12 + 8 * p.nf;
+    // phase-1 warp-private tables (5 KiB per warp; fields padded to the NF template)
+    const int budget_w = 5 * 1024;
+    const int nft = p.nf <= 1 ? 1 : p.nf <= 2 ? 2 : p.nf <= 4 ? 4 : 8;
+    const int ed = 4 + 8 * nft, eh = 12 + 8 * nft;
     if (p.key_mode != KM_HASH && p.C * 2 * ed <= budget_w) {
       p.local_direct = 1;
-      int te = budget_w / ed;
-      p.local_pl = (int)(te / p.C);
+      p.local_pl = (int)std::min<int64_t>(1024, budget_w / (ed * p.C));
       p.local_entries = p.local_pl * (int)p.C;
       p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
     } else {
@@ -314,7 +318,8 @@ static saber_status size_plan(saber_query *q) {
       if (sb > p.C) sb = (int)p.C;
       p.SB = sb;
       p.S = (int)((p.C + sb - 1) / sb);
-      p.p2_smem = gpb * sb * 8 * (1 + p.nf);
+      p.p2_smem = 0;        // van Herk windows keep no state in shared memory
+      (void)gpb; (void)smem_budget;
     } else {
       p.GS = 256;
       p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + p.nf)));
@@ -347,7 +352,9 @@ static saber_status size_plan(saber_query *q) {
       off += ((p.rows_cap * p.col_bytes[i]) + 255) & ~255ll;
     }
   } else {
-    p.carry_cap = p.win_kind == WK_COUNT ? p.s + p.l + 16 : T + 16;
+    // the uncovered tail is < s tuples (count) or spans < s time units (time,
+    // rate unknown: sized generously, overflow is SABER_ECAPACITY)
+    p.carry_cap = p.win_kind == WK_COUNT ? p.s + p.l + 16 : std::max<int64_t>(T, 1 << 20) + 16;
     p.rows_cap = T + p.carry_cap;
     p.win_cap = p.win_kind == WK_COUNT ? T / p.l + 4 : T + 4;
     p.S = 1;
@@ -368,6 +375,10 @@ static saber_status alloc_query(saber_query *q) {
   if (p.nagg > 0) {
     CK(cudaMalloc(&q->qd.table, (size_t)p.R * p.slot_words * 8));
     CK(cudaMalloc(&q->qd.pane_ts, (size_t)p.R * 8));
+    if (p.key_mode != KM_HASH) {
+      CK(cudaMalloc(&q->qd.vh_pre, (size_t)p.R * p.slot_words * 8));
+      CK(cudaMalloc(&q->qd.vh_suf, (size_t)p.R * p.slot_words * 8));
+    }
   } else {
     q->qd.carry_cap = p.carry_cap;
     CK(cudaMalloc(&q->qd.carry[0], (size_t)p.carry_cap * p.tuple_bytes));
@@ -391,6 +402,8 @@ static saber_status alloc_query(saber_query *q) {
       CK(cudaMallocHost(&s.h_hdr, (size_t)p.win_cap * sizeof(saber_win_hdr)));
     }
     CK(cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
+    if (q->cfg.profile)
+      for (auto &e : s.prof) CK(cudaEventCreate(&e));
   }
   CK(set_kernel_attributes(p));
   CK(cudaDeviceGetAttribute(&q->nsm, cudaDevAttrMultiProcessorCount, q->device));
@@ -422,11 +435,18 @@ static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuple
   if (s.state != SLOT_FREE) return fail(q, SABER_EAGAIN, "no free result slot");
   const Plan &p = q->plan;
   cudaError_t e;
+  int launches = 0;
+  cudaEvent_t *evs = q->cfg.profile ? s.prof : nullptr;
   if (p.nagg > 0)
     e = launch_agg_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish, q->p1_grid,
-                        q->p2_grid, q->win_chunk, q->cs);
+                        q->p2_grid, q->win_chunk, q->cs, evs, &launches);
   else
-    e = launch_select_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish, q->sel_grid, q->cs);
+    e = launch_select_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish, q->sel_grid,
+                           q->cs, evs, &launches);
+  q->stats.kernel_launches += launches;
+  s.profiled = evs != nullptr;
+  s.scanned = (p.nagg == 0) || ntuples > 0;
+  if (s.scanned) q->stats.scan_launches += 1;
   if (e != cudaSuccess) return fail(q, SABER_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e));
   CK(cudaMemcpyAsync(s.h_meta, s.dev.meta, sizeof(SlotMeta), cudaMemcpyDeviceToHost, q->cs));
   CK(cudaEventRecord(s.done, q->cs));
@@ -506,13 +526,15 @@ void saber_query_destroy(saber_query *q) {
     cudaFree(s.dev.rows); cudaFree(s.dev.hdr); cudaFree(s.dev.counts); cudaFree(s.dev.meta);
     cudaFreeHost(s.h_meta); cudaFreeHost(s.h_rows); cudaFreeHost(s.h_hdr);
     if (s.done) cudaEventDestroy(s.done);
+    for (auto e : s.prof) if (e) cudaEventDestroy(e);
   }
   for (auto &g : q->stages) {
     cudaFreeHost(g.h); cudaFree(g.d);
     if (g.free_ev) cudaEventDestroy(g.free_ev);
   }
-  for (auto &r : q->registered) cudaHostUnregister(r.first);
-  cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
+  for (auto &r : q->registered)
+    if (std::find(q->prereg.begin(), q->prereg.end(), r.first) == q->prereg.end()) cudaHostUnregister(r.first);
+  cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.vh_pre); cudaFree(q->qd.vh_suf); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
   cudaFree(q->qd.carry[0]); cudaFree(q->qd.carry[1]); cudaFree(q->qd.tile_ctr); cudaFree(q->d_tmp);
   if (q->cs) cudaStreamDestroy(q->cs);
   if (q->h2d) cudaStreamDestroy(q->h2d);
@@ -603,6 +625,8 @@ saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t n
   CK(cudaSetDevice(q->device));
   const int64_t tbytes = q->task_tuples * p.tuple_bytes;
   const int64_t whole = ((int64_t)nbytes + q->stage_fill) / tbytes;
+  if (whole > (int64_t)q->slots.size())
+    return fail(q, SABER_EINVAL, "submit at most result_slots * task_bytes per call");
   if (whole > free_slots(q)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
   const bool reg = is_registered(q, host_tuples, nbytes);
   const unsigned char *src = (const unsigned char *)host_tuples;
@@ -644,7 +668,16 @@ saber_status saber_register_host(saber_query *q, void *ptr, size_t nbytes) {
   std::lock_guard<std::mutex> lk(q->mu);
   CK(cudaSetDevice(q->device));
   cudaError_t e = cudaHostRegister(ptr, nbytes, cudaHostRegisterDefault);
-  if (e == cudaErrorHostMemoryAlreadyRegistered) { cudaGetLastError(); return SABER_OK; }
+  cudaPointerAttributes attr{};
+  if (e != cudaSuccess && cudaPointerGetAttributes(&attr, ptr) == cudaSuccess && attr.type == cudaMemoryTypeHost)
+    e = cudaErrorHostMemoryAlreadyRegistered;
+  if (e == cudaErrorHostMemoryAlreadyRegistered) {   // already page-locked (e.g. torch pinned memory)
+    cudaGetLastError();
+    q->registered.emplace_back(nullptr, 0);
+    q->registered.back() = {ptr, nbytes};
+    q->prereg.push_back(ptr);
+    return SABER_OK;
+  }
   if (e != cudaSuccess) return fail(q, SABER_ECUDA, std::string("cudaHostRegister: ") + cudaGetErrorString(e));
   q->registered.emplace_back(ptr, nbytes);
   return SABER_OK;
@@ -696,6 +729,13 @@ saber_status saber_results_poll(saber_query *q, saber_results *out, int32_t time
   }
   s.meta = *s.h_meta;
   const Plan &p = q->plan;
+  if (s.profiled) {
+    float a = 0, b = 0;
+    if (cudaEventElapsedTime(&a, s.prof[0], s.prof[1]) == cudaSuccess && s.scanned) q->stats.scan_ms += a;
+    if (cudaEventElapsedTime(&b, s.prof[1], s.prof[2]) == cudaSuccess) q->stats.assemble_ms += b;
+    cudaGetLastError();
+    s.profiled = false;
+  }
   if (s.meta.error) {
     q->sticky = status_from_err(s.meta.error);
     return fail(q, q->sticky, err_text(s.meta.error));
@@ -758,6 +798,18 @@ saber_status saber_query_sync(saber_query *q) {
   if (!q) return SABER_EINVAL;
   CK(cudaSetDevice(q->device));
   CK(cudaStreamSynchronize(q->cs));
+  return SABER_OK;
+}
+
+saber_status saber_query_record(saber_query *q, void *cuda_stream) {
+  if (!q) return SABER_EINVAL;
+  std::lock_guard<std::mutex> lk(q->mu);
+  CK(cudaSetDevice(q->device));
+  cudaEvent_t ev;
+  CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+  CK(cudaEventRecord(ev, q->cs));
+  CK(cudaStreamWaitEvent((cudaStream_t)cuda_stream, ev, 0));
+  CK(cudaEventDestroy(ev));
   return SABER_OK;
 }
 

@@ -66,7 +66,8 @@ class Config(C.Structure):
     _fields_ = [("device", C.c_int32), ("task_bytes", C.c_int64), ("pipeline_depth", C.c_int32),
                 ("result_mode", C.c_int32), ("result_bytes", C.c_int64), ("hash_capacity", C.c_int64),
                 ("max_panes", C.c_int64), ("base_index", C.c_int64), ("first_window", C.c_int64),
-                ("emit_on_finish", C.c_int32), ("result_slots", C.c_int32), ("reserved", C.c_int32 * 6)]
+                ("emit_on_finish", C.c_int32), ("result_slots", C.c_int32), ("profile", C.c_int32),
+                ("reserved", C.c_int32 * 5)]
 
 
 class WinHdr(C.Structure):
@@ -86,7 +87,8 @@ class Stats(C.Structure):
     _fields_ = [("tasks", C.c_int64), ("tuples", C.c_int64), ("bytes_in", C.c_int64), ("windows", C.c_int64),
                 ("rows", C.c_int64), ("out_tuples", C.c_int64), ("tasks_pending", C.c_int64),
                 ("last_complete", C.c_int64), ("last_opening", C.c_int64), ("last_closing", C.c_int64),
-                ("last_pending", C.c_int64)]
+                ("last_pending", C.c_int64), ("kernel_launches", C.c_int64), ("scan_launches", C.c_int64),
+                ("scan_ms", C.c_double), ("assemble_ms", C.c_double)]
 
 
 # every function declared in include/saber.h: name -> (restype, argtypes)
@@ -101,6 +103,7 @@ SIGNATURES = {
     "saber_results_release": (C.c_int, [C.c_void_p, C.POINTER(Results)]),
     "saber_query_stats": (C.c_int, [C.c_void_p, C.POINTER(Stats)]),
     "saber_query_sync": (C.c_int, [C.c_void_p]),
+    "saber_query_record": (C.c_int, [C.c_void_p, C.c_void_p]),
     "saber_query_destroy": (None, [C.c_void_p]),
     "saber_last_error": (C.c_char_p, [C.c_void_p]),
     "saber_partition_plan": (C.c_int, [C.POINTER(Schema), C.POINTER(Window), C.c_void_p, C.c_int64, C.c_int64,
@@ -193,7 +196,7 @@ class Query:
 
     def __init__(self, spec, device=None, task_bytes=64 << 20, result_mode=RESULTS_HOST, result_bytes=0,
                  hash_capacity=0, max_panes=0, base_index=0, first_window=0, emit_on_finish=True,
-                 result_slots=8, pipeline_depth=3):
+                 result_slots=8, pipeline_depth=3, profile=False):
         self.L = lib()
         self.m = _Marshalled(spec)
         self.spec = spec
@@ -210,6 +213,7 @@ class Query:
         cfg.first_window = int(first_window)
         cfg.emit_on_finish = 1 if emit_on_finish else 0
         cfg.result_slots = int(result_slots)
+        cfg.profile = 1 if profile else 0
         self.cfg = cfg
         h = C.c_void_p()
         _check(self.L.saber_query_create(C.byref(self.m.schema), C.byref(self.m.op), C.byref(self.m.window),
@@ -259,6 +263,9 @@ class Query:
                                       ("nrows", "<i4"), ("flags", "<i4")])
             if nw and r.hdr:
                 C.memmove(hdr.ctypes.data, r.hdr, nw * 32)
+            elif nw:   # σ/π (IStream) slices carry no per-window headers: ids only
+                hdr["window_id"] = r.first_window + np.arange(nw)
+                hdr["ts"] = -1
             keys, vals, tuples = [], [], b""
             if self.m.aggs_spec:
                 for c in range(self.m.nkeys):
@@ -287,6 +294,10 @@ class Query:
     def sync(self):
         _check(self.L.saber_query_sync(self.h), self.h)
 
+    def record(self, stream=0):
+        """Make CUDA stream `stream` wait for everything enqueued on this query."""
+        _check(self.L.saber_query_record(self.h, C.c_void_p(stream)), self.h)
+
     def last_error(self):
         m = self.L.saber_last_error(self.h)
         return m.decode() if m else ""
@@ -310,6 +321,7 @@ class Query:
             np.asarray(data).view(np.uint8).reshape(-1)
         tb = self.tuple_bytes
         chunk = chunk_bytes or self.cfg.task_bytes
+        chunk = min(chunk, self.cfg.task_bytes * max(1, self.cfg.result_slots - 1))
         chunk = max(tb, (chunk // tb) * tb)
         slices = []
         off = 0
