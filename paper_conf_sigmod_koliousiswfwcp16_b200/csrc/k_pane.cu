@@ -71,6 +71,15 @@ __device__ __forceinline__ int64_t fdiv(int64_t x, int64_t d, double inv) {
   return x / d;
 }
 
+// pane division: shift for power-of-two pane lengths, reciprocal otherwise
+__device__ __forceinline__ int64_t pdiv(const Plan &p, int64_t x) {
+  return p.g_shift >= 0 ? (x >> p.g_shift) : fdiv(x, p.g, p.g_inv);
+}
+__device__ __forceinline__ uint64_t shfl_up64(uint64_t v) {
+  const uint32_t lo = __shfl_up_sync(kFull, (uint32_t)v, 1), hi = __shfl_up_sync(kFull, (uint32_t)(v >> 32), 1);
+  return ((uint64_t)hi << 32) | lo;
+}
+
 // field access straight from the shared-memory tuple (runtime byte offsets)
 __device__ __forceinline__ int64_t s_int(const unsigned char *t, int word, int type) {
   return type == T_I32 ? (int64_t) * (const int32_t *)(t + 4 * word) : *(const int64_t *)(t + 4 * word);
@@ -126,8 +135,13 @@ __device__ __forceinline__ uint64_t s_field(const Field &f, const unsigned char 
   }
 }
 
+__device__ __forceinline__ uint64_t fadd64(uint64_t a, uint64_t b) {
+  return (uint64_t)__double_as_longlong(__longlong_as_double((long long)a) + __longlong_as_double((long long)b));
+}
+
 // leaders of each equal-key lane group receive the group's combined fields
-template <int NF>
+// (FAST: every field is an fp64 sum, combine = add, identity = +0.0)
+template <int NF, bool FAST>
 __device__ __forceinline__ void warp_combine(const Plan &p, bool act, unsigned m, uint64_t (&fv)[NF]) {
   const int lane = threadIdx.x & 31;
   const int leader = m ? __ffs(m) - 1 : -1;
@@ -145,11 +159,12 @@ __device__ __forceinline__ void warp_combine(const Plan &p, bool act, unsigned m
       const bool mine = act && leader == L;
 #pragma unroll
       for (int i = 0; i < NF; ++i) {
-        if (i >= p.nf) break;
-        const int kind = p.field[i].kind;
-        uint64_t v = mine ? fv[i] : field_identity(kind);
+        if (!FAST && i >= p.nf) break;
+        const int kind = FAST ? FK_SUM_F : p.field[i].kind;
+        uint64_t v = mine ? fv[i] : (FAST ? 0ull : field_identity(kind));
 #pragma unroll
-        for (int x = 16; x; x >>= 1) v = field_combine(kind, v, shfl_xor64(v, x));
+        for (int x = 16; x; x >>= 1)
+          v = FAST ? fadd64(v, shfl_xor64(v, x)) : field_combine(kind, v, shfl_xor64(v, x));
         if (lane == L) fv[i] = v;
       }
     }
@@ -164,9 +179,9 @@ __device__ __forceinline__ void warp_combine(const Plan &p, bool act, unsigned m
       rest &= rest - 1;
 #pragma unroll
       for (int i = 0; i < NF; ++i) {
-        if (i >= p.nf) break;
+        if (!FAST && i >= p.nf) break;
         const uint64_t o = shfl64(fv[i], s);
-        if (ok) acc[i] = field_combine(p.field[i].kind, acc[i], o);
+        if (ok) acc[i] = FAST ? fadd64(acc[i], o) : field_combine(p.field[i].kind, acc[i], o);
       }
     }
 #pragma unroll
@@ -192,8 +207,8 @@ __device__ __forceinline__ void flush_entry(const Plan &p, State *st, uint64_t *
     if (i < p.nf) red_field(p.field[i].kind, &base[fld_off(p, i) + idx], fv[i]);
 }
 
-template <bool HASHED, int WK, int NF>
-__global__ void __launch_bounds__(kP1Threads, 2)
+template <bool HASHED, int WK, int NF, bool FAST>
+__global__ void __launch_bounds__(kP1Threads, HASHED ? 2 : 3)
 k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
            uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
   extern __shared__ __align__(128) unsigned char smem[];
@@ -302,23 +317,18 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     const int64_t spos = pos0 + lo + k * ST;             // global position of stage tuple 0
     int64_t pf, pl;                                      // stage pane range (CTA-uniform)
     if (WK == WK_COUNT) {
-      pf = fdiv(spos, p.g, p.g_inv);
-      pl = fdiv(spos + ntup - 1, p.g, p.g_inv);
+      pf = pdiv(p, spos);
+      pl = pdiv(p, spos + ntup - 1);
     } else {
       const int64_t t0 = *(const int64_t *)(sb + 4 * tsw), t1 = *(const int64_t *)(sb + (ntup - 1) * tb + 4 * tsw);
-      pf = t0 >= p.T0 ? fdiv(t0 - p.T0, p.g, p.g_inv) : 0;
-      pl = t1 >= p.T0 ? fdiv(t1 - p.T0, p.g, p.g_inv) : -1;
+      pf = t0 >= p.T0 ? pdiv(p, t0 - p.T0) : 0;
+      pl = t1 >= p.T0 ? pdiv(p, t1 - p.T0) : -1;
     }
     if (pf < min_pane) pf = min_pane;
     const int ib = wid * per_warp;
     const int ie = ib + per_warp < ntup ? ib + per_warp : ntup;
-    // K1 order check, once per tuple
-    for (int i = ib + lane; i < ie; i += 32) {
-      const int64_t tau = *(const int64_t *)(sb + i * tb + 4 * tsw);
-      const int64_t up = i > 0 ? *(const int64_t *)(sb + (i - 1) * tb + 4 * tsw) : prev_last;
-      if (tau < up) err |= ERR_ORDER;
-      if (tau < 0) err |= ERR_TS;
-    }
+    // τ of the tuple before this warp's slice (K1 order check, done in the first round)
+    int64_t carry_tau = (ib > 0 && ib <= ntup) ? *(const int64_t *)(sb + (ib - 1) * tb + 4 * tsw) : prev_last;
     int64_t cur = pf;
     bool first_round = true;
     while (cur <= pl) {
@@ -329,43 +339,82 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         pbase = cur;
       }
       const int64_t wend = pbase + PL;
+      const int64_t wlo = pbase > min_pane ? pbase : min_pane;
+      const bool all_in = (pf >= wlo) & (pl < wend);    // CTA-uniform: no per-tuple window test
+      int64_t cp = 0, cr = 0;                            // count windows: (pane, rem) of this lane's tuple
+      if (WK == WK_COUNT) {
+        const int64_t pos = spos + ib + lane;
+        cp = pdiv(p, pos);
+        cr = pos - cp * p.g;
+      }
       for (int i0 = ib; i0 < ie; i0 += 32) {
         const int i = i0 + lane;
         bool valid = i < ie;
         const unsigned char *t = sb + (valid ? i : ib) * tb;
+        const int64_t tau = *(const int64_t *)(t + 4 * tsw);
+        if (first_round) {
+          // K1: τ non-decreasing (L347-349) and non-negative (L349-350); the
+          // predecessor of lane 0 is the previous iteration's lane 31
+          const int64_t up0 = (int64_t)shfl_up64((uint64_t)tau);
+          const int64_t up = lane == 0 ? carry_tau : up0;
+          if (valid & (tau < up)) err |= ERR_ORDER;
+          if (valid & (tau < 0)) err |= ERR_TS;
+          carry_tau = (int64_t)shfl64((uint64_t)tau, 31);
+        }
         int64_t pane;
         if (WK == WK_COUNT) {
-          const int64_t pos = spos + i;
-          pane = fdiv(pos, p.g, p.g_inv);
-          if (valid && first_round && pos == pane * p.g && pane >= min_pane)
-            pane_ts[pane & (p.R - 1)] = *(const int64_t *)(t + 4 * tsw);
+          pane = cp;
+          if (first_round && valid && cr == 0 && pane >= min_pane) pane_ts[pane & (p.R - 1)] = tau;
+          cr += 32;
+          while (cr >= p.g) { cr -= p.g; ++cp; }
         } else {
-          const int64_t tau = *(const int64_t *)(t + 4 * tsw);
           valid &= tau >= p.T0;
-          pane = tau >= p.T0 ? fdiv(tau - p.T0, p.g, p.g_inv) : -1;
+          pane = tau >= p.T0 ? pdiv(p, tau - p.T0) : -1;
         }
-        valid &= (pane >= pbase) & (pane < wend) & (pane >= min_pane);
+        if (!all_in) valid &= (pane >= pbase) & (pane < wend) & (pane >= min_pane);
         if (p.npred && valid) valid &= s_preds(p, t);
-        const uint64_t key = s_key(p, t, valid, err);
+        uint64_t key;
         uint64_t fv[NF];
+        if (FAST) {
+          // all fields are fp64 sums of f32 columns; at most one int32 key column, div 1
+          if (p.key_mode == KM_GLOBAL) key = 0;
+          else {
+            const int32_t v = *(const int32_t *)(t + 4 * p.key[0].word);
+            if (p.key_pack == KP_RADIX) {
+              if ((uint32_t)v >= (uint32_t)p.key[0].domain) {     // domain < 2^31 on the fast path
+                if (valid) err |= ERR_KEY;
+                valid = false;
+              }
+              key = (uint64_t)(uint32_t)v;
+            } else {
+              key = (uint64_t)(int64_t)v ^ 0x8000000000000000ull;
+            }
+          }
 #pragma unroll
-        for (int f = 0; f < NF; ++f) fv[f] = (f < p.nf) ? s_field(p.field[f], t) : 0;
+          for (int f = 0; f < NF; ++f)
+            fv[f] = (uint64_t)__double_as_longlong((double)*(const float *)(t + 4 * p.field[f].word));
+        } else {
+          key = s_key(p, t, valid, err);
+#pragma unroll
+          for (int f = 0; f < NF; ++f) fv[f] = (f < p.nf) ? s_field(p.field[f], t) : 0;
+        }
         const unsigned actm = __ballot_sync(kFull, valid);
         if (!actm) continue;
         if (!HASHED) {
           const int e = valid ? (int)(pane - pbase) * C + (int)key : -1 - lane;
           const unsigned m = __match_any_sync(kFull, e) & actm;
-          warp_combine<NF>(p, valid, m, fv);
+          warp_combine<NF, FAST>(p, valid, m, fv);
           if (valid && (__ffs(m) - 1) == lane) {
             tcnt[e] += (uint32_t)__popc(m);
 #pragma unroll
             for (int f = 0; f < NF; ++f)
-              if (f < p.nf) tf[f * TE + e] = field_combine(p.field[f].kind, tf[f * TE + e], fv[f]);
+              if (FAST) tf[f * TE + e] = fadd64(tf[f * TE + e], fv[f]);
+              else if (f < p.nf) tf[f * TE + e] = field_combine(p.field[f].kind, tf[f * TE + e], fv[f]);
           }
         } else {
           if (occ + 32 > TE / 2) flush_hashed();
           const unsigned m = __match_any_sync(kFull, (unsigned long long)key) & actm;
-          warp_combine<NF>(p, valid, m, fv);
+          warp_combine<NF, FAST>(p, valid, m, fv);
           bool ins = false;
           if (valid && (__ffs(m) - 1) == lane) {
             uint32_t h = (uint32_t)fmix64(key) & (uint32_t)(TE - 1);
@@ -383,7 +432,8 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
             tcnt[h] += (uint32_t)__popc(m);
 #pragma unroll
             for (int f = 0; f < NF; ++f)
-              if (f < p.nf) tf[f * TE + h] = field_combine(p.field[f].kind, tf[f * TE + h], fv[f]);
+              if (FAST) tf[f * TE + h] = fadd64(tf[f * TE + h], fv[f]);
+              else if (f < p.nf) tf[f * TE + h] = field_combine(p.field[f].kind, tf[f * TE + h], fv[f]);
           }
           occ += __popc(__ballot_sync(kFull, ins));
         }
@@ -397,10 +447,10 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
       for (int i = ib + lane; i < ie; i += 32) {
         const unsigned char *t = sb + i * tb;
         int64_t pane;
-        if (WK == WK_COUNT) pane = fdiv(spos + i, p.g, p.g_inv);
+        if (WK == WK_COUNT) pane = pdiv(p, spos + i);
         else {
           const int64_t tau = *(const int64_t *)(t + 4 * tsw);
-          pane = tau >= p.T0 ? fdiv(tau - p.T0, p.g, p.g_inv) : -1;
+          pane = tau >= p.T0 ? pdiv(p, tau - p.T0) : -1;
         }
         if (pane >= wend) atomicMin(&s_next, (long long)pane);
       }
@@ -428,18 +478,20 @@ int p1_nf_template(int nf) { return nf <= 1 ? 1 : nf <= 2 ? 2 : nf <= 4 ? 4 : 8;
 int p1_smem_bytes(const Plan &p) { return kStages * kStageBytes + 2 * kStages * 8 + kP1Warps * p.local_bytes; }
 
 template <bool H, int WK>
-static void *p1_nf(int nf) {
+static void *p1_nf(int nf, bool fast) {
+  if (fast) return nf <= 1 ? (void *)k_pane_agg<H, WK, 1, true> : (void *)k_pane_agg<H, WK, 2, true>;
   switch (p1_nf_template(nf)) {
-    case 1: return (void *)k_pane_agg<H, WK, 1>;
-    case 2: return (void *)k_pane_agg<H, WK, 2>;
-    case 4: return (void *)k_pane_agg<H, WK, 4>;
-    default: return (void *)k_pane_agg<H, WK, 8>;
+    case 1: return (void *)k_pane_agg<H, WK, 1, false>;
+    case 2: return (void *)k_pane_agg<H, WK, 2, false>;
+    case 4: return (void *)k_pane_agg<H, WK, 4, false>;
+    default: return (void *)k_pane_agg<H, WK, 8, false>;
   }
 }
 void *p1_kernel(const Plan &p) {
   const bool h = !p.local_direct;
-  if (p.win_kind == WK_COUNT) return h ? p1_nf<true, WK_COUNT>(p.nf) : p1_nf<false, WK_COUNT>(p.nf);
-  return h ? p1_nf<true, WK_TIME>(p.nf) : p1_nf<false, WK_TIME>(p.nf);
+  const bool f = p.fast_path;
+  if (p.win_kind == WK_COUNT) return h ? p1_nf<true, WK_COUNT>(p.nf, f) : p1_nf<false, WK_COUNT>(p.nf, f);
+  return h ? p1_nf<true, WK_TIME>(p.nf, f) : p1_nf<false, WK_TIME>(p.nf, f);
 }
 
 int p1_blocks_per_sm(const Plan &p) {

@@ -141,8 +141,16 @@ k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t
   const int64_t per = (nw + blockDim.x - 1) / blockDim.x;
   const int64_t a = (int64_t)tid * per, b = (a + per < nw) ? a + per : nw;
   int64_t local = 0;
-  for (int64_t j = a; j < b; ++j)
-    for (int s = 0; s < S; ++s) local += counts[j * S + s];
+  if (S == 1 && per <= 16) {
+    int64_t v[16];                           // issue all loads before summing (one latency)
+#pragma unroll
+    for (int k = 0; k < 16; ++k) v[k] = (a + k < b) ? counts[a + k] : 0;
+#pragma unroll
+    for (int k = 0; k < 16; ++k) local += v[k];
+  } else {
+    for (int64_t j = a; j < b; ++j)
+      for (int s = 0; s < S; ++s) local += counts[j * S + s];
+  }
   int64_t x = local;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
@@ -180,6 +188,7 @@ k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t
   }
   if (tid == blockDim.x - 1) {
     meta->nrows = run;
+    st->sel_rows = run;
     if (run > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
   }
 }
@@ -199,6 +208,7 @@ __global__ void k_task_end(const Plan p, State *st, SlotMeta *meta) {
     st->carry_sel ^= 1;
     st->zero_lo = st->zero_hi = 0;
   } else {
+    meta->nrows = st->sel_rows;     // written by the window pass (fused) or k_win_scan
     meta->ntuples = 0;
   }
   st->J0 = st->J1;

@@ -33,7 +33,8 @@ __device__ __forceinline__ uint64_t combine_cnt_or_field(const Plan &p, int f, u
   return f < 0 ? a + b : field_combine(p.field[f].kind, a, b);
 }
 
-// one thread per (block of K panes, slot)
+// one thread per (block of K panes, table word, direction): the DENSE/GLOBAL pane
+// slot is [cnt C][f0 C][f1 C].., identical in the table and in the van Herk arrays
 __global__ void __launch_bounds__(256)
 k_vh_build(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
            uint64_t *__restrict__ pre, uint64_t *__restrict__ suf) {
@@ -41,32 +42,240 @@ k_vh_build(const Plan p, const State *__restrict__ st, const uint64_t *__restric
   if (J1 <= J0) return;
   const int64_t lo = J0 * p.L, hi = (J1 - 1) * p.L + p.K - 1;
   const int64_t b0 = lo / p.K, b1 = hi / p.K;
-  const int64_t items = (b1 - b0 + 1) * p.C;
-  const int64_t co = cnt_off(p);
+  const int64_t words = p.slot_words;                 // C * (1 + nf)
+  const int64_t items = (b1 - b0 + 1) * words * 2;
+  const int64_t Rm = p.R - 1;
   for (int64_t it = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; it < items; it += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = b0 + it / p.C;
-    const int64_t slot = it % p.C;
+    const int64_t w = it % words;
+    const int64_t rest = it / words;
+    const bool prefix = rest & 1;
+    const int64_t b = b0 + (rest >> 1);
+    const int f = (int)(w / p.C) - 1;                   // -1: count
+    const int kind = f < 0 ? -1 : p.field[f].kind;
     const int64_t bs = b * p.K, be = (bs + p.K - 1 < hi) ? bs + p.K - 1 : hi;
-    for (int f = -1; f < p.nf; ++f) {
-      const int64_t src = (f < 0 ? co : fld_off(p, f)) + slot;
-      const int64_t dst = (f < 0 ? 0 : vh_off(p, f)) + slot;
-      const uint64_t id = f < 0 ? 0ull : field_identity(p.field[f].kind);
-      if (bs >= lo) {                       // prefix arrays are only read for blocks starting >= lo
-        uint64_t acc = id;
-        for (int64_t q = bs; q <= be; ++q) {
-          const int64_t r = (q & (p.R - 1)) * p.slot_words;
-          acc = combine_cnt_or_field(p, f, acc, table[r + src]);
-          pre[(q & (p.R - 1)) * p.slot_words + dst] = acc;
-        }
+    uint64_t acc = kind < 0 ? 0ull : field_identity(kind);
+    if (prefix) {
+      if (bs < lo) continue;                             // prefixes are only read for blocks starting >= lo
+#pragma unroll 4
+      for (int64_t q = bs; q <= be; ++q) {
+        const int64_t r = (q & Rm) * words + w;
+        const uint64_t v = table[r];
+        acc = kind < 0 ? acc + v : field_combine(kind, acc, v);
+        pre[r] = acc;
       }
-      uint64_t acc = id;
+    } else {
       const int64_t qlo = bs > lo ? bs : lo;
+#pragma unroll 4
       for (int64_t q = be; q >= qlo; --q) {
-        const int64_t r = (q & (p.R - 1)) * p.slot_words;
-        acc = combine_cnt_or_field(p, f, acc, table[r + src]);
-        suf[(q & (p.R - 1)) * p.slot_words + dst] = acc;
+        const int64_t r = (q & Rm) * words + w;
+        const uint64_t v = table[r];
+        acc = kind < 0 ? acc + v : field_combine(kind, acc, v);
+        suf[r] = acc;
       }
     }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Single pass over the windows closed by a task (DENSE/GLOBAL): CTAs take window
+// chunks in ticket order, count the rows of every (window, slab) item, obtain
+// the chunk's output offset by decoupled look-back over earlier chunks, write
+// the window headers and then the rows.  Replaces count pass + scan + emit pass.
+__device__ __forceinline__ uint64_t lb_ld(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void lb_st(uint64_t *p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v));
+}
+__device__ __forceinline__ uint64_t lb_pack(uint64_t epoch, uint64_t flag, uint64_t v) {
+  return ((epoch & 0xffffffull) << 40) | (flag << 38) | (v & ((1ull << 38) - 1));
+}
+
+constexpr int kFusedMaxItems = 256;
+
+template <int GS>
+__global__ void __launch_bounds__(256)
+k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre, const uint64_t *__restrict__ suf,
+            const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
+            uint64_t *__restrict__ status, int *__restrict__ ticket, int WC) {
+  constexpr int gpb = 256 / GS;
+  __shared__ int s_cnt[kFusedMaxItems];
+  __shared__ int s_off[kFusedMaxItems];
+  __shared__ int s_total;
+  __shared__ int64_t s_base;
+  __shared__ int s_t;
+  const int grp = threadIdx.x / GS, gt = threadIdx.x % GS, lane = threadIdx.x & 31;
+  const int SB = p.SB, S = p.S;
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  if (nw <= 0) return;
+  const uint64_t epoch = (uint64_t)st->tile_epoch;
+  const int64_t nchunks = (nw + WC - 1) / WC;
+  for (;;) {
+    if (threadIdx.x == 0) s_t = atomicAdd(ticket, 1);
+    __syncthreads();
+    const int64_t t = s_t;
+    if (t >= nchunks) break;
+    const int64_t ja = J0 + t * WC;
+    const int nwc = (int)((J1 - ja) < WC ? (J1 - ja) : WC);
+    const int nitems = nwc * S;
+    // pass 1: rows per (window, slab) item
+    for (int it0 = 0; it0 < nitems; it0 += gpb) {
+      const int it = it0 + grp;
+      int my = 0;
+      if (it < nitems) {
+        const int64_t j = ja + it / S;
+        const int slab = it % S;
+        const int64_t slot0 = (int64_t)slab * SB;
+        const int nslot = (int)((p.C - slot0) < SB ? (p.C - slot0) : SB);
+        const int64_t a = j * p.L;
+        const bool aligned = (a % p.K) == 0;
+        const uint64_t *sa = suf + (a & (p.R - 1)) * p.slot_words + slot0;
+        const uint64_t *pb = pre + ((a + p.K - 1) & (p.R - 1)) * p.slot_words + slot0;
+        for (int s = gt; s < nslot; s += GS) {
+          const int64_t c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
+          if (c <= 0) continue;
+          if (p.nhave) {
+            uint64_t fv[kMaxField];
+            for (int f = 0; f < p.nf; ++f) {
+              const uint64_t x = sa[vh_off(p, f) + s];
+              fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
+            }
+            if (!having_ok(p, c, fv)) continue;
+          }
+          ++my;
+        }
+      }
+      if (GS == 32) {
+#pragma unroll
+        for (int o = 16; o; o >>= 1) my += __shfl_xor_sync(kFull, my, o);
+        if (gt == 0 && it < nitems) s_cnt[it] = my;
+      } else {
+        my = __reduce_add_sync(kFull, (unsigned)my);
+        __shared__ int s_part[8];
+        if (lane == 0) s_part[threadIdx.x >> 5] = my;
+        __syncthreads();
+        if (threadIdx.x == 0 && it < nitems) {
+          int sum = 0;
+          for (int w = 0; w < 8; ++w) sum += s_part[w];
+          s_cnt[it] = sum;
+        }
+        __syncthreads();
+      }
+    }
+    __syncthreads();
+    // exclusive scan of the chunk's item counts (warp 0)
+    if (threadIdx.x < 32) {
+      int run = 0;
+      for (int b = 0; b < nitems; b += 32) {
+        const int v = (b + lane < nitems) ? s_cnt[b + lane] : 0;
+        int x = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(kFull, x, o);
+          if (lane >= o) x += y;
+        }
+        if (b + lane < nitems) s_off[b + lane] = run + x - v;
+        run += __shfl_sync(kFull, x, 31);
+      }
+      if (lane == 0) s_total = run;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      const uint64_t total = (uint64_t)s_total;
+      int64_t excl = 0;
+      if (t == 0) {
+        lb_st(&status[0], lb_pack(epoch, 2, total));
+      } else {
+        lb_st(&status[t], lb_pack(epoch, 1, total));
+        for (int64_t i = t - 1;;) {
+          const uint64_t sv = lb_ld(&status[i]);
+          const uint64_t flag = (sv >> 38) & 3ull;
+          if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
+          excl += (int64_t)(sv & ((1ull << 38) - 1));
+          if (flag == 2) break;
+          --i;
+        }
+        lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
+      }
+      s_base = excl;
+      if (t == nchunks - 1) {
+        st->sel_rows = excl + (int64_t)total;
+        if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+      }
+    }
+    __syncthreads();
+    const int64_t base = s_base;
+    // window headers
+    for (int w = threadIdx.x; w < nwc; w += blockDim.x) {
+      const int64_t j = ja + w;
+      WinHdr h;
+      h.window_id = j;
+      h.ts = (p.win_kind == WK_TIME) ? p.T0 + j * p.l : pane_ts[(j * p.L) & (p.R - 1)];
+      h.row_offset = base + s_off[w * S];
+      int nr = 0;
+      for (int s = 0; s < S; ++s) nr += s_cnt[w * S + s];
+      h.nrows = nr;
+      h.flags = 0;
+      hdr[j - J0] = h;
+    }
+    // pass 2: rows
+    for (int it0 = 0; it0 < nitems; it0 += gpb) {
+      const int it = it0 + grp;
+      if (it >= nitems) continue;
+      const int64_t j = ja + it / S;
+      const int slab = it % S;
+      const int64_t slot0 = (int64_t)slab * SB;
+      const int nslot = (int)((p.C - slot0) < SB ? (p.C - slot0) : SB);
+      const int64_t a = j * p.L;
+      const bool aligned = (a % p.K) == 0;
+      const uint64_t *sa = suf + (a & (p.R - 1)) * p.slot_words + slot0;
+      const uint64_t *pb = pre + ((a + p.K - 1) & (p.R - 1)) * p.slot_words + slot0;
+      int64_t r = base + s_off[it];
+      for (int s0 = 0; s0 < nslot; s0 += GS) {
+        const int s = s0 + gt;
+        bool present = false;
+        int64_t c = 0;
+        uint64_t fv[kMaxField];
+        if (s < nslot) {
+          c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
+          if (c > 0) {
+            for (int f = 0; f < p.nf; ++f) {
+              const uint64_t x = sa[vh_off(p, f) + s];
+              fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
+            }
+            present = !p.nhave || having_ok(p, c, fv);
+          }
+        }
+        // rank among the group's present slots (GS = 32: one warp; GS = 256: 8 warps)
+        const unsigned bal = __ballot_sync(kFull, present);
+        int rank = __popc(bal & ((1u << lane) - 1u));
+        int tot = __popc(bal);
+        if (GS == 256) {
+          __shared__ int s_w[8];
+          __syncwarp();
+          if (lane == 0) s_w[threadIdx.x >> 5] = tot;
+          __syncthreads();
+          int before = 0, all = 0;
+          for (int w = 0; w < 8; ++w) {
+            const int x = s_w[w];
+            if (w < (threadIdx.x >> 5)) before += x;
+            all += x;
+          }
+          rank += before;
+          tot = all;
+          __syncthreads();
+        }
+        if (present) {
+          int64_t kv[kMaxKey];
+          decode_key(p, (uint64_t)(slot0 + s), kv);
+          write_row(p, rows, r + rank, kv, c, fv);
+        }
+        r += tot;
+      }
+    }
+    __syncthreads();
   }
 }
 
@@ -271,6 +480,22 @@ cudaError_t launch_windows(const Plan &p, const QueryDev &q, const SlotDev &s, b
       k_win_vh<true><<<grid, 256, 0, st>>>(p, q.st, q.vh_pre, q.vh_suf, s.counts, s.rows);
     }
   }
+  return cudaGetLastError();
+}
+
+// DENSE/GLOBAL: van Herk arrays, then one fused count + look-back + emit pass
+cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st) {
+  k_vh_build<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  const int gpb = 256 / p.GS;
+  int wc = gpb * 8 / p.S;
+  if (wc * p.S > kFusedMaxItems) wc = kFusedMaxItems / p.S;
+  if (wc < 1) wc = 1;
+  if (p.GS == 32)
+    k_win_fused<32><<<grid, 256, 0, st>>>(p, q.st, q.vh_pre, q.vh_suf, q.pane_ts, (WinHdr *)s.hdr, s.rows,
+                                          q.tile_status, q.tile_ctr, wc);
+  else
+    k_win_fused<256><<<grid, 256, 0, st>>>(p, q.st, q.vh_pre, q.vh_suf, q.pane_ts, (WinHdr *)s.hdr, s.rows,
+                                           q.tile_status, q.tile_ctr, wc);
   return cudaGetLastError();
 }
 

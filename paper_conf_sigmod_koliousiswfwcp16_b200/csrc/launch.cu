@@ -44,11 +44,15 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
     *launches += 1;
   }
   if (evs) cudaEventRecord(evs[1], st);
-  if ((e = launch_windows(p, q, s, false, p2_grid, win_chunk, st))) return e;
-  if ((e = launch_win_scan(p, q, s, st))) return e;
-  if ((e = launch_windows(p, q, s, true, p2_grid, win_chunk, st))) return e;
+  if (p.key_mode == KM_HASH) {
+    if ((e = launch_windows(p, q, s, false, p2_grid, win_chunk, st))) return e;
+    if ((e = launch_win_scan(p, q, s, st))) return e;
+    if ((e = launch_windows(p, q, s, true, p2_grid, win_chunk, st))) return e;
+  } else {
+    if ((e = launch_windows_fused(p, q, s, p2_grid, st))) return e;
+  }
   if ((e = launch_task_end(p, q, s, st))) return e;
-  *launches += p.key_mode == KM_HASH ? 4 : 5;
+  *launches += p.key_mode == KM_HASH ? 4 : 3;
   if (evs) cudaEventRecord(evs[2], st);
   return cudaGetLastError();
 }

@@ -47,6 +47,7 @@ struct Plan {
   int32_t win_kind, pad0;
   int64_t s, l, T0, g, K, L;
   double g_inv;                   // 1/g for the reciprocal division in K1
+  int32_t g_shift, pad7;          // log2(g) if g is a power of two, else -1
   // σ
   int32_t npred, pad1;
   Pred pred[kMaxPred];
@@ -73,6 +74,7 @@ struct Plan {
   int32_t local_entries;          // entries per warp
   int32_t local_pl;               // panes per direct table
   int32_t local_bytes;            // bytes per warp
+  int32_t fast_path, pad6;        // all fields fp64 sums of f32 columns, <= 1 int32 key (div 1), nf <= 2
   // phase-2 window assembly
   int32_t S, SB, GS, pad5;        // key slabs, slots per slab, threads per slab group
   int32_t state_cap, p2_smem;     // hash state entries per CTA, dynamic smem bytes

@@ -162,6 +162,10 @@ static saber_status build_plan(saber_query *q, const saber_schema *sc, const sab
   p.s = w->size; p.l = w->slide; p.T0 = w->kind == SABER_WIN_TIME ? w->origin : 0;
   p.g = gcd64(p.s, p.l); p.K = p.s / p.g; p.L = p.l / p.g;
   p.g_inv = 1.0 / (double)p.g;
+  p.g_shift = -1;
+  if ((p.g & (p.g - 1)) == 0)
+    for (int b = 0; b < 63; ++b)
+      if ((1ll << b) == p.g) p.g_shift = b;
 
   p.npred = op->npred;
   for (int i = 0; i < op->npred; ++i) {
@@ -293,10 +297,12 @@ static saber_status size_plan(saber_query *q) {
     else R = std::min(next_pow2(need + (1 << 20)), floor_pow2(std::max<int64_t>(budget / slot_bytes, 1)));
     if (R < need + 16) R = next_pow2(need + 16);
     p.R = R;
-    // phase-1 warp-private tables (5 KiB per warp; fields padded to the NF template)
-    const int budget_w = 5 * 1024;
+    // phase-1 warp-private tables, fields padded to the NF template: 2.5 KiB per
+    // warp for direct-indexed tables (3 CTAs/SM), 5 KiB for hashed ones (2 CTAs/SM)
     const int nft = p.nf <= 1 ? 1 : p.nf <= 2 ? 2 : p.nf <= 4 ? 4 : 8;
     const int ed = 4 + 8 * nft, eh = 12 + 8 * nft;
+    int budget_w = 2560;
+    if (p.key_mode == KM_HASH || p.C * 2 * ed > budget_w) budget_w = 5 * 1024;
     if (p.key_mode != KM_HASH && p.C * 2 * ed <= budget_w) {
       p.local_direct = 1;
       p.local_pl = (int)std::min<int64_t>(1024, budget_w / (ed * p.C));
@@ -307,6 +313,15 @@ static saber_status size_plan(saber_query *q) {
       p.local_entries = (int)floor_pow2(budget_w / eh);
       p.local_pl = 1;
       p.local_bytes = ((p.local_entries * eh) + 15) & ~15;
+    }
+    {
+      bool fast = p.nf <= 2;
+      for (int f = 0; f < p.nf; ++f) fast &= p.field[f].kind == FK_SUM_F && p.field[f].type == T_F32;
+      if (p.nkeys > 1) fast = false;
+      if (p.nkeys == 1)
+        fast &= p.key[0].type == T_I32 && p.key[0].div == 1 &&
+                ((p.key_pack == KP_RADIX && p.key[0].domain < (1ll << 31)) || p.key_pack == KP_BIASED64);
+      p.fast_path = fast ? 1 : 0;
     }
     // phase-2 geometry
     const int smem_budget = 96 * 1024;
@@ -378,6 +393,10 @@ static saber_status alloc_query(saber_query *q) {
     if (p.key_mode != KM_HASH) {
       CK(cudaMalloc(&q->qd.vh_pre, (size_t)p.R * p.slot_words * 8));
       CK(cudaMalloc(&q->qd.vh_suf, (size_t)p.R * p.slot_words * 8));
+      // look-back status of the fused window pass: one entry per window chunk
+      q->qd.tile_status_cap = p.win_cap + 16;
+      CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
+      CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
     }
   } else {
     q->qd.carry_cap = p.carry_cap;
