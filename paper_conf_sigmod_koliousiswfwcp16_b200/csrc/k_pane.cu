@@ -10,12 +10,16 @@
 //   σ   conjunction of `col op const` (L1320-1322)
 //   γ   GROUP BY key (dense radix index or packed 64-bit key)
 //   α   fields of the accumulator (count, fp64/int64 sums, min/max)
-// and is folded into a warp-private shared-memory table after warp-level
-// de-duplication (__match_any_sync + shuffles; no shared-memory atomics).  The
-// CTA advances over a pane window [pbase, pbase+PL) that is uniform across its
-// warps; leaving it flushes the tables into the device pane ring with L2
-// atomics (RED), after summing the eight warp tables (DIRECT mode) so each
-// (pane, key) costs one set of REDs per CTA.
+// and is folded into a shared-memory table private to its warp (or lane):
+//   LANE    tiny key counts: one table column per lane, plain read-modify-write
+//   DIRECT  small dense key domains: per-warp table indexed (pane, key), shared
+//           memory atomics (measured ~0.8 SM-cycles per update on B200)
+//   HASHED  large / unbounded domains: per-warp open-addressing table of one
+//           pane, key claimed by CAS (the paper's GPU hash, L1337-1349), atomics
+// The CTA advances over a pane window [pbase, pbase+PL) that is uniform across
+// its warps; leaving it flushes the tables into the device pane ring with L2
+// atomics (RED), after summing the warp/lane copies of an entry (LANE, DIRECT)
+// so each (pane, key) costs one set of REDs per CTA.
 #include <cuda_runtime.h>
 #include <climits>
 #include <stdint.h>
@@ -28,6 +32,7 @@ namespace sb {
 constexpr int kP1Threads = 256, kP1Warps = kP1Threads / 32;
 constexpr int kStageBytes = 16384;
 constexpr int kStages = 3;
+enum { TM_LANE = 0, TM_DIRECT = 1, TM_HASHED = 2 };
 
 // ---------------------------------------------------------------- PTX helpers
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -70,7 +75,6 @@ __device__ __forceinline__ int64_t fdiv(int64_t x, int64_t d, double inv) {
   }
   return x / d;
 }
-
 // pane division: shift for power-of-two pane lengths, reciprocal otherwise
 __device__ __forceinline__ int64_t pdiv(const Plan &p, int64_t x) {
   return p.g_shift >= 0 ? (x >> p.g_shift) : fdiv(x, p.g, p.g_inv);
@@ -139,53 +143,13 @@ __device__ __forceinline__ uint64_t fadd64(uint64_t a, uint64_t b) {
   return (uint64_t)__double_as_longlong(__longlong_as_double((long long)a) + __longlong_as_double((long long)b));
 }
 
-// leaders of each equal-key lane group receive the group's combined fields
-// (FAST: every field is an fp64 sum, combine = add, identity = +0.0)
-template <int NF, bool FAST>
-__device__ __forceinline__ void warp_combine(const Plan &p, bool act, unsigned m, uint64_t (&fv)[NF]) {
-  const int lane = threadIdx.x & 31;
-  const int leader = m ? __ffs(m) - 1 : -1;
-  const int npeer = __popc(m);
-  const int maxn = (int)__reduce_max_sync(kFull, act ? (unsigned)npeer : 0u);
-  if (maxn <= 1) return;
-  const unsigned lmask = __ballot_sync(kFull, act && leader == lane);
-  const int ng = __popc(lmask);
-  if (ng * 5 < maxn - 1) {
-    // few groups with many members (no GROUP BY, tiny G): one butterfly per group
-    unsigned rem = lmask;
-    while (rem) {
-      const int L = __ffs(rem) - 1;
-      rem &= rem - 1;
-      const bool mine = act && leader == L;
-#pragma unroll
-      for (int i = 0; i < NF; ++i) {
-        if (!FAST && i >= p.nf) break;
-        const int kind = FAST ? FK_SUM_F : p.field[i].kind;
-        uint64_t v = mine ? fv[i] : (FAST ? 0ull : field_identity(kind));
-#pragma unroll
-        for (int x = 16; x; x >>= 1)
-          v = FAST ? fadd64(v, shfl_xor64(v, x)) : field_combine(kind, v, shfl_xor64(v, x));
-        if (lane == L) fv[i] = v;
-      }
-    }
-  } else {
-    unsigned rest = act ? (m & (m - 1)) : 0u;   // peers after the leader
-    uint64_t acc[NF];
-#pragma unroll
-    for (int i = 0; i < NF; ++i) acc[i] = fv[i];
-    for (int k = 1; k < maxn; ++k) {
-      const bool ok = rest != 0u;
-      const int s = ok ? __ffs(rest) - 1 : lane;
-      rest &= rest - 1;
-#pragma unroll
-      for (int i = 0; i < NF; ++i) {
-        if (!FAST && i >= p.nf) break;
-        const uint64_t o = shfl64(fv[i], s);
-        if (ok) acc[i] = FAST ? fadd64(acc[i], o) : field_combine(p.field[i].kind, acc[i], o);
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < NF; ++i) fv[i] = acc[i];
+// shared-memory atomic update of one accumulator field
+__device__ __forceinline__ void atom_field(int kind, uint64_t *addr, uint64_t v) {
+  switch (kind) {
+    case FK_SUM_F: atomicAdd((double *)addr, __longlong_as_double((long long)v)); break;
+    case FK_SUM_I: atomicAdd((unsigned long long *)addr, (unsigned long long)v); break;
+    case FK_MIN: atomicMin((unsigned long long *)addr, (unsigned long long)v); break;
+    default: atomicMax((unsigned long long *)addr, (unsigned long long)v); break;
   }
 }
 
@@ -207,8 +171,8 @@ __device__ __forceinline__ void flush_entry(const Plan &p, State *st, uint64_t *
     if (i < p.nf) red_field(p.field[i].kind, &base[fld_off(p, i) + idx], fv[i]);
 }
 
-template <bool HASHED, int WK, int NF, bool FAST>
-__global__ void __launch_bounds__(kP1Threads, HASHED ? 2 : 3)
+template <int MODE, int WK, int NF, bool FAST>
+__global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? 3 : 2)
 k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
            uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
   extern __shared__ __align__(128) unsigned char smem[];
@@ -220,41 +184,43 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   uint64_t *full = (uint64_t *)(smem + kStages * kStageBytes);
   uint64_t *empty = full + kStages;
   unsigned char *tabs = (unsigned char *)(empty + kStages);
+  // table geometry: TE entries per warp; LANE mode stores every entry once per lane
   const int TE = p.local_entries;
+  const int CW = MODE == TM_LANE ? 32 : 1;               // copies of an entry (lanes)
   unsigned char *wt = tabs + (size_t)wid * p.local_bytes;
-  uint64_t *tkeys = (uint64_t *)wt;
-  uint64_t *tf = (uint64_t *)(wt + (HASHED ? 8 * TE : 0));
-  uint32_t *tcnt = (uint32_t *)(wt + (HASHED ? 8 * TE : 0) + (size_t)8 * TE * NF);
-  for (int e = lane; e < TE; e += 32) {
-    if (HASHED) tkeys[e] = kEmpty;
+  uint64_t *tkeys = (uint64_t *)wt;                      // HASHED only
+  uint64_t *tf = (uint64_t *)(wt + (MODE == TM_HASHED ? 8 * TE : 0));   // [NF][TE*CW]
+  uint32_t *tcnt = (uint32_t *)((unsigned char *)tf + (size_t)8 * TE * CW * NF);   // [TE*CW]
+  for (int e = lane; e < TE * CW; e += 32) {
+    if (MODE == TM_HASHED) tkeys[e] = kEmpty;
     tcnt[e] = 0;
 #pragma unroll
-    for (int f = 0; f < NF; ++f) tf[f * TE + e] = f < p.nf ? field_identity(p.field[f].kind) : 0;
+    for (int f = 0; f < NF; ++f) tf[f * TE * CW + e] = f < p.nf ? field_identity(p.field[f].kind) : 0;
   }
 
   // contiguous, stage-aligned range of this CTA
   const int64_t per = ((n + gridDim.x - 1) / gridDim.x + ST - 1) / ST * ST;
   const int64_t lo = (int64_t)blockIdx.x * per;
   const int64_t hi = lo + per < n ? lo + per : n;
-  const int64_t nst = hi > lo ? (hi - lo + ST - 1) / ST : 0;
+  const int nst = hi > lo ? (int)((hi - lo + ST - 1) / ST) : 0;
   if (tid == 0) {
     for (int i = 0; i < kStages; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], kP1Warps); }
     fence_mbar_init();
   }
   __syncthreads();
-  auto issue = [&](int64_t k) {
-    const int slot = (int)(k % kStages);
-    const int64_t cnt = (hi - lo - k * ST) < ST ? (hi - lo - k * ST) : ST;
+  auto issue = [&](int k) {
+    const int slot = k % kStages;
+    const int64_t cnt = (hi - lo - (int64_t)k * ST) < ST ? (hi - lo - (int64_t)k * ST) : ST;
     const uint32_t bytes = (uint32_t)(cnt * tb);
     mbar_expect_tx(&full[slot], bytes);
-    bulk_g2s(stages + slot * kStageBytes, tup + (lo + k * ST) * tb, bytes, &full[slot]);
+    bulk_g2s(stages + slot * kStageBytes, tup + (lo + (int64_t)k * ST) * tb, bytes, &full[slot]);
   };
   if (tid == 0)
-    for (int64_t k = 0; k < kStages && k < nst; ++k) issue(k);
+    for (int k = 0; k < kStages && k < nst; ++k) issue(k);
 
   const int64_t pos0 = st->task_pos;
   const int64_t min_pane = st->J0 * p.L;
-  const int PL = HASHED ? 1 : p.local_pl;
+  const int PL = MODE == TM_HASHED ? 1 : p.local_pl;
   const int C = (int)p.C;
   const int tsw = p.ts_word;
   int err = 0;
@@ -263,7 +229,8 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   int64_t prev_last = (lo > 0 && lo < hi) ? *(const int64_t *)(tup + (lo - 1) * tb + 4 * tsw) : INT64_MIN;
   const int per_warp = (ST + kP1Warps - 1) / kP1Warps;
 
-  auto flush_direct = [&]() {
+  // sum the warp (and lane) copies of each entry, one set of L2 REDs per entry
+  auto flush_shared = [&]() {
     __syncthreads();
     for (int e = tid; e < TE; e += kP1Threads) {
       uint32_t c = 0;
@@ -271,19 +238,21 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
 #pragma unroll
       for (int f = 0; f < NF; ++f) fv[f] = f < p.nf ? field_identity(p.field[f].kind) : 0;
       for (int w = 0; w < kP1Warps; ++w) {
-        unsigned char *ow = tabs + (size_t)w * p.local_bytes;
-        uint64_t *of = (uint64_t *)ow;
-        uint32_t *oc = (uint32_t *)(ow + (size_t)8 * TE * NF);
-        const uint32_t cw = oc[e];
-        if (!cw) continue;
-        c += cw;
-        oc[e] = 0;
+        uint64_t *of = (uint64_t *)(tabs + (size_t)w * p.local_bytes);
+        uint32_t *oc = (uint32_t *)((unsigned char *)of + (size_t)8 * TE * CW * NF);
+        for (int l = 0; l < CW; ++l) {
+          const int x = e * CW + ((l + tid) & (CW - 1));   // rotate lanes: fewer bank conflicts
+          const uint32_t cw = oc[x];
+          if (!cw) continue;
+          c += cw;
+          oc[x] = 0;
 #pragma unroll
-        for (int f = 0; f < NF; ++f)
-          if (f < p.nf) {
-            fv[f] = field_combine(p.field[f].kind, fv[f], of[f * TE + e]);
-            of[f * TE + e] = field_identity(p.field[f].kind);
-          }
+          for (int f = 0; f < NF; ++f)
+            if (f < p.nf) {
+              fv[f] = field_combine(p.field[f].kind, fv[f], of[f * TE * CW + x]);
+              of[f * TE * CW + x] = field_identity(p.field[f].kind);
+            }
+        }
       }
       if (c) flush_entry<NF>(p, st, table, pbase + e / C, (uint64_t)(e % C), c, fv, err);
     }
@@ -308,14 +277,14 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     occ = 0;
   };
 
-  for (int64_t k = 0; k < nst; ++k) {
-    const int slot = (int)(k % kStages);
+  for (int k = 0; k < nst; ++k) {
+    const int slot = k % kStages;
     const uint32_t phase = (uint32_t)((k / kStages) & 1);
     mbar_wait(&full[slot], phase);
     const unsigned char *sb = stages + slot * kStageBytes;
-    const int ntup = (int)((hi - lo - k * ST) < ST ? (hi - lo - k * ST) : ST);
-    const int64_t spos = pos0 + lo + k * ST;             // global position of stage tuple 0
-    int64_t pf, pl;                                      // stage pane range (CTA-uniform)
+    const int ntup = (int)((hi - lo - (int64_t)k * ST) < ST ? (hi - lo - (int64_t)k * ST) : ST);
+    const int64_t spos = pos0 + lo + (int64_t)k * ST;     // global position of stage tuple 0
+    int64_t pf, pl;                                        // stage pane range (CTA-uniform)
     if (WK == WK_COUNT) {
       pf = pdiv(p, spos);
       pl = pdiv(p, spos + ntup - 1);
@@ -327,26 +296,28 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     if (pf < min_pane) pf = min_pane;
     const int ib = wid * per_warp;
     const int ie = ib + per_warp < ntup ? ib + per_warp : ntup;
-    // τ of the tuple before this warp's slice (K1 order check, done in the first round)
+    // τ of the tuple before this warp's slice (K1 order check, first round)
     int64_t carry_tau = (ib > 0 && ib <= ntup) ? *(const int64_t *)(sb + (ib - 1) * tb + 4 * tsw) : prev_last;
     int64_t cur = pf;
     bool first_round = true;
     while (cur <= pl) {
       if (pbase < 0 || cur < pbase || cur >= pbase + PL) {
         if (pbase >= 0) {
-          if (HASHED) flush_hashed(); else flush_direct();
+          if (MODE == TM_HASHED) flush_hashed(); else flush_shared();
         }
         pbase = cur;
       }
       const int64_t wend = pbase + PL;
       const int64_t wlo = pbase > min_pane ? pbase : min_pane;
       const bool all_in = (pf >= wlo) & (pl < wend);    // CTA-uniform: no per-tuple window test
-      int64_t cp = 0, cr = 0;                            // count windows: (pane, rem) of this lane's tuple
+      int64_t cp = 0;                                    // count windows: pane of this lane's tuple
+      int cr = 0;                                        //                and its offset in the pane
       if (WK == WK_COUNT) {
         const int64_t pos = spos + ib + lane;
         cp = pdiv(p, pos);
-        cr = pos - cp * p.g;
+        cr = (int)(pos - cp * p.g);
       }
+      const int g32 = (int)p.g;
       for (int i0 = ib; i0 < ie; i0 += 32) {
         const int i = i0 + lane;
         bool valid = i < ie;
@@ -366,7 +337,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
           pane = cp;
           if (first_round && valid && cr == 0 && pane >= min_pane) pane_ts[pane & (p.R - 1)] = tau;
           cr += 32;
-          while (cr >= p.g) { cr -= p.g; ++cp; }
+          while (cr >= g32) { cr -= g32; ++cp; }
         } else {
           valid &= tau >= p.T0;
           pane = tau >= p.T0 ? pdiv(p, tau - p.T0) : -1;
@@ -398,25 +369,29 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
 #pragma unroll
           for (int f = 0; f < NF; ++f) fv[f] = (f < p.nf) ? s_field(p.field[f], t) : 0;
         }
-        const unsigned actm = __ballot_sync(kFull, valid);
-        if (!actm) continue;
-        if (!HASHED) {
-          const int e = valid ? (int)(pane - pbase) * C + (int)key : -1 - lane;
-          const unsigned m = __match_any_sync(kFull, e) & actm;
-          warp_combine<NF, FAST>(p, valid, m, fv);
-          if (valid && (__ffs(m) - 1) == lane) {
-            tcnt[e] += (uint32_t)__popc(m);
+        if (MODE == TM_LANE) {
+          if (valid) {       // this lane's own column: plain read-modify-write
+            const int e = ((int)(pane - pbase) * C + (int)key) * 32 + lane;
+            tcnt[e] += 1u;
 #pragma unroll
             for (int f = 0; f < NF; ++f)
-              if (FAST) tf[f * TE + e] = fadd64(tf[f * TE + e], fv[f]);
-              else if (f < p.nf) tf[f * TE + e] = field_combine(p.field[f].kind, tf[f * TE + e], fv[f]);
+              if (FAST) tf[f * TE * 32 + e] = fadd64(tf[f * TE * 32 + e], fv[f]);
+              else if (f < p.nf)
+                tf[f * TE * 32 + e] = field_combine(p.field[f].kind, tf[f * TE * 32 + e], fv[f]);
+          }
+        } else if (MODE == TM_DIRECT) {
+          if (valid) {
+            const int e = (int)(pane - pbase) * C + (int)key;
+            atomicAdd(&tcnt[e], 1u);
+#pragma unroll
+            for (int f = 0; f < NF; ++f)
+              if (FAST) atomicAdd((double *)&tf[f * TE + e], __longlong_as_double((long long)fv[f]));
+              else if (f < p.nf) atom_field(p.field[f].kind, &tf[f * TE + e], fv[f]);
           }
         } else {
-          if (occ + 32 > TE / 2) flush_hashed();
-          const unsigned m = __match_any_sync(kFull, (unsigned long long)key) & actm;
-          warp_combine<NF, FAST>(p, valid, m, fv);
+          if (occ + 32 > TE / 2) flush_hashed();     // keep the load factor <= 1/2
           bool ins = false;
-          if (valid && (__ffs(m) - 1) == lane) {
+          if (valid) {
             uint32_t h = (uint32_t)fmix64(key) & (uint32_t)(TE - 1);
             volatile uint64_t *vk = tkeys;
             for (;;) {
@@ -429,15 +404,14 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
               }
               h = (h + 1) & (uint32_t)(TE - 1);
             }
-            tcnt[h] += (uint32_t)__popc(m);
+            atomicAdd(&tcnt[h], 1u);
 #pragma unroll
             for (int f = 0; f < NF; ++f)
-              if (FAST) tf[f * TE + h] = fadd64(tf[f * TE + h], fv[f]);
-              else if (f < p.nf) tf[f * TE + h] = field_combine(p.field[f].kind, tf[f * TE + h], fv[f]);
+              if (FAST) atomicAdd((double *)&tf[f * TE + h], __longlong_as_double((long long)fv[f]));
+              else if (f < p.nf) atom_field(p.field[f].kind, &tf[f * TE + h], fv[f]);
           }
           occ += __popc(__ballot_sync(kFull, ins));
         }
-        __syncwarp();
       }
       first_round = false;
       if (pl < wend) break;
@@ -467,7 +441,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     }
   }
   if (pbase >= 0) {
-    if (HASHED) flush_hashed(); else flush_direct();
+    if (MODE == TM_HASHED) flush_hashed(); else flush_shared();
   }
   if (err) atomicOr(&st->error, err);
 }
@@ -477,21 +451,27 @@ int p1_nf_template(int nf) { return nf <= 1 ? 1 : nf <= 2 ? 2 : nf <= 4 ? 4 : 8;
 
 int p1_smem_bytes(const Plan &p) { return kStages * kStageBytes + 2 * kStages * 8 + kP1Warps * p.local_bytes; }
 
-template <bool H, int WK>
+template <int M, int WK>
 static void *p1_nf(int nf, bool fast) {
-  if (fast) return nf <= 1 ? (void *)k_pane_agg<H, WK, 1, true> : (void *)k_pane_agg<H, WK, 2, true>;
+  if (fast) return nf <= 1 ? (void *)k_pane_agg<M, WK, 1, true> : (void *)k_pane_agg<M, WK, 2, true>;
   switch (p1_nf_template(nf)) {
-    case 1: return (void *)k_pane_agg<H, WK, 1, false>;
-    case 2: return (void *)k_pane_agg<H, WK, 2, false>;
-    case 4: return (void *)k_pane_agg<H, WK, 4, false>;
-    default: return (void *)k_pane_agg<H, WK, 8, false>;
+    case 1: return (void *)k_pane_agg<M, WK, 1, false>;
+    case 2: return (void *)k_pane_agg<M, WK, 2, false>;
+    case 4: return (void *)k_pane_agg<M, WK, 4, false>;
+    default: return (void *)k_pane_agg<M, WK, 8, false>;
+  }
+}
+template <int WK>
+static void *p1_mode(const Plan &p) {
+  const bool f = p.fast_path;
+  switch (p.local_mode) {
+    case TM_LANE: return p1_nf<TM_LANE, WK>(p.nf, f);
+    case TM_DIRECT: return p1_nf<TM_DIRECT, WK>(p.nf, f);
+    default: return p1_nf<TM_HASHED, WK>(p.nf, f);
   }
 }
 void *p1_kernel(const Plan &p) {
-  const bool h = !p.local_direct;
-  const bool f = p.fast_path;
-  if (p.win_kind == WK_COUNT) return h ? p1_nf<true, WK_COUNT>(p.nf, f) : p1_nf<false, WK_COUNT>(p.nf, f);
-  return h ? p1_nf<true, WK_TIME>(p.nf, f) : p1_nf<false, WK_TIME>(p.nf, f);
+  return p.win_kind == WK_COUNT ? p1_mode<WK_COUNT>(p) : p1_mode<WK_TIME>(p);
 }
 
 int p1_blocks_per_sm(const Plan &p) {

@@ -70,7 +70,7 @@ struct Plan {
   int64_t slot_words;             // 8-byte words per slot
   int32_t hash_bits, pad4;        // log2(C) in HASH mode
   // phase-1 warp-private table
-  int32_t local_direct;           // 1: direct index (pl*C + key); 0: one-pane hash
+  int32_t local_mode;             // 0 LANE (lane-private), 1 DIRECT (warp, atomics), 2 HASHED (one-pane hash)
   int32_t local_entries;          // entries per warp
   int32_t local_pl;               // panes per direct table
   int32_t local_bytes;            // bytes per warp

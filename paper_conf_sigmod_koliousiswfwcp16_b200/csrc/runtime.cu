@@ -297,20 +297,26 @@ static saber_status size_plan(saber_query *q) {
     else R = std::min(next_pow2(need + (1 << 20)), floor_pow2(std::max<int64_t>(budget / slot_bytes, 1)));
     if (R < need + 16) R = next_pow2(need + 16);
     p.R = R;
-    // phase-1 warp-private tables, fields padded to the NF template: 2.5 KiB per
-    // warp for direct-indexed tables (3 CTAs/SM), 5 KiB for hashed ones (2 CTAs/SM)
+    // phase-1 shared-memory tables, fields padded to the NF template:
+    //   LANE   (C <= 8 keys): 8 KiB per warp, one column per lane, no atomics (2 CTAs/SM)
+    //   DIRECT (small dense C): 2.5 KiB per warp, shared atomics (3 CTAs/SM)
+    //   HASHED (large/unbounded C): 5 KiB per warp, one pane at a time (2 CTAs/SM)
     const int nft = p.nf <= 1 ? 1 : p.nf <= 2 ? 2 : p.nf <= 4 ? 4 : 8;
     const int ed = 4 + 8 * nft, eh = 12 + 8 * nft;
-    int budget_w = 2560;
-    if (p.key_mode == KM_HASH || p.C * 2 * ed > budget_w) budget_w = 5 * 1024;
-    if (p.key_mode != KM_HASH && p.C * 2 * ed <= budget_w) {
-      p.local_direct = 1;
-      p.local_pl = (int)std::min<int64_t>(1024, budget_w / (ed * p.C));
+    const int lane_budget = 8 * 1024, direct_budget = 2560, hash_budget = 5 * 1024;
+    if (p.key_mode != KM_HASH && p.C * 2 * 32 * ed <= lane_budget) {
+      p.local_mode = 0;
+      p.local_pl = (int)std::min<int64_t>(1024, lane_budget / (32 * ed * p.C));
+      p.local_entries = p.local_pl * (int)p.C;
+      p.local_bytes = ((p.local_entries * 32 * ed) + 15) & ~15;
+    } else if (p.key_mode != KM_HASH && p.C * 2 * ed <= direct_budget) {
+      p.local_mode = 1;
+      p.local_pl = (int)std::min<int64_t>(1024, direct_budget / (ed * p.C));
       p.local_entries = p.local_pl * (int)p.C;
       p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
     } else {
-      p.local_direct = 0;
-      p.local_entries = (int)floor_pow2(budget_w / eh);
+      p.local_mode = 2;
+      p.local_entries = (int)floor_pow2(hash_budget / eh);
       p.local_pl = 1;
       p.local_bytes = ((p.local_entries * eh) + 15) & ~15;
     }
