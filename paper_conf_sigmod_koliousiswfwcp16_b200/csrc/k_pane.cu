@@ -30,7 +30,7 @@
 namespace sb {
 
 constexpr int kP1Threads = 256, kP1Warps = kP1Threads / 32;
-constexpr int kStageBytes = 16384;
+constexpr int kStageBytes = 16384;   // 512 32-B tuples: 2 iterations per warp per stage
 constexpr int kStages = 3;
 enum { TM_LANE = 0, TM_DIRECT = 1, TM_HASHED = 2 };
 
@@ -310,14 +310,23 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
       const int64_t wend = pbase + PL;
       const int64_t wlo = pbase > min_pane ? pbase : min_pane;
       const bool all_in = (pf >= wlo) & (pl < wend);    // CTA-uniform: no per-tuple window test
-      int64_t cp = 0;                                    // count windows: pane of this lane's tuple
-      int cr = 0;                                        //                and its offset in the pane
+      const int lo_ofs = (int)(wlo - pbase);             // first live offset in the window
+      // count windows: this lane's tuple as (pane offset from pbase, position in the pane),
+      // 32-bit when the pane window spans < 2^30 positions (g32 > 0)
+      const int g32 = (p.g * (int64_t)(PL + 2) < (1ll << 30)) ? (int)p.g : 0;
+      int po = 0, cr = 0;
+      int64_t cp = 0;
       if (WK == WK_COUNT) {
         const int64_t pos = spos + ib + lane;
-        cp = pdiv(p, pos);
-        cr = (int)(pos - cp * p.g);
+        if (g32) {
+          const int r = (int)(pos - pbase * p.g);       // < 0 for tuples before the window (later rounds)
+          po = p.g_shift >= 0 ? (r >> p.g_shift) : (r >= 0 ? r / g32 : -((g32 - 1 - r) / g32));
+          cr = r - po * g32;                            // in [0, g): floor division
+        } else {
+          cp = pdiv(p, pos);
+          cr = (int)(pos - cp * p.g);
+        }
       }
-      const int g32 = (int)p.g;
       for (int i0 = ib; i0 < ie; i0 += 32) {
         const int i = i0 + lane;
         bool valid = i < ie;
@@ -333,16 +342,27 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
           carry_tau = (int64_t)shfl64((uint64_t)tau, 31);
         }
         int64_t pane;
-        if (WK == WK_COUNT) {
-          pane = cp;
-          if (first_round && valid && cr == 0 && pane >= min_pane) pane_ts[pane & (p.R - 1)] = tau;
+        int pw;                                          // this tuple's pane offset from pbase
+        if (WK == WK_COUNT && g32) {
+          pw = po;
+          pane = pbase + po;
+          if (first_round && valid && cr == 0 && po >= lo_ofs) pane_ts[pane & (p.R - 1)] = tau;
+          if (!all_in) valid &= (po >= lo_ofs) & (po < PL);
           cr += 32;
-          while (cr >= g32) { cr -= g32; ++cp; }
+          while (cr >= g32) { cr -= g32; ++po; }
         } else {
-          valid &= tau >= p.T0;
-          pane = tau >= p.T0 ? pdiv(p, tau - p.T0) : -1;
+          if (WK == WK_COUNT) {
+            pane = cp;
+            if (first_round && valid && cr == 0 && pane >= min_pane) pane_ts[pane & (p.R - 1)] = tau;
+            cr += 32;
+            while (cr >= (int)p.g) { cr -= (int)p.g; ++cp; }
+          } else {
+            valid &= tau >= p.T0;
+            pane = tau >= p.T0 ? pdiv(p, tau - p.T0) : -1;
+          }
+          if (!all_in) valid &= (pane >= pbase) & (pane < wend) & (pane >= min_pane);
+          pw = (int)(pane - pbase);
         }
-        if (!all_in) valid &= (pane >= pbase) & (pane < wend) & (pane >= min_pane);
         if (p.npred && valid) valid &= s_preds(p, t);
         uint64_t key;
         uint64_t fv[NF];
@@ -371,7 +391,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         }
         if (MODE == TM_LANE) {
           if (valid) {       // this lane's own column: plain read-modify-write
-            const int e = ((int)(pane - pbase) * C + (int)key) * 32 + lane;
+            const int e = (pw * C + (int)key) * 32 + lane;
             tcnt[e] += 1u;
 #pragma unroll
             for (int f = 0; f < NF; ++f)
@@ -381,7 +401,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
           }
         } else if (MODE == TM_DIRECT) {
           if (valid) {
-            const int e = (int)(pane - pbase) * C + (int)key;
+            const int e = pw * C + (int)key;
             atomicAdd(&tcnt[e], 1u);
 #pragma unroll
             for (int f = 0; f < NF; ++f)
