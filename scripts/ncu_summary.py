@@ -56,10 +56,21 @@ def report(path):
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units = rows[0], rows[1]
     res = []
+    unit_of = dict(zip(hdr, units))
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
+             "nsecond": 1e-3, "usecond": 1, "msecond": 1e3, "second": 1e6}
     for v in rows[2:]:
         d = dict(zip(hdr, v))
         name = d.get("Kernel Name", "?").split("(")[0]
-        m = {k: _f(d.get(k)) for k in KEYS if k in d}
+        m = {}
+        for k in KEYS:
+            if k not in d:
+                continue
+            val, u = _f(d.get(k)), unit_of.get(k, "")
+            if val is not None and u in scale:      # bytes in bytes, durations in microseconds
+                val = val * scale[u]
+                k = k + (".bytes" if "byte" in u else ".us")
+            m[k] = val
         stalls = {h.replace("smsp__pcsamp_warps_issue_stalled_", ""): _f(d[h]) for h in hdr
                   if h.startswith("smsp__pcsamp_warps_issue_stalled_") and not h.endswith("_not_issued")}
         stalls = dict(sorted(((k, v) for k, v in stalls.items() if v), key=lambda x: -x[1])[:8])

@@ -268,3 +268,46 @@ def test_device_generator_matches_numpy(saber):
                     C.c_void_p(buf.data_ptr()), None)
         torch.cuda.synchronize()
         assert buf.cpu().numpy().tobytes() == gen.generate(kind, n, 7, i0=i0, rate=3, groups=64), kind
+
+
+# ------------------------------------------------------- task partitioning ---
+@pytest.mark.parametrize("cfg", ["count", "time", "istream_time"])
+@pytest.mark.parametrize("parts", [2, 3])
+def test_partitioned_queries_match_single_gpu(saber, oracle_lib, cfg, parts):
+    """The multi-GPU plan, run as sequential partitions on one GPU: each partition
+    gets its predecessor's halo (saber_partition_plan on the device), base_index
+    and first_window, and only the last emits on finish."""
+    import torch
+    if cfg == "count":
+        spec, g = workloads.c3(groups=64)
+        spec["window"] = workloads.count_window(4096, 512)
+        n = 1 << 17
+    elif cfg == "time":
+        spec, g = workloads.c4(rate=97)
+        n = 1 << 17
+    else:
+        spec, g = workloads.c2(sel=0.3)
+        spec["window"] = workloads.time_window(50, 7)
+        g = dict(g, rate=13)
+        n = 1 << 16
+    data = gen.generate(g["kind"], n, g["seed"], rate=g["rate"], groups=g.get("groups", 64))
+    tb = spec["schema"]["tuple_bytes"]
+    dev = torch.from_numpy(np.frombuffer(data, np.uint8).copy()).cuda()
+    exp = oracle_lib.run(spec, data, nthreads=8)
+    bounds = [(r * n // parts, (r + 1) * n // parts) for r in range(parts)]
+    slices, first_window, base_index = [], 0, 0
+    for r, (b, e) in enumerate(bounds):
+        q = saber.Query(spec, task_bytes=(1 << 20) + tb * 11, base_index=base_index, first_window=first_window,
+                        emit_on_finish=(r == parts - 1))
+        got = q.run(np.frombuffer(data, np.uint8)[base_index * tb:e * tb])
+        q.close()
+        slices.append(got)
+        if r < parts - 1:
+            first_window, base_index = saber.partition_plan(spec, dev.data_ptr() + b * tb, b, e - b)
+    merged = {"win_id": np.concatenate([s["win_id"] for s in slices]),
+              "win_ts": np.concatenate([s["win_ts"] for s in slices]),
+              "win_nrows": np.concatenate([s["win_nrows"] for s in slices]),
+              "keys": [np.concatenate([s["keys"][i] for s in slices]) for i in range(len(slices[0]["keys"]))],
+              "vals": [np.concatenate([s["vals"][i] for s in slices]) for i in range(len(slices[0]["vals"]))],
+              "tuples": b"".join(s["tuples"] for s in slices)}
+    compare(spec, merged, exp)
