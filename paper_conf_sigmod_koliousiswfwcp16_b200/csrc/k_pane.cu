@@ -32,7 +32,7 @@ namespace sb {
 constexpr int kP1Threads = 256, kP1Warps = kP1Threads / 32;
 constexpr int kStageBytes = 16384;   // 512 32-B tuples: 2 iterations per warp per stage
 constexpr int kStages = 3;
-enum { TM_LANE = 0, TM_DIRECT = 1, TM_HASHED = 2 };
+enum { TM_LANE = 0, TM_DIRECT = 1, TM_HASHED = 2, TM_SHARED = 3 };
 
 // ---------------------------------------------------------------- PTX helpers
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -187,11 +187,12 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   // table geometry: TE entries per warp; LANE mode stores every entry once per lane
   const int TE = p.local_entries;
   const int CW = MODE == TM_LANE ? 32 : 1;               // copies of an entry (lanes)
-  unsigned char *wt = tabs + (size_t)wid * p.local_bytes;
+  constexpr int NCOPY = MODE == TM_SHARED ? 1 : kP1Warps;  // one table per warp, or one per CTA
+  unsigned char *wt = tabs + (MODE == TM_SHARED ? 0 : (size_t)wid * p.local_bytes);
   uint64_t *tkeys = (uint64_t *)wt;                      // HASHED only
   uint64_t *tf = (uint64_t *)(wt + (MODE == TM_HASHED ? 8 * TE : 0));   // [NF][TE*CW]
   uint32_t *tcnt = (uint32_t *)((unsigned char *)tf + (size_t)8 * TE * CW * NF);   // [TE*CW]
-  for (int e = lane; e < TE * CW; e += 32) {
+  for (int e = (MODE == TM_SHARED ? tid : lane); e < TE * CW; e += (MODE == TM_SHARED ? kP1Threads : 32)) {
     if (MODE == TM_HASHED) tkeys[e] = kEmpty;
     tcnt[e] = 0;
 #pragma unroll
@@ -237,7 +238,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
       uint64_t fv[NF];
 #pragma unroll
       for (int f = 0; f < NF; ++f) fv[f] = f < p.nf ? field_identity(p.field[f].kind) : 0;
-      for (int w = 0; w < kP1Warps; ++w) {
+      for (int w = 0; w < NCOPY; ++w) {
         uint64_t *of = (uint64_t *)(tabs + (size_t)w * p.local_bytes);
         uint32_t *oc = (uint32_t *)((unsigned char *)of + (size_t)8 * TE * CW * NF);
         for (int l = 0; l < CW; ++l) {
@@ -399,7 +400,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
               else if (f < p.nf)
                 tf[f * TE * 32 + e] = field_combine(p.field[f].kind, tf[f * TE * 32 + e], fv[f]);
           }
-        } else if (MODE == TM_DIRECT) {
+        } else if (MODE == TM_DIRECT || MODE == TM_SHARED) {
           if (valid) {
             const int e = pw * C + (int)key;
             atomicAdd(&tcnt[e], 1u);
@@ -469,7 +470,9 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
 // ---------------------------------------------------------------- host side
 int p1_nf_template(int nf) { return nf <= 1 ? 1 : nf <= 2 ? 2 : nf <= 4 ? 4 : 8; }
 
-int p1_smem_bytes(const Plan &p) { return kStages * kStageBytes + 2 * kStages * 8 + kP1Warps * p.local_bytes; }
+int p1_smem_bytes(const Plan &p) {
+  return kStages * kStageBytes + 2 * kStages * 8 + (p.local_mode == TM_SHARED ? 1 : kP1Warps) * p.local_bytes;
+}
 
 template <int M, int WK>
 static void *p1_nf(int nf, bool fast) {
@@ -487,6 +490,7 @@ static void *p1_mode(const Plan &p) {
   switch (p.local_mode) {
     case TM_LANE: return p1_nf<TM_LANE, WK>(p.nf, f);
     case TM_DIRECT: return p1_nf<TM_DIRECT, WK>(p.nf, f);
+    case TM_SHARED: return p1_nf<TM_SHARED, WK>(p.nf, f);
     default: return p1_nf<TM_HASHED, WK>(p.nf, f);
   }
 }

@@ -211,6 +211,10 @@ __global__ void k_task_end(const Plan p, State *st, SlotMeta *meta) {
     meta->nrows = st->sel_rows;     // written by the window pass (fused) or k_win_scan
     meta->ntuples = 0;
   }
+  if (p.slab_mode && st->J1 > st->J0) {
+    const int64_t c = (st->J1 - 1) * p.L + p.K;
+    if (c > st->compacted_hi) st->compacted_hi = c;
+  }
   st->J0 = st->J1;
 }
 
@@ -239,6 +243,7 @@ __global__ void k_init_state(State *st, int64_t base_index, int64_t first_window
   s.pane_hi = -1;
   s.first_task = 1;
   s.carry_pos = base_index;
+  s.compacted_hi = first_window * L;
   *st = s;
 }
 

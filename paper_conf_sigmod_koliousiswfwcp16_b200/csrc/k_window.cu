@@ -506,3 +506,180 @@ void *p2_kernel_count(const Plan &p) {
   return p.key_mode == KM_HASH ? (void *)k_win_hash<false> : (void *)k_win_vh<false>;
 }
 }  // namespace sb
+
+// ===========================================================================
+// HASH keys with a declared (radix-packed) domain larger than the dense table:
+// "slab mode".  After a task's scan, every pane that a closed window needs is
+// compacted once from its hash table into key-range buckets (slab = key / SB,
+// a counting sort by slab; PAPER.md L1350-1353 also compacts sparse GPU hash
+// tables).  Window assembly then slides a *dense* per-slab state over the
+// buckets: each pane entry is read twice (enter, leave) and each window-slab
+// costs SB/256 shared-memory slot checks per thread plus its output rows.
+namespace sb {
+
+__device__ __forceinline__ uint32_t *ck_key(const Plan &p, uint64_t *base) { return (uint32_t *)base; }
+__device__ __forceinline__ uint32_t *ck_cnt(const Plan &p, uint64_t *base) { return (uint32_t *)base + p.C; }
+__device__ __forceinline__ uint64_t *ck_fld(const Plan &p, uint64_t *base, int f) { return base + p.C + (int64_t)f * p.C; }
+
+__global__ void __launch_bounds__(256)
+k_pane_compact(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
+               uint64_t *__restrict__ clist, int32_t *__restrict__ coff) {
+  extern __shared__ __align__(16) int s_hist[];          // [S + 1] counts, then [S] cursors
+  const int S = p.S, SB = p.SB;
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  int64_t lo = st->compacted_hi;                         // panes below were compacted by earlier tasks
+  if (lo < J0 * p.L) lo = J0 * p.L;
+  const int64_t hi = (J1 - 1) * p.L + p.K;
+  const int64_t cw = p.C * (1 + p.nf);                     // clist words per pane slot
+  int *cur = s_hist + S + 1;
+  for (int64_t q = lo + blockIdx.x; q < hi; q += gridDim.x) {
+    const int64_t slot = q & (p.R - 1);
+    const uint64_t *tab = table + slot * p.slot_words;
+    uint64_t *cl = clist + slot * cw;
+    for (int i = threadIdx.x; i <= S; i += blockDim.x) s_hist[i] = 0;
+    __syncthreads();
+    for (int64_t h = threadIdx.x; h < p.C; h += blockDim.x) {
+      const uint64_t k = tab[h];
+      if (k != kEmpty) atomicAdd(&s_hist[(int)(k / (uint64_t)SB)], 1);
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {                                // exclusive scan of S bucket sizes
+      const int lane = threadIdx.x;
+      int run = 0;
+      for (int b = 0; b < S; b += 32) {
+        const int v = b + lane < S ? s_hist[b + lane] : 0;
+        int x = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(kFull, x, o);
+          if (lane >= o) x += y;
+        }
+        if (b + lane < S) cur[b + lane] = run + x - v;
+        run += __shfl_sync(kFull, x, 31);
+      }
+      if (lane == 0) cur[S] = run;
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i <= S; i += blockDim.x) coff[slot * (S + 1) + i] = cur[i];
+    __syncthreads();
+    for (int64_t h = threadIdx.x; h < p.C; h += blockDim.x) {
+      const uint64_t k = tab[h];
+      if (k == kEmpty) continue;
+      const int pos = atomicAdd(&cur[(int)(k / (uint64_t)SB)], 1);
+      ck_key(p, cl)[pos] = (uint32_t)k;
+      ck_cnt(p, cl)[pos] = (uint32_t)tab[p.C + h];
+      for (int f = 0; f < p.nf; ++f) ck_fld(p, cl, f)[pos] = tab[fld_off(p, f) + h];
+    }
+    __syncthreads();
+  }
+}
+
+template <bool EMIT>
+__global__ void __launch_bounds__(256)
+k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, const int32_t *__restrict__ coff,
+           int64_t *__restrict__ counts, unsigned char *__restrict__ rows, int W) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ int scan_sm[40];
+  const int S = p.S, SB = p.SB;
+  int64_t *scnt = (int64_t *)smem;
+  uint64_t *sf = (uint64_t *)(scnt + SB);
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  if (nw <= 0) return;
+  const int64_t cw = p.C * (1 + p.nf);
+  const int64_t nchunks = (nw + W - 1) / W;
+  const int64_t nitems = nchunks * S;
+  for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
+    const int64_t chunk = item / S;
+    const int slab = (int)(item % S);
+    const uint32_t kbase = (uint32_t)slab * (uint32_t)SB;
+    const int64_t ja = J0 + chunk * W;
+    const int64_t jb = ja + W < J1 ? ja + W : J1;
+    __syncthreads();
+    for (int s = threadIdx.x; s < SB; s += blockDim.x) {
+      scnt[s] = 0;
+      for (int f = 0; f < p.nf; ++f) sf[f * SB + s] = field_identity(p.field[f].kind);
+    }
+    __syncthreads();
+    // entries of one pane have distinct keys: plain read-modify-write, barrier per pane
+    auto visit = [&](int64_t q, int sign, bool minmax) {
+      const int64_t slot = q & (p.R - 1);
+      uint64_t *cl = clist + slot * cw;
+      const int a = coff[slot * (S + 1) + slab], b = coff[slot * (S + 1) + slab + 1];
+      for (int e = a + threadIdx.x; e < b; e += blockDim.x) {
+        const int s = (int)(ck_key(p, cl)[e] - kbase);
+        if (!minmax) scnt[s] += sign * (int64_t)ck_cnt(p, cl)[e];
+        for (int f = 0; f < p.nf; ++f) {
+          const int kind = p.field[f].kind;
+          const uint64_t v = ck_fld(p, cl, f)[e];
+          if (!minmax && kind == FK_SUM_F)
+            sf[f * SB + s] = (uint64_t)__double_as_longlong(__longlong_as_double((long long)sf[f * SB + s]) +
+                                                           sign * __longlong_as_double((long long)v));
+          else if (!minmax && kind == FK_SUM_I) sf[f * SB + s] = (uint64_t)((int64_t)sf[f * SB + s] + sign * (int64_t)v);
+          else if (minmax && (kind == FK_MIN || kind == FK_MAX)) sf[f * SB + s] = field_combine(kind, sf[f * SB + s], v);
+        }
+      }
+      __syncthreads();
+    };
+    for (int64_t q = ja * p.L; q < ja * p.L + p.K; ++q) visit(q, +1, false);
+    for (int64_t j = ja; j < jb; ++j) {
+      if (j > ja) {
+        for (int64_t q = (j - 1) * p.L + p.K; q < j * p.L + p.K; ++q) visit(q, +1, false);
+        for (int64_t q = (j - 1) * p.L; q < j * p.L; ++q) visit(q, -1, false);
+      }
+      for (int s = threadIdx.x; s < SB; s += blockDim.x)
+        if (scnt[s] == 0)
+          for (int f = 0; f < p.nf; ++f)
+            if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) sf[f * SB + s] = 0;
+      if (p.has_minmax) {
+        for (int s = threadIdx.x; s < SB; s += blockDim.x)
+          for (int f = 0; f < p.nf; ++f)
+            if (p.field[f].kind == FK_MIN || p.field[f].kind == FK_MAX) sf[f * SB + s] = field_identity(p.field[f].kind);
+        __syncthreads();
+        for (int64_t q = j * p.L; q < j * p.L + p.K; ++q) visit(q, 0, true);
+      }
+      __syncthreads();
+      int my = 0;
+      uint64_t fv[kMaxField];
+      for (int s = threadIdx.x; s < SB; s += blockDim.x) {
+        if (scnt[s] <= 0) continue;
+        if (p.nhave) {
+          for (int f = 0; f < p.nf; ++f) fv[f] = sf[f * SB + s];
+          if (!having_ok(p, scnt[s], fv)) continue;
+        }
+        ++my;
+      }
+      int total;
+      const int excl = group_excl_scan(my, 256, scan_sm, total);
+      const int64_t ci = (j - J0) * S + slab;
+      if (!EMIT) {
+        if (threadIdx.x == 0) counts[ci] = total;
+      } else {
+        int64_t r = counts[ci] + excl;
+        for (int s = threadIdx.x; s < SB; s += blockDim.x) {
+          if (scnt[s] <= 0) continue;
+          for (int f = 0; f < p.nf; ++f) fv[f] = sf[f * SB + s];
+          if (p.nhave && !having_ok(p, scnt[s], fv)) continue;
+          int64_t kv[kMaxKey];
+          decode_key(p, (uint64_t)(kbase + (uint32_t)s), kv);
+          write_row(p, rows, r++, kv, scnt[s], fv);
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
+cudaError_t launch_windows_slab(const Plan &p, const QueryDev &q, const SlotDev &s, bool emit, int grid, int W,
+                                cudaStream_t st) {
+  if (!emit) {
+    k_pane_compact<<<148 * 4, 256, (2 * p.S + 2) * sizeof(int), st>>>(p, q.st, q.table, q.clist, q.coff);
+    k_win_slab<false><<<grid, 256, p.p2_smem, st>>>(p, q.st, q.clist, q.coff, s.counts, s.rows, W);
+  } else {
+    k_win_slab<true><<<grid, 256, p.p2_smem, st>>>(p, q.st, q.clist, q.coff, s.counts, s.rows, W);
+  }
+  return cudaGetLastError();
+}
+void *slab_kernel(bool emit) { return emit ? (void *)k_win_slab<true> : (void *)k_win_slab<false>; }
+
+}  // namespace sb

@@ -19,6 +19,8 @@ struct QueryDev {
   uint64_t *table;          // pane ring: R slots × slot_words
   uint64_t *vh_pre;         // van Herk block-prefix arrays (DENSE/GLOBAL), same geometry
   uint64_t *vh_suf;         // van Herk block-suffix arrays
+  uint64_t *clist;          // slab mode: per pane slot, entries bucketed by key range
+  int32_t *coff;            // slab mode: per pane slot, S+1 bucket offsets
   int64_t *pane_ts;         // R
   uint64_t *tile_status;    // IStream look-back
   int64_t tile_status_cap;

@@ -15,6 +15,12 @@ cudaError_t set_kernel_attributes(const Plan &p) {
     if (e) return e;
     if (p.key_mode == KM_HASH) {
       e = cudaFuncSetAttribute(p2_kernel_count(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
+      if (e) return e;
+    }
+    if (p.slab_mode) {
+      e = cudaFuncSetAttribute(slab_kernel(false), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
+      if (e) return e;
+      e = cudaFuncSetAttribute(slab_kernel(true), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
     }
   }
   return e;
@@ -22,7 +28,7 @@ cudaError_t set_kernel_attributes(const Plan &p) {
 
 int p2_blocks_per_sm(const Plan &p) {
   int b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, p2_kernel(p), 256, p.p2_smem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, p.slab_mode ? slab_kernel(true) : p2_kernel(p), 256, p.p2_smem);
   return b > 0 ? b : 1;
 }
 int sel_blocks_per_sm(const Plan &p) {
@@ -44,7 +50,12 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
     *launches += 1;
   }
   if (evs) cudaEventRecord(evs[1], st);
-  if (p.key_mode == KM_HASH) {
+  if (p.slab_mode) {
+    if ((e = launch_windows_slab(p, q, s, false, p2_grid, win_chunk, st))) return e;
+    if ((e = launch_win_scan(p, q, s, st))) return e;
+    if ((e = launch_windows_slab(p, q, s, true, p2_grid, win_chunk, st))) return e;
+    *launches += 1;
+  } else if (p.key_mode == KM_HASH) {
     if ((e = launch_windows(p, q, s, false, p2_grid, win_chunk, st))) return e;
     if ((e = launch_win_scan(p, q, s, st))) return e;
     if ((e = launch_windows(p, q, s, true, p2_grid, win_chunk, st))) return e;

@@ -24,6 +24,9 @@ void *p2_kernel_count(const Plan &p);
 cudaError_t launch_windows(const Plan &p, const QueryDev &q, const SlotDev &s, bool emit, int grid, int win_chunk,
                            cudaStream_t st);
 cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st);
+cudaError_t launch_windows_slab(const Plan &p, const QueryDev &q, const SlotDev &s, bool emit, int grid, int W,
+                                cudaStream_t st);
+void *slab_kernel(bool emit);
 // k_select.cu
 void *sel_kernel(const Plan &p);
 cudaError_t launch_select(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int grid,

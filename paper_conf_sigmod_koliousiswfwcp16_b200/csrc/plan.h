@@ -79,6 +79,7 @@ struct Plan {
   int32_t S, SB, GS, pad5;        // key slabs, slots per slab, threads per slab group
   int32_t state_cap, p2_smem;     // hash state entries per CTA, dynamic smem bytes
   int32_t has_minmax, has_inv;    // min/max fields present; invertible (count/sum) fields
+  int32_t slab_mode, pad8;        // HASH + radix keys: compacted key-range buckets, dense slab state
   // output
   int32_t ncols, row_bytes;       // aggregation output columns, bytes per row
   int32_t col_bytes[kMaxCols];
@@ -109,6 +110,7 @@ struct State {
   int32_t carry_sel, first_task;  // which carry buffer is current; first task flag
   int64_t sel_rows;               // rows written by the compaction kernel
   int64_t tile_epoch;             // look-back epoch
+  int64_t compacted_hi;           // slab mode: panes < compacted_hi have bucketed lists
 };
 
 // Per result slot metadata, copied to the host after a task.

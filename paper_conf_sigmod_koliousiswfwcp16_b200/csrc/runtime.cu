@@ -314,6 +314,12 @@ static saber_status size_plan(saber_query *q) {
       p.local_pl = (int)std::min<int64_t>(1024, direct_budget / (ed * p.C));
       p.local_entries = p.local_pl * (int)p.C;
       p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
+    } else if (p.key_mode != KM_HASH && p.C * 2 * ed <= 48 * 1024) {
+      // one dense table per CTA, shared atomics (mid-size declared domains)
+      p.local_mode = 3;
+      p.local_pl = (int)std::min<int64_t>(1024, (48 * 1024) / (ed * p.C));
+      p.local_entries = p.local_pl * (int)p.C;
+      p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
     } else {
       p.local_mode = 2;
       p.local_entries = (int)floor_pow2(hash_budget / eh);
@@ -352,6 +358,19 @@ static saber_status size_plan(saber_query *q) {
       p.SB = (int)sb;
       p.S = (int)(p.C / sb);
       p.p2_smem = p.state_cap * 8 * (2 + p.nf);
+      // radix-packed keys with a declared domain: key-range slabs with a dense
+      // shared-memory state (48 KiB) over compacted pane buckets
+      if (p.key_pack == KP_RADIX && p.G < (1ll << 31)) {
+        const int64_t slab = floor_pow2((48 * 1024) / (8 * (1 + p.nf)));
+        const int64_t S = (p.G + slab - 1) / slab;
+        if (S <= 1024) {
+          p.slab_mode = 1;
+          q->win_chunk = 128;          // K-pane initialisation amortised over 128 windows
+          p.SB = (int)slab;
+          p.S = (int)S;
+          p.p2_smem = (int)(slab * 8 * (1 + p.nf));
+        }
+      }
     }
     // output columns (keys then aggregates)
     p.ncols = p.nkeys + p.nagg;
@@ -364,7 +383,9 @@ static saber_status size_plan(saber_query *q) {
     int64_t rb = c.result_bytes;
     if (rb <= 0) {
       long double bound = (long double)p.win_cap * rows_per_win * p.row_bytes;
-      rb = (int64_t)std::min<long double>(std::max<long double>(bound, 1 << 20), 1ll << 30);
+      // device-resident results may use up to 4 GiB per slot; pinned host mirrors stay <= 1 GiB
+      const int64_t cap = c.result_mode == SABER_RESULTS_DEVICE ? (4ll << 30) : (1ll << 30);
+      rb = (int64_t)std::min<long double>(std::max<long double>(bound, 1 << 20), (long double)cap);
     }
     p.rows_cap = std::max<int64_t>(1, rb / p.row_bytes);
     int64_t off = 0;
@@ -403,6 +424,10 @@ static saber_status alloc_query(saber_query *q) {
       q->qd.tile_status_cap = p.win_cap + 16;
       CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
       CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
+    }
+    if (p.slab_mode) {
+      CK(cudaMalloc(&q->qd.clist, (size_t)p.R * p.C * (1 + p.nf) * 8));
+      CK(cudaMalloc(&q->qd.coff, (size_t)p.R * (p.S + 1) * 4));
     }
   } else {
     q->qd.carry_cap = p.carry_cap;
@@ -559,7 +584,8 @@ void saber_query_destroy(saber_query *q) {
   }
   for (auto &r : q->registered)
     if (std::find(q->prereg.begin(), q->prereg.end(), r.first) == q->prereg.end()) cudaHostUnregister(r.first);
-  cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.vh_pre); cudaFree(q->qd.vh_suf); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
+  cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.vh_pre); cudaFree(q->qd.vh_suf);
+  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
   cudaFree(q->qd.carry[0]); cudaFree(q->qd.carry[1]); cudaFree(q->qd.tile_ctr); cudaFree(q->d_tmp);
   if (q->cs) cudaStreamDestroy(q->cs);
   if (q->h2d) cudaStreamDestroy(q->h2d);
