@@ -6,6 +6,11 @@
 #include "device_util.cuh"
 #include "plan.h"
 
+// loops over the query's fields / key columns with compile-time bounds, so small
+// per-thread arrays indexed by the loop variable stay in registers
+#define FOR_F(f) _Pragma("unroll") for (int f = 0; f < kMaxField; ++f) if (f < p.nf)
+#define FOR_K(i) _Pragma("unroll") for (int i = 0; i < kMaxKey; ++i) if (i < p.nkeys)
+
 namespace sb {
 
 struct WinHdr { int64_t window_id, ts, row_offset; int32_t nrows, flags; };
@@ -134,21 +139,29 @@ __device__ __forceinline__ int64_t global_insert(const Plan &p, State *st, uint6
 // window assembly helpers
 struct AggVal { uint64_t bits; bool isf; };
 
+// fv[i] for a runtime i without dynamic register indexing (no local-memory spill)
+__device__ __forceinline__ uint64_t pick_field(const uint64_t *fv, int i) {
+  uint64_t r = fv[0];
+#pragma unroll
+  for (int k = 1; k < kMaxField; ++k) r = (i == k) ? fv[k] : r;
+  return r;
+}
+
 __device__ __forceinline__ AggVal finalize(const Plan &p, int a, int64_t cnt, const uint64_t *fv) {
   const AggOut &o = p.agg[a];
   AggVal r;
   r.isf = o.out_float;
+  const uint64_t x = o.field >= 0 ? pick_field(fv, o.field) : 0;
   switch (o.fn) {
     case AG_COUNT: r.bits = (uint64_t)cnt; break;
-    case AG_SUM: r.bits = fv[o.field]; break;
+    case AG_SUM: r.bits = x; break;
     case AG_AVG: {
-      double sum = (p.field[o.field].kind == FK_SUM_F) ? __longlong_as_double((long long)fv[o.field])
-                                                      : (double)(int64_t)fv[o.field];
+      double sum = (p.field[o.field].kind == FK_SUM_F) ? __longlong_as_double((long long)x) : (double)(int64_t)x;
       r.bits = (uint64_t)__double_as_longlong(sum / (double)cnt);   // reading A11
       break;
     }
     default: {
-      uint64_t u = fv[o.field];
+      uint64_t u = x;
       r.bits = o.is_float_col ? (uint64_t)__double_as_longlong(dec_dbl(u)) : (uint64_t)dec_int(u);
     }
   }
@@ -169,7 +182,7 @@ __device__ __forceinline__ bool having_ok(const Plan &p, int64_t cnt, const uint
 __device__ __forceinline__ void write_row(const Plan &p, unsigned char *rows, int64_t r, const int64_t *kv,
                                           int64_t cnt, const uint64_t *fv) {
   if (r >= p.rows_cap) return;
-  for (int i = 0; i < p.nkeys; ++i) {
+  FOR_K(i) {
     unsigned char *c = rows + p.col_off[i];
     if (p.col_bytes[i] == 4) ((int32_t *)c)[r] = (int32_t)kv[i];
     else ((int64_t *)c)[r] = kv[i];
@@ -182,7 +195,14 @@ __device__ __forceinline__ void write_row(const Plan &p, unsigned char *rows, in
 
 __device__ __forceinline__ void decode_key(const Plan &p, uint64_t k, int64_t *kv) {
   if (p.key_pack == KP_RADIX) {
-    for (int i = 0; i < p.nkeys; ++i) kv[i] = (int64_t)((k / (uint64_t)p.key[i].stride) % (uint64_t)p.key[i].domain);
+    if (p.nkeys == 1) {
+      kv[0] = (int64_t)k;                                   // single key: the packed key is the value
+    } else if (p.G <= 0xffffffffll) {                         // 32-bit divisions
+      FOR_K(i)
+        kv[i] = (int64_t)(((uint32_t)k / (uint32_t)p.key[i].stride) % (uint32_t)p.key[i].domain);
+    } else {
+      FOR_K(i) kv[i] = (int64_t)((k / (uint64_t)p.key[i].stride) % (uint64_t)p.key[i].domain);
+    }
   } else if (p.key_pack == KP_BIASED64) {
     kv[0] = (int64_t)(k ^ 0x8000000000000000ull);
   } else {

@@ -76,6 +76,138 @@ k_vh_build(const Plan p, const State *__restrict__ st, const uint64_t *__restric
   }
 }
 
+__device__ __forceinline__ uint64_t shfl_up64_n(uint64_t v, int o) {
+  const uint32_t lo = __shfl_up_sync(kFull, (uint32_t)v, o), hi = __shfl_up_sync(kFull, (uint32_t)(v >> 32), o);
+  return ((uint64_t)hi << 32) | lo;
+}
+
+// Long windows (K > 64 panes): one CTA per (block, table word, direction); the
+// block's panes are split into 256 chunks, each thread scans its chunk, the CTA
+// scans the chunk totals, and each thread re-walks its chunk adding its offset.
+__global__ void __launch_bounds__(256)
+k_vh_build_long(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
+                uint64_t *__restrict__ pre, uint64_t *__restrict__ suf) {
+  __shared__ uint64_t s_tot[256];
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  const int64_t lo = J0 * p.L, hi = (J1 - 1) * p.L + p.K - 1;
+  const int64_t b0 = lo / p.K, b1 = hi / p.K;
+  const int64_t words = p.slot_words;
+  const int64_t items = (b1 - b0 + 1) * words * 2;
+  const int64_t Rm = p.R - 1;
+  const int tid = threadIdx.x;
+  for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const int64_t w = it % words;
+    const int64_t rest = it / words;
+    const bool prefix = rest & 1;
+    const int64_t b = b0 + (rest >> 1);
+    const int f = (int)(w / p.C) - 1;
+    const int kind = f < 0 ? -1 : p.field[f].kind;
+    const int64_t bs = b * p.K, be = (bs + p.K - 1 < hi) ? bs + p.K - 1 : hi;
+    const int64_t qa = prefix ? bs : (bs > lo ? bs : lo);      // scanned pane range [qa, be]
+    if (prefix && bs < lo) continue;                             // uniform across the CTA
+    const uint64_t id = kind < 0 ? 0ull : field_identity(kind);
+    const int64_t len = be - qa + 1;
+    const int64_t ch = (len + 255) / 256;
+    // chunk t covers positions [t*ch, (t+1)*ch) of the scan order
+    const int64_t c0 = tid * ch, c1 = (c0 + ch < len) ? c0 + ch : len;
+    auto pane_of = [&](int64_t k) { return prefix ? qa + k : be - k; };
+    uint64_t acc = id;
+    for (int64_t k = c0; k < c1; ++k) {
+      const uint64_t v = table[(pane_of(k) & Rm) * words + w];
+      acc = kind < 0 ? acc + v : field_combine(kind, acc, v);
+    }
+    s_tot[tid] = acc;
+    __syncthreads();
+    if (tid < 32) {                                   // exclusive scan of 256 chunk totals (warp 0)
+      uint64_t v[8];
+      uint64_t lt = id;
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        v[k] = s_tot[tid * 8 + k];
+        lt = kind < 0 ? lt + v[k] : field_combine(kind, lt, v[k]);
+      }
+      uint64_t x = lt;                                // inclusive warp scan of lane totals
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t y = shfl_up64_n(x, o);
+        if (tid >= o) x = kind < 0 ? x + y : field_combine(kind, y, x);
+      }
+      uint64_t run = shfl_up64_n(x, 1);
+      if (tid == 0) run = id;
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        s_tot[tid * 8 + k] = run;
+        run = kind < 0 ? run + v[k] : field_combine(kind, run, v[k]);
+      }
+    }
+    __syncthreads();
+    acc = s_tot[tid];
+    uint64_t *dst = prefix ? pre : suf;
+    for (int64_t k = c0; k < c1; ++k) {
+      const int64_t r = (pane_of(k) & Rm) * words + w;
+      const uint64_t v = table[r];
+      acc = kind < 0 ? acc + v : field_combine(kind, acc, v);
+      dst[r] = acc;
+    }
+    __syncthreads();
+  }
+}
+
+// Long windows, many table words: one warp per (block, word, direction), lane =
+// chunk of the block's panes; no shared memory, no barriers.
+__global__ void __launch_bounds__(256)
+k_vh_build_warp(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
+                uint64_t *__restrict__ pre, uint64_t *__restrict__ suf) {
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  const int lane = threadIdx.x & 31;
+  const int64_t lo = J0 * p.L, hi = (J1 - 1) * p.L + p.K - 1;
+  const int64_t b0 = lo / p.K, b1 = hi / p.K;
+  const int64_t words = p.slot_words;
+  const int64_t items = (b1 - b0 + 1) * words * 2;
+  const int64_t Rm = p.R - 1;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t it = gw; it < items; it += nwarps) {
+    const int64_t w = it % words;                        // consecutive warps: consecutive words
+    const int64_t rest = it / words;
+    const bool prefix = rest & 1;
+    const int64_t b = b0 + (rest >> 1);
+    const int f = (int)(w / p.C) - 1;
+    const int kind = f < 0 ? -1 : p.field[f].kind;
+    const int64_t bs = b * p.K, be = (bs + p.K - 1 < hi) ? bs + p.K - 1 : hi;
+    if (prefix && bs < lo) continue;                     // warp-uniform
+    const int64_t qa = prefix ? bs : (bs > lo ? bs : lo);
+    const uint64_t id = kind < 0 ? 0ull : field_identity(kind);
+    const int64_t len = be - qa + 1;
+    const int64_t ch = (len + 31) / 32;
+    const int64_t c0 = lane * ch, c1 = (c0 + ch < len) ? c0 + ch : len;
+    auto pane_of = [&](int64_t k) { return prefix ? qa + k : be - k; };
+    uint64_t acc = id;
+#pragma unroll 4
+    for (int64_t k = c0; k < c1; ++k) {
+      const uint64_t v = table[(pane_of(k) & Rm) * words + w];
+      acc = kind < 0 ? acc + v : field_combine(kind, acc, v);
+    }
+    uint64_t x = acc;                                    // inclusive scan of chunk totals
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint64_t y = shfl_up64_n(x, o);
+      if (lane >= o) x = kind < 0 ? x + y : field_combine(kind, y, x);
+    }
+    uint64_t run = shfl_up64_n(x, 1);
+    if (lane == 0) run = id;
+    uint64_t *dst = prefix ? pre : suf;
+#pragma unroll 4
+    for (int64_t k = c0; k < c1; ++k) {
+      const int64_t r = (pane_of(k) & Rm) * words + w;
+      run = kind < 0 ? run + table[r] : field_combine(kind, run, table[r]);
+      dst[r] = run;
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------
 // Single pass over the windows closed by a task (DENSE/GLOBAL): CTAs take window
 // chunks in ticket order, count the rows of every (window, slab) item, obtain
@@ -103,6 +235,7 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
   constexpr int gpb = 256 / GS;
   __shared__ int s_cnt[kFusedMaxItems];
   __shared__ int s_off[kFusedMaxItems];
+  __shared__ int s_scan[40];
   __shared__ int s_total;
   __shared__ int64_t s_base;
   __shared__ int s_t;
@@ -138,7 +271,7 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
           if (c <= 0) continue;
           if (p.nhave) {
             uint64_t fv[kMaxField];
-            for (int f = 0; f < p.nf; ++f) {
+            FOR_F(f) {
               const uint64_t x = sa[vh_off(p, f) + s];
               fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
             }
@@ -233,46 +366,48 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
       const uint64_t *sa = suf + (a & (p.R - 1)) * p.slot_words + slot0;
       const uint64_t *pb = pre + ((a + p.K - 1) & (p.R - 1)) * p.slot_words + slot0;
       int64_t r = base + s_off[it];
-      for (int s0 = 0; s0 < nslot; s0 += GS) {
-        const int s = s0 + gt;
-        bool present = false;
-        int64_t c = 0;
-        uint64_t fv[kMaxField];
-        if (s < nslot) {
-          c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
-          if (c > 0) {
-            for (int f = 0; f < p.nf; ++f) {
-              const uint64_t x = sa[vh_off(p, f) + s];
-              fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
-            }
-            present = !p.nhave || having_ok(p, c, fv);
-          }
+      auto value = [&](int s, int64_t &c, uint64_t (&fv)[kMaxField]) -> bool {
+        c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
+        if (c <= 0) return false;
+        FOR_F(f) {
+          const uint64_t x = sa[vh_off(p, f) + s];
+          fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
         }
-        // rank among the group's present slots (GS = 32: one warp; GS = 256: 8 warps)
-        const unsigned bal = __ballot_sync(kFull, present);
-        int rank = __popc(bal & ((1u << lane) - 1u));
-        int tot = __popc(bal);
-        if (GS == 256) {
-          __shared__ int s_w[8];
-          __syncwarp();
-          if (lane == 0) s_w[threadIdx.x >> 5] = tot;
-          __syncthreads();
-          int before = 0, all = 0;
-          for (int w = 0; w < 8; ++w) {
-            const int x = s_w[w];
-            if (w < (threadIdx.x >> 5)) before += x;
-            all += x;
+        return !p.nhave || having_ok(p, c, fv);
+      };
+      if (GS == 32) {
+        // warp: rows in slot (key) order, one ballot per 32 slots
+        for (int s0 = 0; s0 < nslot; s0 += GS) {
+          const int s = s0 + gt;
+          int64_t c = 0;
+          uint64_t fv[kMaxField];
+          const bool present = s < nslot && value(s, c, fv);
+          const unsigned bal = __ballot_sync(kFull, present);
+          if (present) {
+            int64_t kv[kMaxKey];
+            decode_key(p, (uint64_t)(slot0 + s), kv);
+            write_row(p, rows, r + __popc(bal & ((1u << lane) - 1u)), kv, c, fv);
           }
-          rank += before;
-          tot = all;
-          __syncthreads();
+          r += __popc(bal);
         }
-        if (present) {
+      } else {
+        // block: each thread's present slots are contiguous rows (one block scan per item)
+        int my = 0;
+        for (int s = gt; s < nslot; s += GS) {
+          int64_t c;
+          uint64_t fv[kMaxField];
+          my += value(s, c, fv);
+        }
+        int tot;
+        r += group_excl_scan(my, 256, s_scan, tot);
+        for (int s = gt; s < nslot; s += GS) {
+          int64_t c;
+          uint64_t fv[kMaxField];
+          if (!value(s, c, fv)) continue;
           int64_t kv[kMaxKey];
           decode_key(p, (uint64_t)(slot0 + s), kv);
-          write_row(p, rows, r + rank, kv, c, fv);
+          write_row(p, rows, r++, kv, c, fv);
         }
-        r += tot;
       }
     }
     __syncthreads();
@@ -307,7 +442,7 @@ k_win_vh(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre,
       int64_t c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
       if (c <= 0) continue;
       uint64_t fv[kMaxField];
-      for (int f = 0; f < p.nf; ++f) {
+      FOR_F(f) {
         const uint64_t x = sa[vh_off(p, f) + s];
         fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
       }
@@ -326,7 +461,7 @@ k_win_vh(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre,
       int64_t c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
       if (c <= 0) continue;
       uint64_t fv[kMaxField];
-      for (int f = 0; f < p.nf; ++f) {
+      FOR_F(f) {
         const uint64_t x = sa[vh_off(p, f) + s];
         fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
       }
@@ -367,7 +502,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
     for (int h = threadIdx.x; h < ST; h += blockDim.x) {
       skeys[h] = kEmpty;
       scnt[h] = 0;
-      for (int f = 0; f < p.nf; ++f) sf[f * ST + h] = field_identity(p.field[f].kind);
+      FOR_F(f) sf[f * ST + h] = field_identity(p.field[f].kind);
     }
     __syncthreads();
     auto find = [&](uint64_t k) -> int {
@@ -399,7 +534,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
         if (!minmax) {
           atomicAdd((unsigned long long *)&scnt[s], (unsigned long long)(sign * (int64_t)b[p.C + h]));
         }
-        for (int f = 0; f < p.nf; ++f) {
+        FOR_F(f) {
           const int kind = p.field[f].kind;
           const uint64_t v = b[fld_off(p, f) + h];
           if (!minmax && kind == FK_SUM_F) atomicAdd((double *)&sf[f * ST + s], sign * __longlong_as_double((long long)v));
@@ -418,11 +553,11 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
       __syncthreads();
       for (int h = threadIdx.x; h < ST; h += blockDim.x)
         if (scnt[h] == 0)
-          for (int f = 0; f < p.nf; ++f)
+          FOR_F(f)
             if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) sf[f * ST + h] = 0;
       if (p.has_minmax) {
         for (int h = threadIdx.x; h < ST; h += blockDim.x)
-          for (int f = 0; f < p.nf; ++f)
+          FOR_F(f)
             if (p.field[f].kind == FK_MIN || p.field[f].kind == FK_MAX) sf[f * ST + h] = field_identity(p.field[f].kind);
         __syncthreads();
         for (int64_t q = j * p.L; q < j * p.L + p.K; ++q) visit_pane(q, 0, true);
@@ -432,7 +567,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
       uint64_t fv[kMaxField];
       for (int h = threadIdx.x; h < ST; h += blockDim.x) {
         if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
-        for (int f = 0; f < p.nf; ++f) fv[f] = sf[f * ST + h];
+        FOR_F(f) fv[f] = sf[f * ST + h];
         if (having_ok(p, scnt[h], fv)) ++my;
       }
       int total;
@@ -444,7 +579,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
         int64_t r = counts[ci] + excl;
         for (int h = threadIdx.x; h < ST; h += blockDim.x) {
           if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
-          for (int f = 0; f < p.nf; ++f) fv[f] = sf[f * ST + h];
+          FOR_F(f) fv[f] = sf[f * ST + h];
           if (!having_ok(p, scnt[h], fv)) continue;
           int64_t kv[kMaxKey];
           decode_key(p, skeys[h], kv);
@@ -485,7 +620,11 @@ cudaError_t launch_windows(const Plan &p, const QueryDev &q, const SlotDev &s, b
 
 // DENSE/GLOBAL: van Herk arrays, then one fused count + look-back + emit pass
 cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st) {
-  k_vh_build<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  // long windows: a CTA per (block, word) when there are few words (no GROUP BY),
+  // a warp per (block, word) otherwise; short windows: a thread per (block, word)
+  if (p.K > 64 && p.slot_words < 64) k_vh_build_long<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  else if (p.K > 64) k_vh_build_warp<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  else k_vh_build<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   const int gpb = 256 / p.GS;
   int wc = gpb * 8 / p.S;
   if (wc * p.S > kFusedMaxItems) wc = kFusedMaxItems / p.S;
@@ -569,7 +708,7 @@ k_pane_compact(const Plan p, const State *__restrict__ st, const uint64_t *__res
       const int pos = atomicAdd(&cur[(int)(k / (uint64_t)SB)], 1);
       ck_key(p, cl)[pos] = (uint32_t)k;
       ck_cnt(p, cl)[pos] = (uint32_t)tab[p.C + h];
-      for (int f = 0; f < p.nf; ++f) ck_fld(p, cl, f)[pos] = tab[fld_off(p, f) + h];
+      FOR_F(f) ck_fld(p, cl, f)[pos] = tab[fld_off(p, f) + h];
     }
     __syncthreads();
   }
@@ -598,7 +737,7 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
     __syncthreads();
     for (int s = threadIdx.x; s < SB; s += blockDim.x) {
       scnt[s] = 0;
-      for (int f = 0; f < p.nf; ++f) sf[f * SB + s] = field_identity(p.field[f].kind);
+      FOR_F(f) sf[f * SB + s] = field_identity(p.field[f].kind);
     }
     __syncthreads();
     // entries of one pane have distinct keys: plain read-modify-write, barrier per pane
@@ -609,7 +748,7 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
       for (int e = a + threadIdx.x; e < b; e += blockDim.x) {
         const int s = (int)(ck_key(p, cl)[e] - kbase);
         if (!minmax) scnt[s] += sign * (int64_t)ck_cnt(p, cl)[e];
-        for (int f = 0; f < p.nf; ++f) {
+        FOR_F(f) {
           const int kind = p.field[f].kind;
           const uint64_t v = ck_fld(p, cl, f)[e];
           if (!minmax && kind == FK_SUM_F)
@@ -629,11 +768,11 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
       }
       for (int s = threadIdx.x; s < SB; s += blockDim.x)
         if (scnt[s] == 0)
-          for (int f = 0; f < p.nf; ++f)
+          FOR_F(f)
             if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) sf[f * SB + s] = 0;
       if (p.has_minmax) {
         for (int s = threadIdx.x; s < SB; s += blockDim.x)
-          for (int f = 0; f < p.nf; ++f)
+          FOR_F(f)
             if (p.field[f].kind == FK_MIN || p.field[f].kind == FK_MAX) sf[f * SB + s] = field_identity(p.field[f].kind);
         __syncthreads();
         for (int64_t q = j * p.L; q < j * p.L + p.K; ++q) visit(q, 0, true);
@@ -644,7 +783,7 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
       for (int s = threadIdx.x; s < SB; s += blockDim.x) {
         if (scnt[s] <= 0) continue;
         if (p.nhave) {
-          for (int f = 0; f < p.nf; ++f) fv[f] = sf[f * SB + s];
+          FOR_F(f) fv[f] = sf[f * SB + s];
           if (!having_ok(p, scnt[s], fv)) continue;
         }
         ++my;
@@ -658,7 +797,7 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
         int64_t r = counts[ci] + excl;
         for (int s = threadIdx.x; s < SB; s += blockDim.x) {
           if (scnt[s] <= 0) continue;
-          for (int f = 0; f < p.nf; ++f) fv[f] = sf[f * SB + s];
+          FOR_F(f) fv[f] = sf[f * SB + s];
           if (p.nhave && !having_ok(p, scnt[s], fv)) continue;
           int64_t kv[kMaxKey];
           decode_key(p, (uint64_t)(kbase + (uint32_t)s), kv);
