@@ -50,7 +50,7 @@ def parse():
     ap.add_argument("--sel", type=float, default=0.5)
     ap.add_argument("--rate", type=int, default=0)
     ap.add_argument("--tuples-log2", type=int, default=0, help="tuples per GPU (default: the config's)")
-    ap.add_argument("--task-mb", type=int, default=256)
+    ap.add_argument("--task-mb", type=int, default=1024, help="query task size φ in MiB")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -301,11 +301,13 @@ def main():
     times, stats_acc = [], []
     out_rows = out_tuples = out_windows = 0
     clk_dir = os.path.join(ROOT, "gpurun_out") if os.path.isdir(os.path.join(ROOT, "gpurun_out")) else "/tmp"
+    # one long-lived query; every step replays the stream after saber_query_reset
+    q = saber.Query(spec, base_index=base_index, first_window=first_window,
+                    emit_on_finish=(rank == world - 1), task_bytes=task_bytes,
+                    result_mode=saber.RESULTS_DEVICE, profile=True, result_slots=8, device=local)
     with Clocks(local, os.path.join(clk_dir, f"clocks_rank{rank}.csv")) as clk:
         for it in range(args.warmup + args.steps):
-            q = saber.Query(spec, base_index=base_index, first_window=first_window,
-                            emit_on_finish=(rank == world - 1), task_bytes=task_bytes,
-                            result_mode=saber.RESULTS_DEVICE, profile=True, result_slots=8, device=local)
+            q.reset(base_index, first_window)
             barrier()
             torch.cuda.synchronize()
             ev0 = torch.cuda.Event(enable_timing=True)
@@ -325,11 +327,11 @@ def main():
             torch.cuda.synchronize()
             ms = ev0.elapsed_time(ev1)
             st = q.stats()
-            q.close()
             if it >= args.warmup:
                 times.append(ms)
                 stats_acc.append(st)
                 out_windows, out_rows, out_tuples = counts()
+    q.close()
     clocks = clk.summary()
     ms_rank = statistics.median(times)
     print(f"[bench rank {rank}] device-resident step ms: {[round(t, 3) for t in times]}", file=sys.stderr)
@@ -364,10 +366,11 @@ def main():
         host_np = host.numpy()
         e_times = []
         d2h_bytes = 0
+        q = saber.Query(spec, task_bytes=task_bytes, result_mode=saber.RESULTS_HOST, device=local,
+                        base_index=base_index, first_window=first_window, emit_on_finish=(rank == world - 1))
+        q.register_host(host_np)
         for it in range(args.warmup + min(args.steps, 3)):
-            q = saber.Query(spec, task_bytes=task_bytes, result_mode=saber.RESULTS_HOST, device=local,
-                            base_index=base_index, first_window=first_window, emit_on_finish=(rank == world - 1))
-            q.register_host(host_np)
+            q.reset(base_index, first_window)
             barrier()
             torch.cuda.synchronize()
             t0 = time.perf_counter()
@@ -401,10 +404,10 @@ def main():
                 got_bytes += sum(k.nbytes for k in s.keys) + sum(v.nbytes for v in s.vals) + len(s.tuples) + s.nwindows * 32
             torch.cuda.synchronize()
             dt = time.perf_counter() - t0
-            q.close()
             if it >= args.warmup:
                 e_times.append(dt)
                 d2h_bytes = got_bytes
+        q.close()
         e_s = max_over_ranks(statistics.median(e_times))
         e2e = {"value": total_tuples / e_s, "unit": "tuples/s", "h2d_bytes_per_step": n * tb,
                "d2h_bytes_per_step": d2h_bytes, "s_per_step": e_s,

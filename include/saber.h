@@ -231,6 +231,11 @@ saber_status saber_query_stats(const saber_query *q, saber_stats *out);
 
 /* Block until all enqueued work of q is complete (results stay pending). */
 saber_status saber_query_sync(saber_query *q);
+/* Restart q on a new stream with the same plan and buffers (nothing is
+ * reallocated).  Every polled slice must have been released (else
+ * SABER_EAGAIN); results not yet polled are discarded; the sticky error and
+ * the statistics are cleared.  base_index / first_window as in saber_config. */
+saber_status saber_query_reset(saber_query *q, int64_t base_index, int64_t first_window);
 /* Make `cuda_stream` (a cudaStream_t; NULL = legacy default stream) wait for
  * all work enqueued on q so far, without blocking the host (stream-ordered
  * completion, e.g. for CUDA-event timing around a whole query). */

@@ -233,9 +233,10 @@ __global__ void k_carry(const Plan p, const State *st, const uint4 *task, const 
   }
 }
 
-__global__ void k_init_state(State *st, int64_t base_index, int64_t first_window, int64_t L) {
+__global__ void k_init_state(State *st, int64_t base_index, int64_t first_window, int64_t L, int64_t epoch0) {
   if (threadIdx.x) return;
   State s = {};
+  s.tile_epoch = epoch0;          // look-back epochs stay unique across resets
   s.pos_next = base_index;
   s.J0 = first_window;
   s.J1 = first_window;
@@ -297,8 +298,8 @@ cudaError_t launch_carry(const Plan &p, const QueryDev &q, const void *tuples, c
                                (uint4 *)q.carry[0], (uint4 *)q.carry[1]);
   return cudaGetLastError();
 }
-cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, cudaStream_t s) {
-  k_init_state<<<1, 32, 0, s>>>(q.st, base_index, p.first_window, p.L);
+cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, int64_t epoch0, cudaStream_t s) {
+  k_init_state<<<1, 32, 0, s>>>(q.st, base_index, p.first_window, p.L, epoch0);
   return cudaGetLastError();
 }
 cudaError_t launch_partition_plan(int ts_word, int tuple_words, int win_kind, int64_t s, int64_t l, int64_t T0,

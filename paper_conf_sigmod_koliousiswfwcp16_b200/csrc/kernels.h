@@ -38,7 +38,7 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
 cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
                                int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
                                int sel_grid, cudaStream_t st, cudaEvent_t *evs, int *launches);
-cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, cudaStream_t st);
+cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, int64_t epoch0, cudaStream_t st);
 cudaError_t launch_partition_plan(int ts_word, int tuple_words, int win_kind, int64_t s, int64_t l,
                                   int64_t T0, const void *tuples, int64_t begin, int64_t n,
                                   int64_t *dev_out2, cudaStream_t st);

@@ -83,6 +83,7 @@ struct saber_query {
   std::vector<void *> prereg;   // registered by someone else: never unregistered here
   std::mutex mu;
   int64_t *d_tmp = nullptr;
+  int64_t epoch_base = 0;       // look-back epoch offset across saber_query_reset
 };
 
 static saber_status fail(saber_query *q, saber_status s, const std::string &msg) {
@@ -463,7 +464,7 @@ static saber_status alloc_query(saber_query *q) {
   } else {
     q->sel_grid = sel_blocks_per_sm(p) * q->nsm;
   }
-  CK(launch_init_state(p, q->qd, q->cfg.base_index, q->cs));
+  CK(launch_init_state(p, q->qd, q->cfg.base_index, 0, q->cs));
   CK(cudaStreamSynchronize(q->cs));
   return SABER_OK;
 }
@@ -632,15 +633,20 @@ static bool is_registered(saber_query *q, const void *p, size_t n) {
   return false;
 }
 
-static saber_status ensure_stages(saber_query *q) {
-  if (!q->stages.empty()) return SABER_OK;
-  q->stages.resize(q->cfg.pipeline_depth);
+// device staging buffers are always needed for host submits; pinned host
+// staging only for the copyin path (unregistered caller memory)
+static saber_status ensure_stages(saber_query *q, bool need_host) {
   const size_t tb = (size_t)q->task_tuples * q->plan.tuple_bytes;
-  for (auto &g : q->stages) {
-    CK(cudaMallocHost(&g.h, tb));
-    CK(cudaMalloc(&g.d, tb));
-    CK(cudaEventCreateWithFlags(&g.free_ev, cudaEventDisableTiming));
+  if (q->stages.empty()) {
+    q->stages.resize(q->cfg.pipeline_depth);
+    for (auto &g : q->stages) {
+      CK(cudaMalloc(&g.d, tb));
+      CK(cudaEventCreateWithFlags(&g.free_ev, cudaEventDisableTiming));
+    }
   }
+  if (need_host)
+    for (auto &g : q->stages)
+      if (!g.h) CK(cudaMallocHost(&g.h, tb));
   return SABER_OK;
 }
 
@@ -672,7 +678,6 @@ saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t n
   const Plan &p = q->plan;
   if (nbytes % p.tuple_bytes) return fail(q, SABER_EINVAL, "nbytes is not a multiple of tuple_bytes");
   if (nbytes == 0) return SABER_OK;
-  if (saber_status s = ensure_stages(q)) return s;
   CK(cudaSetDevice(q->device));
   const int64_t tbytes = q->task_tuples * p.tuple_bytes;
   const int64_t whole = ((int64_t)nbytes + q->stage_fill) / tbytes;
@@ -680,6 +685,8 @@ saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t n
     return fail(q, SABER_EINVAL, "submit at most result_slots * task_bytes per call");
   if (whole > free_slots(q)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
   const bool reg = is_registered(q, host_tuples, nbytes);
+  const bool copyin = !reg || q->stage_fill > 0 || (int64_t)nbytes % tbytes != 0;
+  if (saber_status s = ensure_stages(q, copyin)) return s;
   const unsigned char *src = (const unsigned char *)host_tuples;
   int64_t left = (int64_t)nbytes;
   cudaEvent_t last_h2d = nullptr;
@@ -842,6 +849,33 @@ saber_status saber_query_stats(const saber_query *q, saber_stats *out) {
   if (!q || !out) return SABER_EINVAL;
   *out = q->stats;
   out->tasks_pending = q->next_task - q->next_poll;
+  return SABER_OK;
+}
+
+saber_status saber_query_reset(saber_query *q, int64_t base_index, int64_t first_window) {
+  if (!q || base_index < 0 || first_window < 0) return fail(q, SABER_EINVAL, "reset arguments");
+  std::lock_guard<std::mutex> lk(q->mu);
+  for (auto &s : q->slots)
+    if (s.state == SLOT_POLLED) return fail(q, SABER_EAGAIN, "release every polled slice before reset");
+  CK(cudaSetDevice(q->device));
+  CK(cudaStreamSynchronize(q->h2d));
+  CK(cudaStreamSynchronize(q->cs));
+  for (auto &s : q->slots) { s.state = SLOT_FREE; s.task_id = -1; s.profiled = false; }
+  for (auto &g : q->stages) g.used = false;
+  q->cfg.base_index = base_index;
+  q->cfg.first_window = first_window;
+  q->plan.first_window = first_window;
+  q->stage_fill = 0;
+  q->cur_stage = 0;
+  q->closed = false;
+  q->sticky = SABER_OK;
+  q->err.clear();
+  q->stats = saber_stats{};
+  // task ids restart at 0; look-back epochs continue past every task run so far
+  q->epoch_base += q->next_task + 1;
+  q->next_task = q->next_poll = 0;
+  CK(launch_init_state(q->plan, q->qd, base_index, q->epoch_base, q->cs));
+  CK(cudaStreamSynchronize(q->cs));
   return SABER_OK;
 }
 

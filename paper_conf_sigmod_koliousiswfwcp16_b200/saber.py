@@ -104,6 +104,7 @@ SIGNATURES = {
     "saber_query_stats": (C.c_int, [C.c_void_p, C.POINTER(Stats)]),
     "saber_query_sync": (C.c_int, [C.c_void_p]),
     "saber_query_record": (C.c_int, [C.c_void_p, C.c_void_p]),
+    "saber_query_reset": (C.c_int, [C.c_void_p, C.c_int64, C.c_int64]),
     "saber_query_destroy": (None, [C.c_void_p]),
     "saber_last_error": (C.c_char_p, [C.c_void_p]),
     "saber_partition_plan": (C.c_int, [C.POINTER(Schema), C.POINTER(Window), C.c_void_p, C.c_int64, C.c_int64,
@@ -293,6 +294,10 @@ class Query:
 
     def sync(self):
         _check(self.L.saber_query_sync(self.h), self.h)
+
+    def reset(self, base_index=0, first_window=0):
+        """Restart on a new stream, keeping the plan and every buffer."""
+        _check(self.L.saber_query_reset(self.h, int(base_index), int(first_window)), self.h)
 
     def record(self, stream=0):
         """Make CUDA stream `stream` wait for everything enqueued on this query."""
