@@ -1,174 +1,229 @@
-// k_select.cu -- σ/π with stream compaction (IStream), §5.4 L1315-1327.
+// k_select.cu -- σ/π with stream compaction (IStream): PAPER.md §5.4 L1315-1327.
+//
+// The paper evaluates the predicate into a binary vector in work-group memory
+// and prefix-sums it into contiguous output addresses per fragment, offset by
+// the fragment's start.  Here:
+//   k_select      every CTA streams a contiguous range of the task through
+//                 shared memory with 1-D TMA bulk copies (3 stages in flight),
+//                 evaluates σ per tuple, ranks the selected tuples with warp
+//                 ballots + a CTA scan per stage, and writes the projected rows,
+//                 compacted and in stream order, into its own staging segment
+//                 (starting at its range offset); its row count goes to cta_cnt;
+//   k_select_fix  each CTA segment is moved to its exclusive offset (a scan of
+//                 the per-CTA counts) -- no serial look-back chain between CTAs.
+// Only positions [cover_lo, cover_hi) -- tuples whose first window closed in
+// this task, position identity (reading A9) -- are emitted; the virtual input is
+// [carry (uncovered tail of earlier tasks) ++ task].
 #include <cuda_runtime.h>
 #include <stdint.h>
 
 #include "common.cuh"
 #include "launch_internal.h"
+#include "tma.cuh"
 
 namespace sb {
 
-constexpr int kSelThreads = 256;
-constexpr int kSelPer = 8;            // tuples per thread per tile
-constexpr int kSelTile = kSelThreads * kSelPer;
+constexpr int kSelThreads = 256, kSelWarps = 8;
+constexpr int kSelStageBytes = 32768;
+constexpr int kSelStages = 3;
+constexpr int kSelMaxIter = kSelStageBytes / 16 / kSelThreads;   // tuples per thread per stage (16-B tuples)
 
-// --------------------------------------------------------------------------
-// σ/π with stream compaction (IStream)
-__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t *p) {
-  uint64_t v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
-  return v;
+__device__ __forceinline__ int64_t sel_s_int(const unsigned char *t, int word, int type) {
+  return type == T_I32 ? (int64_t) * (const int32_t *)(t + 4 * word) : *(const int64_t *)(t + 4 * word);
 }
-__device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
-  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v));
-}
-constexpr uint64_t kFlagA = 1, kFlagP = 2;
-__device__ __forceinline__ uint64_t pack_status(uint64_t epoch, uint64_t flag, uint64_t v) {
-  return ((epoch & 0xffffffull) << 40) | (flag << 38) | (v & ((1ull << 38) - 1));
+__device__ __forceinline__ double sel_s_flt(const unsigned char *t, int word, int type) {
+  return type == T_F32 ? (double)*(const float *)(t + 4 * word) : *(const double *)(t + 4 * word);
 }
 
-template <int NW>
-__global__ void __launch_bounds__(kSelThreads)
-k_select(const Plan p, State *__restrict__ st, const uint4 *__restrict__ task,
-         const uint4 *__restrict__ carry0, const uint4 *__restrict__ carry1,
-         uint64_t *__restrict__ status, int *__restrict__ tile_ctr, unsigned char *__restrict__ rows) {
-  __shared__ int s_cnt[kSelPer][kSelThreads / 32];
-  __shared__ int s_off[kSelPer][kSelThreads / 32];
-  __shared__ int64_t s_tile, s_excl;
+__global__ void __launch_bounds__(kSelThreads, 2)
+k_select(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ task,
+         const unsigned char *__restrict__ carry0, const unsigned char *__restrict__ carry1,
+         unsigned char *__restrict__ stage_rows, int64_t *__restrict__ cta_cnt) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ int s_cnt[kSelMaxIter][kSelWarps];
+  __shared__ int s_off[kSelMaxIter][kSelWarps];
   __shared__ int s_total;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const int64_t lo = st->cover_lo, hi = st->cover_hi;
+  const int tb = p.tuple_bytes;
+  const int ST = kSelStageBytes / tb;                     // tuples per stage
+  const int NIT = ST / kSelThreads;                       // tuples per thread per stage
+  unsigned char *stages = smem;
+  uint64_t *full = (uint64_t *)(smem + kSelStages * kSelStageBytes);
+  uint64_t *empty = full + kSelStages;
+  const int64_t cl = st->cover_lo, ch = st->cover_hi;
   const int64_t tpos = st->task_pos, cpos = st->carry_pos;
-  const uint4 *carry = st->carry_sel ? carry1 : carry0;
-  const uint64_t epoch = (uint64_t)st->tile_epoch;
-  const int64_t ntiles = (hi - lo + kSelTile - 1) / kSelTile;
-  const int CW = NW / 4;
-  int err = 0;
-  for (;;) {
-    if (tid == 0) s_tile = atomicAdd(tile_ctr, 1);
-    __syncthreads();
-    const int64_t t = s_tile;
-    if (t >= ntiles) break;
-    const int64_t base = lo + t * kSelTile;
-    uint32_t w[kSelPer][NW];
-    bool sel[kSelPer];
-#pragma unroll
-    for (int k = 0; k < kSelPer; ++k) {
-      const int64_t pos = base + k * kSelThreads + tid;
-      if (pos < hi) {
-        const uint4 *src = pos < tpos ? carry + (pos - cpos) * CW : task + (pos - tpos) * CW;
-        load_tuple<NW>(src, (unsigned)p.chunk_mask, w[k]);
-      } else {
-#pragma unroll
-        for (int c = 0; c < NW; ++c) w[k][c] = 0;
-      }
-    }
-#pragma unroll
-    for (int k = 0; k < kSelPer; ++k) {
-      const int64_t pos = base + k * kSelThreads + tid;
-      const bool inb = pos < hi;
-      const int64_t tau = get_int<NW>(w[k], p.ts_word, T_I64);
-      int64_t up = (int64_t)shfl64((uint64_t)tau, (lane + 31) & 31);
-      if (lane == 0 && pos > cpos && inb) {
-        const int64_t pp = pos - 1;
-        const unsigned char *src = pp < tpos ? (const unsigned char *)carry + (pp - cpos) * p.tuple_bytes
-                                             : (const unsigned char *)task + (pp - tpos) * p.tuple_bytes;
-        up = *(const int64_t *)(src + 4 * p.ts_word);
-      } else if (lane == 0) {
-        up = INT64_MIN;
-      }
-      if (inb && tau < up) err |= ERR_ORDER;
-      if (inb && tau < 0) err |= ERR_TS;
-      bool s = inb;
-      if (p.win_kind == WK_TIME) s &= tau >= p.T0;
-      if (p.npred) s &= eval_preds<NW>(p, w[k]);
-      sel[k] = s;
-      const unsigned bal = __ballot_sync(kFull, s);
-      if (lane == 0) s_cnt[k][wid] = __popc(bal);
-    }
-    __syncthreads();
-    if (wid == 0) {
-      // 64 (k, warp) counts in order: lane holds 2 consecutive entries
-      const int i0 = 2 * lane, i1 = 2 * lane + 1;
-      const int c0 = s_cnt[i0 / 8][i0 % 8], c1 = s_cnt[i1 / 8][i1 % 8];
-      int x = c0 + c1;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int y = __shfl_up_sync(kFull, x, o);
-        if (lane >= o) x += y;
-      }
-      const int ex = x - c0 - c1;
-      s_off[i0 / 8][i0 % 8] = ex;
-      s_off[i1 / 8][i1 % 8] = ex + c0;
-      if (lane == 31) s_total = x;
-    }
-    __syncthreads();
-    if (tid == 0) {
-      // decoupled look-back over tiles (single pass)
-      const uint64_t total = (uint64_t)s_total;
-      int64_t excl = 0;
-      if (t == 0) {
-        st_relaxed(&status[0], pack_status(epoch, kFlagP, total));
-      } else {
-        st_relaxed(&status[t], pack_status(epoch, kFlagA, total));
-        int64_t i = t - 1;
-        for (;;) {
-          const uint64_t sv = ld_relaxed(&status[i]);
-          const uint64_t flag = (sv >> 38) & 3ull;
-          if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
-          excl += (int64_t)(sv & ((1ull << 38) - 1));
-          if (flag == kFlagP) break;
-          --i;
-        }
-        st_relaxed(&status[t], pack_status(epoch, kFlagP, (uint64_t)excl + total));
-      }
-      s_excl = excl;
-      if (t == ntiles - 1) st->sel_rows = excl + (int64_t)total;
-    }
-    __syncthreads();
-    const int64_t excl = s_excl;
-    const int ow = p.out_row_words;
-    const unsigned lt = (1u << lane) - 1u;
-#pragma unroll
-    for (int k = 0; k < kSelPer; ++k) {
-      const unsigned bal = __ballot_sync(kFull, sel[k]);
-      if (sel[k]) {
-        const int64_t r = excl + s_off[k][wid] + __popc(bal & lt);
-        uint32_t *dst = (uint32_t *)(rows + r * (int64_t)ow * 4);
-        if (r < p.rows_cap) {
-          if ((ow & 3) == 0) {
-            for (int c = 0; c < ow; c += 4)
-              *(uint4 *)(dst + c) = make_uint4(sel_word<NW>(w[k], p.proj_word[c]), sel_word<NW>(w[k], p.proj_word[c + 1]),
-                                               sel_word<NW>(w[k], p.proj_word[c + 2]), sel_word<NW>(w[k], p.proj_word[c + 3]));
-          } else {
-            for (int c = 0; c < ow; ++c) dst[c] = sel_word<NW>(w[k], p.proj_word[c]);
-          }
-        }
-      }
-    }
-    __syncthreads();
+  const unsigned char *carry = st->carry_sel ? carry1 : carry0;
+  // contiguous, stage-aligned range of this CTA within [cover_lo, cover_hi)
+  const int64_t n = ch - cl;
+  const int64_t per = ((n + gridDim.x - 1) / gridDim.x + ST - 1) / ST * ST;
+  const int64_t lo = cl + (int64_t)blockIdx.x * per;
+  const int64_t hi = lo + per < ch ? lo + per : ch;
+  const int nst = hi > lo ? (int)((hi - lo + ST - 1) / ST) : 0;
+  if (tid == 0) {
+    for (int i = 0; i < kSelStages; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], kSelWarps); }
+    fence_mbar_init();
   }
-  if (tid == 0 && ntiles == 0) { /* sel_rows already 0 from k_task_begin */ }
+  __syncthreads();
+  auto issue = [&](int k) {          // copy stage k of [carry ++ task]
+    const int slot = k % kSelStages;
+    const int64_t a = lo + (int64_t)k * ST, b = (a + ST < hi) ? a + ST : hi;
+    mbar_expect_tx(&full[slot], (uint32_t)((b - a) * tb));
+    unsigned char *dst = stages + slot * kSelStageBytes;
+    if (a < tpos) {
+      const int64_t e = b < tpos ? b : tpos;
+      bulk_g2s(dst, carry + (a - cpos) * tb, (uint32_t)((e - a) * tb), &full[slot]);
+      if (b > tpos) bulk_g2s(dst + (e - a) * tb, task, (uint32_t)((b - tpos) * tb), &full[slot]);
+    } else {
+      bulk_g2s(dst, task + (a - tpos) * tb, (uint32_t)((b - a) * tb), &full[slot]);
+    }
+  };
+  if (tid == 0)
+    for (int k = 0; k < kSelStages && k < nst; ++k) issue(k);
+  const int ow = p.out_row_words;
+  const unsigned ltmask = (1u << lane) - 1u;
+  unsigned char *out = stage_rows + (lo - cl) * (int64_t)ow * 4;   // this CTA's staging segment
+  int64_t written = 0;
+  int err = 0;
+  int64_t prev_tau = INT64_MIN;                    // τ of the tuple before the CTA range
+  if (lo < hi && lo > cpos) {
+    const int64_t pp = lo - 1;
+    prev_tau = *(const int64_t *)((pp < tpos ? carry + (pp - cpos) * tb : task + (pp - tpos) * tb) + 4 * p.ts_word);
+  }
+  for (int k = 0; k < nst; ++k) {
+    const int slot = k % kSelStages;
+    const uint32_t phase = (uint32_t)((k / kSelStages) & 1);
+    mbar_wait(&full[slot], phase);
+    const unsigned char *sb = stages + slot * kSelStageBytes;
+    const int64_t a = lo + (int64_t)k * ST;
+    const int ns = (int)((hi - a) < ST ? (hi - a) : ST);
+    unsigned bal[kSelMaxIter];
+#pragma unroll
+    for (int j = 0; j < kSelMaxIter; ++j) {
+      bal[j] = 0;
+      if (j >= NIT) continue;
+      const int i = j * kSelThreads + tid;
+      bool s = i < ns;
+      if (s) {
+        const unsigned char *tp = sb + i * tb;
+        const int64_t tau = *(const int64_t *)(tp + 4 * p.ts_word);
+        const int64_t up = i > 0 ? *(const int64_t *)(tp - tb + 4 * p.ts_word) : prev_tau;
+        if (tau < up) err |= ERR_ORDER;
+        if (tau < 0) err |= ERR_TS;
+        if (p.win_kind == WK_TIME) s &= tau >= p.T0;
+        for (int q = 0; q < p.npred && s; ++q) {
+          const Pred &pr = p.pred[q];
+          s = (pr.type == T_F32 || pr.type == T_F64) ? cmp_op(sel_s_flt(tp, pr.word, pr.type), pr.op, pr.fval)
+                                                      : cmp_op(sel_s_int(tp, pr.word, pr.type), pr.op, pr.ival);
+        }
+      }
+      bal[j] = __ballot_sync(kFull, s);
+      if (lane == 0) s_cnt[j][wid] = __popc(bal[j]);
+    }
+    prev_tau = *(const int64_t *)(sb + (ns - 1) * tb + 4 * p.ts_word);
+    __syncthreads();
+    if (wid == 0) {                                      // scan of the (j, warp) counts in stream order
+      int run = 0;
+      for (int b0 = 0; b0 < NIT * kSelWarps; b0 += 32) {
+        const int idx = b0 + lane;
+        const int v = idx < NIT * kSelWarps ? s_cnt[idx / kSelWarps][idx % kSelWarps] : 0;
+        int x = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(kFull, x, o);
+          if (lane >= o) x += y;
+        }
+        if (idx < NIT * kSelWarps) s_off[idx / kSelWarps][idx % kSelWarps] = run + x - v;
+        run += __shfl_sync(kFull, x, 31);
+      }
+      if (lane == 0) s_total = run;
+    }
+    __syncthreads();
+    // π: projected words of the selected tuples, compacted in stream order
+#pragma unroll
+    for (int j = 0; j < kSelMaxIter; ++j) {
+      if (j >= NIT) continue;
+      if (!((bal[j] >> lane) & 1u)) continue;
+      const int i = j * kSelThreads + tid;
+      const int64_t r = written + s_off[j][wid] + __popc(bal[j] & ltmask);
+      const uint32_t *src = (const uint32_t *)(sb + i * tb);
+      uint32_t *dst = (uint32_t *)(out + r * (int64_t)ow * 4);
+      if ((ow & 3) == 0) {
+        for (int c = 0; c < ow; c += 4)
+          *(uint4 *)(dst + c) = make_uint4(src[p.proj_word[c]], src[p.proj_word[c + 1]], src[p.proj_word[c + 2]],
+                                           src[p.proj_word[c + 3]]);
+      } else {
+        for (int c = 0; c < ow; ++c) dst[c] = src[p.proj_word[c]];
+      }
+    }
+    written += s_total;
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[slot]);
+    if (tid == 0 && k + kSelStages < nst) {
+      mbar_wait(&empty[slot], phase);
+      issue(k + kSelStages);
+    }
+  }
+  if (tid == 0) cta_cnt[blockIdx.x] = written;
   if (err) atomicOr(&st->error, err);
 }
 
-}  // namespace sb
-
-namespace sb {
-
-void *sel_kernel(const Plan &p) {
-  switch (p.tuple_words) {
-    case 4: return (void *)k_select<4>;
-    case 8: return (void *)k_select<8>;
-    case 12: return (void *)k_select<12>;
-    default: return (void *)k_select<16>;
+// move every CTA's staged rows to its exclusive offset in the result slot
+__global__ void __launch_bounds__(256)
+k_select_fix(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ stage_rows,
+             const int64_t *__restrict__ cta_cnt, int ncta, unsigned char *__restrict__ rows) {
+  __shared__ int64_t s_part[8];
+  __shared__ int64_t s_base;
+  const int b = blockIdx.x;
+  if (b >= ncta) return;
+  const int64_t cl = st->cover_lo, ch = st->cover_hi;
+  const int tb = p.tuple_bytes;
+  const int ST = kSelStageBytes / tb;
+  const int64_t n = ch - cl;
+  const int64_t per = ((n + ncta - 1) / ncta + ST - 1) / ST * ST;
+  // exclusive prefix of the counts of CTAs < b (block reduction)
+  int64_t x = 0;
+  for (int i = threadIdx.x; i < b; i += blockDim.x) x += cta_cnt[i];
+#pragma unroll
+  for (int o = 16; o; o >>= 1) x += (int64_t)__shfl_xor_sync(kFull, (unsigned long long)x, o);
+  if ((threadIdx.x & 31) == 0) s_part[threadIdx.x >> 5] = x;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int64_t s = 0;
+    for (int w = 0; w < 8; ++w) s += s_part[w];
+    s_base = s;
+    if (b == ncta - 1) {
+      st->sel_rows = s + cta_cnt[b];
+      if (s + cta_cnt[b] > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+    }
+  }
+  __syncthreads();
+  const int64_t base = s_base, cnt = cta_cnt[b];
+  const int64_t rb = (int64_t)p.out_row_words * 4;
+  const int64_t nbytes = cnt * rb;
+  if (base + cnt > p.rows_cap) return;
+  const unsigned char *src = stage_rows + (int64_t)b * per * rb;
+  unsigned char *dst = rows + base * rb;
+  if ((rb & 15) == 0) {
+    for (int64_t i = threadIdx.x; i < nbytes / 16; i += blockDim.x)
+      ((uint4 *)dst)[i] = ((const uint4 *)src)[i];
+  } else {
+    for (int64_t i = threadIdx.x; i < nbytes / 4; i += blockDim.x)
+      ((uint32_t *)dst)[i] = ((const uint32_t *)src)[i];
   }
 }
+
+void *sel_kernel(const Plan &p) { return (void *)k_select; }
+
+int sel_smem_bytes() { return kSelStages * kSelStageBytes + 2 * kSelStages * 8; }
 
 cudaError_t launch_select(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int grid,
                           cudaStream_t st) {
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&tuples, (void *)&q.carry[0], (void *)&q.carry[1],
-                  (void *)&q.tile_status, (void *)&q.tile_ctr, (void *)&s.rows};
-  return cudaLaunchKernel(sel_kernel(p), dim3(grid), dim3(kSelThreads), args, 0, st);
+                  (void *)&q.sel_stage, (void *)&q.cta_cnt};
+  cudaError_t e = cudaLaunchKernel(sel_kernel(p), dim3(grid), dim3(kSelThreads), args, (size_t)sel_smem_bytes(), st);
+  if (e) return e;
+  k_select_fix<<<grid, 256, 0, st>>>(p, q.st, q.sel_stage, q.cta_cnt, grid, s.rows);
+  return cudaGetLastError();
 }
 
 }  // namespace sb

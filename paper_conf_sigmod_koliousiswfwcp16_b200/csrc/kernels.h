@@ -21,6 +21,8 @@ struct QueryDev {
   uint64_t *vh_suf;         // van Herk block-suffix arrays
   uint64_t *clist;          // slab mode: per pane slot, entries bucketed by key range
   int32_t *coff;            // slab mode: per pane slot, S+1 bucket offsets
+  unsigned char *sel_stage; // σ/π: per-CTA compacted rows before the final placement
+  int64_t *cta_cnt;         // σ/π: rows per CTA
   int64_t *pane_ts;         // R
   uint64_t *tile_status;    // IStream look-back
   int64_t tile_status_cap;

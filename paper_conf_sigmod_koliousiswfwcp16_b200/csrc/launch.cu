@@ -8,6 +8,7 @@ namespace sb {
 
 cudaError_t set_kernel_attributes(const Plan &p) {
   cudaError_t e = cudaSuccess;
+  if (p.nagg == 0) return cudaFuncSetAttribute(sel_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem_bytes());
   if (p.nagg > 0) {
     e = cudaFuncSetAttribute(p1_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p1_smem_bytes(p));
     if (e) return e;
@@ -33,7 +34,7 @@ int p2_blocks_per_sm(const Plan &p) {
 }
 int sel_blocks_per_sm(const Plan &p) {
   int b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sel_kernel(p), 256, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sel_kernel(p), 256, sel_smem_bytes());
   return b > 0 ? b : 1;
 }
 
@@ -78,7 +79,7 @@ cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &
   if (evs) cudaEventRecord(evs[1], st);
   if ((e = launch_carry(p, q, tuples, st))) return e;
   if ((e = launch_task_end(p, q, s, st))) return e;
-  *launches = 4;
+  *launches = 5;
   if (evs) cudaEventRecord(evs[2], st);
   return cudaGetLastError();
 }

@@ -29,6 +29,7 @@ cudaError_t launch_windows_slab(const Plan &p, const QueryDev &q, const SlotDev 
 void *slab_kernel(bool emit);
 // k_select.cu
 void *sel_kernel(const Plan &p);
+int sel_smem_bytes();
 cudaError_t launch_select(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int grid,
                           cudaStream_t st);
 }  // namespace sb

@@ -434,9 +434,8 @@ static saber_status alloc_query(saber_query *q) {
     q->qd.carry_cap = p.carry_cap;
     CK(cudaMalloc(&q->qd.carry[0], (size_t)p.carry_cap * p.tuple_bytes));
     CK(cudaMalloc(&q->qd.carry[1], (size_t)p.carry_cap * p.tuple_bytes));
-    q->qd.tile_status_cap = (q->task_tuples + p.carry_cap) / 2048 + 4;
-    CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
-    CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
+    CK(cudaMalloc(&q->qd.sel_stage, (size_t)p.rows_cap * p.out_row_words * 4 + 16));
+    CK(cudaMalloc(&q->qd.cta_cnt, 8192 * sizeof(int64_t)));
   }
   const int nslots = q->cfg.result_slots > 0 ? q->cfg.result_slots : 8;
   q->slots.resize(nslots);
@@ -586,7 +585,7 @@ void saber_query_destroy(saber_query *q) {
   for (auto &r : q->registered)
     if (std::find(q->prereg.begin(), q->prereg.end(), r.first) == q->prereg.end()) cudaHostUnregister(r.first);
   cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.vh_pre); cudaFree(q->qd.vh_suf);
-  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
+  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.sel_stage); cudaFree(q->qd.cta_cnt); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
   cudaFree(q->qd.carry[0]); cudaFree(q->qd.carry[1]); cudaFree(q->qd.tile_ctr); cudaFree(q->d_tmp);
   if (q->cs) cudaStreamDestroy(q->cs);
   if (q->h2d) cudaStreamDestroy(q->h2d);
