@@ -205,6 +205,28 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
 
   // sum the warp (and lane) copies of each entry, one set of L2 REDs per entry
   auto flush_shared = [&]() {
+    if (MODE == TM_LANE) {
+      // each warp first folds its 32 lane columns into lane 0's copy (shuffles)
+      __syncwarp();
+      for (int e = 0; e < TE; ++e) {
+        const int x = e * 32 + lane;
+        const uint32_t cl = tcnt[x];
+        if (!__any_sync(kFull, cl != 0)) continue;
+        const uint32_t c = __reduce_add_sync(kFull, cl);
+        if (lane == 0) tcnt[x] = c; else tcnt[x] = 0;
+#pragma unroll
+        for (int f = 0; f < NF; ++f) {
+          if (!FAST && f >= p.nf) break;
+          const int kind = FAST ? FK_SUM_F : p.field[f].kind;
+          uint64_t v = tf[f * TE * 32 + x];
+#pragma unroll
+          for (int o = 16; o; o >>= 1)
+            v = FAST ? fadd64(v, shfl_xor64(v, o)) : field_combine(kind, v, shfl_xor64(v, o));
+          tf[f * TE * 32 + x] = lane == 0 ? v : field_identity(kind);
+        }
+      }
+      __syncwarp();
+    }
     __syncthreads();
     for (int e = tid; e < TE; e += kP1Threads) {
       uint32_t c = 0;
@@ -214,8 +236,8 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
       for (int w = 0; w < NCOPY; ++w) {
         uint64_t *of = (uint64_t *)(tabs + (size_t)w * p.local_bytes);
         uint32_t *oc = (uint32_t *)((unsigned char *)of + (size_t)8 * TE * CW * NF);
-        for (int l = 0; l < CW; ++l) {
-          const int x = e * CW + ((l + tid) & (CW - 1));   // rotate lanes: fewer bank conflicts
+        for (int l = 0; l < (MODE == TM_LANE ? 1 : CW); ++l) {
+          const int x = e * CW + l;                        // LANE: lane 0 holds the warp total
           const uint32_t cw = oc[x];
           if (!cw) continue;
           c += cw;
@@ -251,13 +273,16 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     occ = 0;
   };
 
-  for (int k = 0; k < nst; ++k) {
-    const int slot = k % kStages;
-    const uint32_t phase = (uint32_t)((k / kStages) & 1);
+  // count windows: 32-bit pane arithmetic when a pane window spans < 2^30 positions
+  const int g32 = (p.g * (int64_t)(PL + 2) < (1ll << 30)) ? (int)p.g : 0;
+  const int range32 = (int)(hi - lo);                     // tuples of this CTA (< 2^31)
+  int64_t spos = pos0 + lo;                               // global position of stage tuple 0
+  int slot = 0;
+  uint32_t phase = 0;
+  for (int k = 0; k < nst; ++k, spos += ST) {
     mbar_wait(&full[slot], phase);
     const unsigned char *sb = stages + slot * kStageBytes;
-    const int ntup = (int)((hi - lo - (int64_t)k * ST) < ST ? (hi - lo - (int64_t)k * ST) : ST);
-    const int64_t spos = pos0 + lo + (int64_t)k * ST;     // global position of stage tuple 0
+    const int ntup = range32 - k * ST < ST ? range32 - k * ST : ST;
     int64_t pf, pl;                                        // stage pane range (CTA-uniform)
     if (WK == WK_COUNT) {
       pf = pdiv(p, spos);
@@ -285,9 +310,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
       const int64_t wlo = pbase > min_pane ? pbase : min_pane;
       const bool all_in = (pf >= wlo) & (pl < wend);    // CTA-uniform: no per-tuple window test
       const int lo_ofs = (int)(wlo - pbase);             // first live offset in the window
-      // count windows: this lane's tuple as (pane offset from pbase, position in the pane),
-      // 32-bit when the pane window spans < 2^30 positions (g32 > 0)
-      const int g32 = (p.g * (int64_t)(PL + 2) < (1ll << 30)) ? (int)p.g : 0;
+      // count windows: this lane's tuple as (pane offset from pbase, position in the pane)
       int po = 0, cr = 0;
       int64_t cp = 0;
       if (WK == WK_COUNT) {
@@ -301,6 +324,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
           cr = (int)(pos - cp * p.g);
         }
       }
+#pragma unroll 2
       for (int i0 = ib; i0 < ie; i0 += 32) {
         const int i = i0 + lane;
         bool valid = i < ie;
@@ -432,6 +456,9 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     if (tid == 0 && k + kStages < nst) {
       mbar_wait(&empty[slot], phase);
       issue(k + kStages);
+    }
+    if (++slot == kStages) { slot = 0; phase ^= 1u; }
+    if (false) {
     }
   }
   if (pbase >= 0) {
