@@ -63,7 +63,8 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
     st->zero_hi = zhi;
     if (zhi > st->zeroed_hi) st->zeroed_hi = zhi;
     if (phi > st->pane_hi) st->pane_hi = phi;
-    (void)plo;
+    meta->in_tuples = n;
+    meta->in_panes = (n > 0 && phi >= plo) ? phi - plo + 1 : 0;
     if (J1 - J0 > p.win_cap) err |= ERR_RESULT;
     meta->first_window = J0;
     meta->nwindows = J1 - J0;

@@ -74,6 +74,8 @@ struct Plan {
   int32_t local_entries;          // entries per warp
   int32_t local_pl;               // panes per direct table
   int32_t local_bytes;            // bytes per warp
+  int32_t lane_alt;               // DIRECT plan that may switch to LANE per task (time windows)
+  int32_t lane_pl, lane_entries, lane_bytes;
   int32_t fast_path, pad6;        // all fields fp64 sums of f32 columns, <= 1 int32 key (div 1), nf <= 2
   // phase-2 window assembly
   int32_t S, SB, GS, pad5;        // key slabs, slots per slab, threads per slab group
@@ -118,6 +120,7 @@ struct SlotMeta {
   int64_t first_window, nwindows, nrows, ntuples;
   int32_t error, pad;
   int64_t pos_end, tau_last;
+  int64_t in_tuples, in_panes;    // this task's input tuples and the panes they span
 };
 
 }  // namespace sb

@@ -75,6 +75,9 @@ struct saber_query {
   int64_t task_tuples = 0;
   int64_t next_task = 0, next_poll = 0;
   int p1_grid = 0, p2_grid = 0, sel_grid = 0, win_chunk = 32;
+  Plan plan_lane{};             // plan.lane_alt: the same plan with lane-private tables
+  int p1_grid_lane = 0;
+  bool use_lane = false;        // completed tasks showed long panes (set in poll)
   bool closed = false;
   saber_status sticky = SABER_OK;
   std::string err;
@@ -305,13 +308,25 @@ static saber_status size_plan(saber_query *q) {
     const int nft = p.nf <= 1 ? 1 : p.nf <= 2 ? 2 : p.nf <= 4 ? 4 : 8;
     const int ed = 4 + 8 * nft, eh = 12 + 8 * nft;
     const int lane_budget = 8 * 1024, direct_budget = 2560, hash_budget = 5 * 1024;
-    if (p.key_mode != KM_HASH && p.C * 2 * 32 * ed <= lane_budget) {
+    // lane-private tables flush once per few panes: worth it for one key (no GROUP BY:
+    // atomics would all hit one address) or count windows with long panes; time
+    // windows of unknown rate with several keys take warp tables instead
+    const bool lane_ok = p.C == 1 || (p.win_kind == WK_COUNT && p.g >= 64 * p.C);
+    if (p.key_mode != KM_HASH && lane_ok && p.C * 2 * 32 * ed <= lane_budget) {
       p.local_mode = 0;
       p.local_pl = (int)std::min<int64_t>(1024, lane_budget / (32 * ed * p.C));
       p.local_entries = p.local_pl * (int)p.C;
       p.local_bytes = ((p.local_entries * 32 * ed) + 15) & ~15;
     } else if (p.key_mode != KM_HASH && p.C * 2 * ed <= direct_budget) {
       p.local_mode = 1;
+      // time windows: switch to lane-private tables per task once completed tasks show
+      // long panes (>= 64·C tuples per pane), see enqueue_task
+      if (p.win_kind == WK_TIME && p.C * 2 * 32 * ed <= lane_budget) {
+        p.lane_alt = 1;
+        p.lane_pl = (int)std::min<int64_t>(1024, lane_budget / (32 * ed * p.C));
+        p.lane_entries = p.lane_pl * (int)p.C;
+        p.lane_bytes = ((p.lane_entries * 32 * ed) + 15) & ~15;
+      }
       p.local_pl = (int)std::min<int64_t>(1024, direct_budget / (ed * p.C));
       p.local_entries = p.local_pl * (int)p.C;
       p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
@@ -457,6 +472,16 @@ static saber_status alloc_query(saber_query *q) {
   }
   CK(set_kernel_attributes(p));
   CK(cudaDeviceGetAttribute(&q->nsm, cudaDevAttrMultiProcessorCount, q->device));
+  if (p.lane_alt) {
+    Plan &pl = q->plan_lane;
+    pl = p;
+    pl.local_mode = 0;
+    pl.local_pl = p.lane_pl;
+    pl.local_entries = p.lane_entries;
+    pl.local_bytes = p.lane_bytes;
+    CK(set_kernel_attributes(pl));
+    q->p1_grid_lane = p1_blocks_per_sm(pl) * q->nsm;
+  }
   if (p.nagg > 0) {
     q->p1_grid = p1_blocks_per_sm(p) * q->nsm;
     q->p2_grid = p2_blocks_per_sm(p) * q->nsm * 2;
@@ -483,12 +508,14 @@ static int free_slots(saber_query *q) {
 static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuples, int final_, int has_wm, int64_t wm) {
   Slot &s = q->slots[q->next_task % (int64_t)q->slots.size()];
   if (s.state != SLOT_FREE) return fail(q, SABER_EAGAIN, "no free result slot");
-  const Plan &p = q->plan;
+  const bool lane = q->plan.lane_alt && q->use_lane;
+  const Plan &p = lane ? q->plan_lane : q->plan;
   cudaError_t e;
   int launches = 0;
   cudaEvent_t *evs = q->cfg.profile ? s.prof : nullptr;
   if (p.nagg > 0)
-    e = launch_agg_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish, q->p1_grid,
+    e = launch_agg_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish,
+                        lane ? q->p1_grid_lane : q->p1_grid,
                         q->p2_grid, q->win_chunk, q->cs, evs, &launches);
   else
     e = launch_select_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish, q->sel_grid,
@@ -786,6 +813,9 @@ saber_status saber_results_poll(saber_query *q, saber_results *out, int32_t time
   }
   s.meta = *s.h_meta;
   const Plan &p = q->plan;
+  // pane density of large tasks picks the phase-1 table layout of later tasks
+  if (p.lane_alt && s.meta.in_tuples >= (1 << 20) && s.meta.in_panes > 0)
+    q->use_lane = s.meta.in_tuples >= 64 * p.C * s.meta.in_panes;
   if (s.profiled) {
     float a = 0, b = 0;
     if (cudaEventElapsedTime(&a, s.prof[0], s.prof[1]) == cudaSuccess && s.scanned) q->stats.scan_ms += a;

@@ -118,6 +118,17 @@ def test_c4_cm1(saber, oracle_lib, rate):
     check(saber, oracle_lib, spec, data, task_bytes=(2 << 20))
 
 
+@pytest.mark.parametrize("rate", [128, 4096])
+def test_c4_table_layout_switch(saber, oracle_lib, rate):
+    """Time windows with GROUP BY start with warp tables and switch to lane-private
+    tables once polled tasks (>= 1M tuples) show long panes: results must not change."""
+    spec, g = workloads.c4(rate=rate)
+    n = 1 << 22
+    data = gen.generate("cm", n, g["seed"], rate=rate, groups=g["groups"])
+    tb = len(data) // n
+    check(saber, oracle_lib, spec, data, task_bytes=tb * (1 << 20), result_slots=2)
+
+
 def test_c5a_sg2_and_sg1(saber, oracle_lib):
     for spec, g in (workloads.c5a(), workloads.sg1()):
         spec["window"]["size"] = 60          # shorter window so the oracle stays fast
