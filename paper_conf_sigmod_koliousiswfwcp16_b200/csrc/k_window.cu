@@ -414,6 +414,129 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
   }
 }
 
+// ---------------------------------------------------------------------------
+// Few keys (C <= 32, one slab): a warp holds 32/Cp windows side by side, lane =
+// (window, key slot), Cp = C rounded up to a power of two, so no lane idles on a
+// 4-key GROUP BY or a GLOBAL aggregate.  Row order is window-major, key order
+// inside a window, exactly as k_win_fused.  One ballot per (pass, warp) gives
+// every window's row count and every row's offset.
+constexpr int kPackU = 4;     // window passes per warp per chunk
+
+template <bool F>
+__device__ __forceinline__ bool win_value(const Plan &p, const uint64_t *__restrict__ pre,
+                                          const uint64_t *__restrict__ suf, int64_t j, int s, int64_t &c,
+                                          uint64_t (&fv)[kMaxField]) {
+  const int64_t a = j * p.L;
+  const bool aligned = (a % p.K) == 0;
+  const uint64_t *sa = suf + (a & (p.R - 1)) * p.slot_words;
+  const uint64_t *pb = pre + ((a + p.K - 1) & (p.R - 1)) * p.slot_words;
+  c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
+  if (c <= 0) return false;
+  if constexpr (F) {
+    FOR_F(f) {
+      const uint64_t x = sa[vh_off(p, f) + s];
+      fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
+    }
+    return !p.nhave || having_ok(p, c, fv);
+  }
+  return true;
+}
+
+__global__ void __launch_bounds__(256)
+k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre, const uint64_t *__restrict__ suf,
+             const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
+             uint64_t *__restrict__ status, int *__restrict__ ticket, int cshift) {
+  __shared__ int s_wcnt[8];
+  __shared__ int64_t s_base;
+  __shared__ int s_t;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int WPW = 32 >> cshift;                       // windows per warp pass
+  const int wsub = lane >> cshift, slot = lane & ((1 << cshift) - 1);
+  const unsigned seg_lt = (1u << (wsub << cshift)) - 1u;            // lanes of earlier windows
+  const unsigned seg = cshift == 5 ? kFull : (((1u << (1 << cshift)) - 1u) << (wsub << cshift));
+  const unsigned lt = (1u << lane) - 1u;
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  if (nw <= 0) return;
+  const uint64_t epoch = (uint64_t)st->tile_epoch;
+  const int WC = 8 * kPackU * WPW;
+  const int64_t nchunks = (nw + WC - 1) / WC;
+  for (;;) {
+    if (threadIdx.x == 0) s_t = atomicAdd(ticket, 1);
+    __syncthreads();
+    const int64_t t = s_t;
+    if (t >= nchunks) break;
+    const int64_t wb = J0 + t * WC + (int64_t)warp * kPackU * WPW + wsub;
+    unsigned bal[kPackU];
+    int wtot = 0;
+#pragma unroll
+    for (int u = 0; u < kPackU; ++u) {
+      const int64_t j = wb + u * WPW;
+      bool present = false;
+      if (j < J1 && slot < p.C) {
+        int64_t c;
+        uint64_t fv[kMaxField];
+        present = p.nhave ? win_value<true>(p, pre, suf, j, slot, c, fv) : win_value<false>(p, pre, suf, j, slot, c, fv);
+      }
+      bal[u] = __ballot_sync(kFull, present);
+      wtot += __popc(bal[u]);
+    }
+    if (lane == 0) s_wcnt[warp] = wtot;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int run = 0;
+      for (int w = 0; w < 8; ++w) { const int v = s_wcnt[w]; s_wcnt[w] = run; run += v; }
+      const uint64_t total = (uint64_t)run;
+      int64_t excl = 0;
+      if (t == 0) {
+        lb_st(&status[0], lb_pack(epoch, 2, total));
+      } else {
+        lb_st(&status[t], lb_pack(epoch, 1, total));
+        for (int64_t i = t - 1;;) {
+          const uint64_t sv = lb_ld(&status[i]);
+          const uint64_t flag = (sv >> 38) & 3ull;
+          if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
+          excl += (int64_t)(sv & ((1ull << 38) - 1));
+          if (flag == 2) break;
+          --i;
+        }
+        lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
+      }
+      s_base = excl;
+      if (t == nchunks - 1) {
+        st->sel_rows = excl + (int64_t)total;
+        if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+      }
+    }
+    __syncthreads();
+    int64_t r = s_base + s_wcnt[warp];
+#pragma unroll
+    for (int u = 0; u < kPackU; ++u) {
+      const int64_t j = wb + u * WPW;
+      if (j < J1) {
+        if (slot == 0) {
+          WinHdr h;
+          h.window_id = j;
+          h.ts = (p.win_kind == WK_TIME) ? p.T0 + j * p.l : pane_ts[(j * p.L) & (p.R - 1)];
+          h.row_offset = r + __popc(bal[u] & seg_lt);
+          h.nrows = __popc(bal[u] & seg);
+          h.flags = 0;
+          hdr[j - J0] = h;
+        }
+        if ((bal[u] >> lane) & 1u) {
+          int64_t c;
+          uint64_t fv[kMaxField];
+          win_value<true>(p, pre, suf, j, slot, c, fv);
+          int64_t kv[kMaxKey];
+          decode_key(p, (uint64_t)slot, kv);
+          write_row(p, rows, r + __popc(bal[u] & lt), kv, c, fv);
+        }
+      }
+      r += __popc(bal[u]);
+    }
+    __syncthreads();
+  }
+}
+
 // (window, slab) items; a group of GS threads owns the slots of one item
 template <bool EMIT>
 __global__ void __launch_bounds__(256)
@@ -625,6 +748,13 @@ cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev
   if (p.K > 64 && p.slot_words < 64) k_vh_build_long<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   else if (p.K > 64) k_vh_build_warp<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   else k_vh_build<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  if (p.S == 1 && p.C <= 32) {
+    int cshift = 0;
+    while ((1 << cshift) < p.C) ++cshift;
+    k_win_packed<<<grid, 256, 0, st>>>(p, q.st, q.vh_pre, q.vh_suf, q.pane_ts, (WinHdr *)s.hdr, s.rows,
+                                       q.tile_status, q.tile_ctr, cshift);
+    return cudaGetLastError();
+  }
   const int gpb = 256 / p.GS;
   int wc = gpb * 8 / p.S;
   if (wc * p.S > kFusedMaxItems) wc = kFusedMaxItems / p.S;
