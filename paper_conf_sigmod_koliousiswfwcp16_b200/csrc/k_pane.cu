@@ -144,6 +144,67 @@ __device__ __forceinline__ void flush_entry(const Plan &p, State *st, uint64_t *
     if (i < p.nf) red_field(p.field[i].kind, &base[fld_off(p, i) + idx], fv[i]);
 }
 
+// sum the warp (and lane) copies of each table entry of the pane window starting
+// at pbase, one set of L2 REDs per (pane, key) per CTA; CTA-collective
+template <int MODE, int NF, bool FAST>
+__device__ __forceinline__ void flush_tables(const Plan &p, State *st, uint64_t *table, unsigned char *tabs,
+                                          uint64_t *tf, uint32_t *tcnt, int64_t pbase, int &err) {
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int TE = p.local_entries;
+  const int CW = MODE == TM_LANE ? 32 : 1;
+  constexpr int NCOPY = MODE == TM_SHARED ? 1 : kP1Warps;
+  const int C = (int)p.C;
+
+  if (MODE == TM_LANE) {
+    // each warp first folds its 32 lane columns into lane 0's copy (shuffles)
+    __syncwarp();
+    for (int e = 0; e < TE; ++e) {
+      const int x = e * 32 + lane;
+      const uint32_t cl = tcnt[x];
+      if (!__any_sync(kFull, cl != 0)) continue;
+      const uint32_t c = __reduce_add_sync(kFull, cl);
+      if (lane == 0) tcnt[x] = c; else tcnt[x] = 0;
+#pragma unroll
+      for (int f = 0; f < NF; ++f) {
+        if (!FAST && f >= p.nf) break;
+        const int kind = FAST ? FK_SUM_F : p.field[f].kind;
+        uint64_t v = tf[f * TE * 32 + x];
+#pragma unroll
+        for (int o = 16; o; o >>= 1)
+          v = FAST ? fadd64(v, shfl_xor64(v, o)) : field_combine(kind, v, shfl_xor64(v, o));
+        tf[f * TE * 32 + x] = lane == 0 ? v : field_identity(kind);
+      }
+    }
+    __syncwarp();
+  }
+  __syncthreads();
+  for (int e = tid; e < TE; e += kP1Threads) {
+    uint32_t c = 0;
+    uint64_t fv[NF];
+#pragma unroll
+    for (int f = 0; f < NF; ++f) fv[f] = f < p.nf ? field_identity(p.field[f].kind) : 0;
+    for (int w = 0; w < NCOPY; ++w) {
+      uint64_t *of = (uint64_t *)(tabs + (size_t)w * p.local_bytes);
+      uint32_t *oc = (uint32_t *)((unsigned char *)of + (size_t)8 * TE * CW * NF);
+      for (int l = 0; l < (MODE == TM_LANE ? 1 : CW); ++l) {
+        const int x = e * CW + l;                        // LANE: lane 0 holds the warp total
+        const uint32_t cw = oc[x];
+        if (!cw) continue;
+        c += cw;
+        oc[x] = 0;
+#pragma unroll
+        for (int f = 0; f < NF; ++f)
+          if (f < p.nf) {
+            fv[f] = field_combine(p.field[f].kind, fv[f], of[f * TE * CW + x]);
+            of[f * TE * CW + x] = field_identity(p.field[f].kind);
+          }
+      }
+    }
+    if (c) flush_entry<NF>(p, st, table, pbase + e / C, (uint64_t)(e % C), c, fv, err);
+  }
+  __syncthreads();
+}
+
 template <int MODE, int WK, int NF, bool FAST>
 __global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? 3 : 2)
 k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
@@ -160,7 +221,6 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   // table geometry: TE entries per warp; LANE mode stores every entry once per lane
   const int TE = p.local_entries;
   const int CW = MODE == TM_LANE ? 32 : 1;               // copies of an entry (lanes)
-  constexpr int NCOPY = MODE == TM_SHARED ? 1 : kP1Warps;  // one table per warp, or one per CTA
   unsigned char *wt = tabs + (MODE == TM_SHARED ? 0 : (size_t)wid * p.local_bytes);
   uint64_t *tkeys = (uint64_t *)wt;                      // HASHED only
   uint64_t *tf = (uint64_t *)(wt + (MODE == TM_HASHED ? 8 * TE : 0));   // [NF][TE*CW]
@@ -203,57 +263,7 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   int64_t prev_last = (lo > 0 && lo < hi) ? *(const int64_t *)(tup + (lo - 1) * tb + 4 * tsw) : INT64_MIN;
   const int per_warp = (ST + kP1Warps - 1) / kP1Warps;
 
-  // sum the warp (and lane) copies of each entry, one set of L2 REDs per entry
-  auto flush_shared = [&]() {
-    if (MODE == TM_LANE) {
-      // each warp first folds its 32 lane columns into lane 0's copy (shuffles)
-      __syncwarp();
-      for (int e = 0; e < TE; ++e) {
-        const int x = e * 32 + lane;
-        const uint32_t cl = tcnt[x];
-        if (!__any_sync(kFull, cl != 0)) continue;
-        const uint32_t c = __reduce_add_sync(kFull, cl);
-        if (lane == 0) tcnt[x] = c; else tcnt[x] = 0;
-#pragma unroll
-        for (int f = 0; f < NF; ++f) {
-          if (!FAST && f >= p.nf) break;
-          const int kind = FAST ? FK_SUM_F : p.field[f].kind;
-          uint64_t v = tf[f * TE * 32 + x];
-#pragma unroll
-          for (int o = 16; o; o >>= 1)
-            v = FAST ? fadd64(v, shfl_xor64(v, o)) : field_combine(kind, v, shfl_xor64(v, o));
-          tf[f * TE * 32 + x] = lane == 0 ? v : field_identity(kind);
-        }
-      }
-      __syncwarp();
-    }
-    __syncthreads();
-    for (int e = tid; e < TE; e += kP1Threads) {
-      uint32_t c = 0;
-      uint64_t fv[NF];
-#pragma unroll
-      for (int f = 0; f < NF; ++f) fv[f] = f < p.nf ? field_identity(p.field[f].kind) : 0;
-      for (int w = 0; w < NCOPY; ++w) {
-        uint64_t *of = (uint64_t *)(tabs + (size_t)w * p.local_bytes);
-        uint32_t *oc = (uint32_t *)((unsigned char *)of + (size_t)8 * TE * CW * NF);
-        for (int l = 0; l < (MODE == TM_LANE ? 1 : CW); ++l) {
-          const int x = e * CW + l;                        // LANE: lane 0 holds the warp total
-          const uint32_t cw = oc[x];
-          if (!cw) continue;
-          c += cw;
-          oc[x] = 0;
-#pragma unroll
-          for (int f = 0; f < NF; ++f)
-            if (f < p.nf) {
-              fv[f] = field_combine(p.field[f].kind, fv[f], of[f * TE * CW + x]);
-              of[f * TE * CW + x] = field_identity(p.field[f].kind);
-            }
-        }
-      }
-      if (c) flush_entry<NF>(p, st, table, pbase + e / C, (uint64_t)(e % C), c, fv, err);
-    }
-    __syncthreads();
-  };
+  auto flush_shared = [&]() { flush_tables<MODE, NF, FAST>(p, st, table, tabs, tf, tcnt, pbase, err); };
   auto flush_hashed = [&]() {      // warp-private table of one pane
     __syncwarp();
     for (int e = lane; e < TE; e += 32) {
@@ -467,6 +477,178 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   if (err) atomicOr(&st->error, err);
 }
 
+// ---------------------------------------------------------------------------
+// Count windows, fast path (no σ, fp64 sums of f32 columns, no key or one dense
+// int32 key): the same pass as k_pane_agg with all per-stage and per-tuple pane
+// arithmetic in 32 bits relative to the CTA's first pane P0 (division by g via
+// the invariant-divisor multiply, Plan::g_magic), stage bytes read through
+// 32-bit shared addresses, and no runtime key/predicate dispatch.  Count-window
+// panes are contiguous, so a stage's panes [pf, pl] are all non-empty.
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ int64_t lds_s64(uint32_t a) {
+  int64_t v;
+  asm volatile("ld.shared.s64 %0, [%1];" : "=l"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ int divg(const Plan &p, int x) {     // floor(x / g), 0 <= x < 2^30
+  return (int)(((uint64_t)(uint32_t)x * p.g_magic) >> p.g_mshift);
+}
+
+enum { KK_GLOBAL = 1, KK_RADIX = 2 };
+
+template <int MODE, int NF, int KK>
+__global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? 3 : 2)
+k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
+           uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int tb = p.tuple_bytes;
+  const int ST = kStageBytes / tb;
+  unsigned char *stages = smem;
+  uint64_t *full = (uint64_t *)(smem + kStages * kStageBytes);
+  uint64_t *empty = full + kStages;
+  unsigned char *tabs = (unsigned char *)(empty + kStages);
+  const int TE = p.local_entries;
+  const int CW = MODE == TM_LANE ? 32 : 1;
+  unsigned char *wt = tabs + (MODE == TM_SHARED ? 0 : (size_t)wid * p.local_bytes);
+  uint64_t *tf = (uint64_t *)wt;                                    // [NF][TE*CW]
+  uint32_t *tcnt = (uint32_t *)(wt + (size_t)8 * TE * CW * NF);     // [TE*CW]
+  for (int e = (MODE == TM_SHARED ? tid : lane); e < TE * CW; e += (MODE == TM_SHARED ? kP1Threads : 32)) {
+    tcnt[e] = 0;
+#pragma unroll
+    for (int f = 0; f < NF; ++f) tf[f * TE * CW + e] = 0;          // fp64 +0.0
+  }
+  const int64_t per = ((n + gridDim.x - 1) / gridDim.x + ST - 1) / ST * ST;
+  const int64_t lo = (int64_t)blockIdx.x * per;
+  const int64_t hi = lo + per < n ? lo + per : n;
+  const int nst = hi > lo ? (int)((hi - lo + ST - 1) / ST) : 0;
+  if (tid == 0) {
+    for (int i = 0; i < kStages; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], kP1Warps); }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  auto issue = [&](int k) {
+    const int slot = k % kStages;
+    const int64_t cnt = (hi - lo - (int64_t)k * ST) < ST ? (hi - lo - (int64_t)k * ST) : ST;
+    const uint32_t bytes = (uint32_t)(cnt * tb);
+    mbar_expect_tx(&full[slot], bytes);
+    bulk_g2s(stages + slot * kStageBytes, tup + (lo + (int64_t)k * ST) * tb, bytes, &full[slot]);
+  };
+  if (tid == 0)
+    for (int k = 0; k < kStages && k < nst; ++k) issue(k);
+
+  // CTA-relative pane coordinates: global pane = P0 + rel, rel of local tuple x = (R0 + x) / g
+  const int64_t gpos = st->task_pos + lo;
+  const int64_t P0 = gpos / p.g;
+  const int R0 = (int)(gpos - P0 * p.g);
+  const int64_t mp = st->J0 * p.L - P0;                      // panes < min_pane are dropped
+  const int minrel = mp <= 0 ? 0 : (mp > (1 << 30) ? (1 << 30) : (int)mp);
+  const int PL = p.local_pl;
+  const int C = (int)p.C;
+  const int g = (int)p.g;
+  const uint32_t tsoff = 4u * p.ts_word;
+  const uint32_t koff = KK == KK_RADIX ? 4u * p.key[0].word : 0u;
+  const uint32_t dom = KK == KK_RADIX ? (uint32_t)p.key[0].domain : 1u;
+  uint32_t foff[NF];
+#pragma unroll
+  for (int f = 0; f < NF; ++f) foff[f] = 4u * p.field[f].word;      // fast path: NF == p.nf
+  const int64_t Rm = p.R - 1;
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(stages);
+  int err = 0;
+  int prel = -1;                                             // CTA-uniform pane window [prel, prel+PL)
+  int64_t prev_last = (lo > 0 && lo < hi) ? *(const int64_t *)(tup + (lo - 1) * tb + tsoff) : INT64_MIN;
+  const int per_warp = (ST + kP1Warps - 1) / kP1Warps;
+  const int ib = wid * per_warp;
+  const int range32 = (int)(hi - lo);
+  int slot = 0;
+  uint32_t phase = 0;
+  for (int k = 0; k < nst; ++k) {
+    mbar_wait(&full[slot], phase);
+    const uint32_t sb = sbase + (uint32_t)(slot * kStageBytes);
+    const int xs = k * ST;                                   // local index of the stage's tuple 0
+    const int ntup = range32 - xs < ST ? range32 - xs : ST;
+    int pf = divg(p, R0 + xs);
+    const int pl = divg(p, R0 + xs + ntup - 1);
+    if (pf < minrel) pf = minrel;
+    const int ie = ib + per_warp < ntup ? ib + per_warp : ntup;
+    bool first_round = true;
+    for (int cur = pf; cur <= pl;) {
+      if (prel < 0 || cur < prel || cur >= prel + PL) {
+        if (prel >= 0) flush_tables<MODE, NF, true>(p, st, table, tabs, tf, tcnt, P0 + prel, err);
+        prel = cur;
+      }
+      const int wend = prel + PL;
+      const int wlo = prel > minrel ? prel : minrel;
+      const bool all_in = (pf >= wlo) & (pl < wend);
+      const int lo_ofs = wlo - prel;
+#pragma unroll 2
+      for (int i0 = ib; i0 < ie; i0 += 32) {
+        const int i = i0 + lane;
+        bool valid = i < ie;
+        const uint32_t t = sb + (uint32_t)((valid ? i : ib) * tb);
+        const int rel = R0 + xs + i;
+        const int q = divg(p, rel);
+        if (first_round) {
+          // K1: τ non-decreasing (L347-349) and non-negative (L349-350)
+          // (lane 0 reads its predecessor from the stage, or the previous stage's last)
+          const int64_t tau = lds_s64(t + tsoff);
+          int64_t up = (int64_t)shfl_up64((uint64_t)tau);
+          if (lane == 0) up = i > 0 ? lds_s64(t - tb + tsoff) : prev_last;
+          if (valid & (tau < up)) err |= ERR_ORDER;
+          if (valid & (tau < 0)) err |= ERR_TS;
+          if (valid && rel == q * g && q >= minrel) pane_ts[(P0 + q) & Rm] = tau;
+        }
+        const int po = q - prel;
+        if (!all_in) valid &= (po >= lo_ofs) & (po < PL);
+        uint32_t key = 0;
+        if (KK == KK_RADIX) {
+          key = lds_u32(t + koff);
+          if (key >= dom) {
+            if (valid) err |= ERR_KEY;
+            valid = false;
+          }
+        }
+        if (valid) {
+          double fv[NF];
+#pragma unroll
+          for (int f = 0; f < NF; ++f) fv[f] = (double)__uint_as_float(lds_u32(t + foff[f]));  // NF == nf
+          if (MODE == TM_LANE) {
+            const int e = (po * C + (int)key) * 32 + lane;
+            tcnt[e] += 1u;
+#pragma unroll
+            for (int f = 0; f < NF; ++f) {
+              double *a = (double *)&tf[f * TE * 32 + e];
+              *a = *a + fv[f];
+            }
+          } else {
+            const int e = po * C + (int)key;
+            atomicAdd(&tcnt[e], 1u);
+#pragma unroll
+            for (int f = 0; f < NF; ++f) atomicAdd((double *)&tf[f * TE + e], fv[f]);
+          }
+        }
+      }
+      first_round = false;
+      if (pl < wend) break;
+      cur = wend;                                            // count-window panes are contiguous
+    }
+    prev_last = lds_s64(sb + (uint32_t)((ntup - 1) * tb) + tsoff);
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[slot]);
+    if (tid == 0 && k + kStages < nst) {
+      mbar_wait(&empty[slot], phase);
+      issue(k + kStages);
+    }
+    if (++slot == kStages) { slot = 0; phase ^= 1u; }
+  }
+  if (prel >= 0) flush_tables<MODE, NF, true>(p, st, table, tabs, tf, tcnt, P0 + prel, err);
+  if (err) atomicOr(&st->error, err);
+}
+
 // ---------------------------------------------------------------- host side
 int p1_nf_template(int nf) { return nf <= 1 ? 1 : nf <= 2 ? 2 : nf <= 4 ? 4 : 8; }
 
@@ -494,8 +676,37 @@ static void *p1_mode(const Plan &p) {
     default: return p1_nf<TM_HASHED, WK>(p.nf, f);
   }
 }
-void *p1_kernel(const Plan &p) {
+static void *p1_generic(const Plan &p) {
   return p.win_kind == WK_COUNT ? p1_mode<WK_COUNT>(p) : p1_mode<WK_TIME>(p);
+}
+template <int M>
+static void *p1_cnt_nf(const Plan &p, int kk) {
+  if (kk == KK_GLOBAL) return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_GLOBAL> : (void *)k_pane_cnt<M, 2, KK_GLOBAL>;
+  return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_RADIX> : (void *)k_pane_cnt<M, 2, KK_RADIX>;
+}
+// count-window fast kernel, or nullptr when the plan needs the generic one
+static void *p1_cnt(const Plan &p) {
+  if (p.win_kind != WK_COUNT || !p.fast_path || p.npred != 0 || p.g_magic == 0) return nullptr;
+  int kk;
+  if (p.key_mode == KM_GLOBAL) kk = KK_GLOBAL;
+  else if (p.key_mode != KM_HASH && p.key_pack == KP_RADIX && p.nkeys == 1) kk = KK_RADIX;
+  else return nullptr;
+  switch (p.local_mode) {
+    case TM_LANE: return p1_cnt_nf<TM_LANE>(p, kk);
+    case TM_DIRECT: return p1_cnt_nf<TM_DIRECT>(p, kk);
+    case TM_SHARED: return p1_cnt_nf<TM_SHARED>(p, kk);
+    default: return nullptr;
+  }
+}
+void *p1_kernel(const Plan &p) {
+  void *k = p1_cnt(p);
+  return k ? k : p1_generic(p);
+}
+cudaError_t p1_set_attributes(const Plan &p) {
+  cudaError_t e = cudaFuncSetAttribute(p1_generic(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p1_smem_bytes(p));
+  if (e == cudaSuccess && p1_cnt(p))
+    e = cudaFuncSetAttribute(p1_cnt(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p1_smem_bytes(p));
+  return e;
 }
 
 int p1_blocks_per_sm(const Plan &p) {
@@ -511,7 +722,10 @@ cudaError_t launch_pane_agg(const Plan &p, const QueryDev &q, const void *tuples
   int64_t need = (n + stage_t - 1) / stage_t;     // at least one stage per CTA
   int g = (int)(need < grid ? need : grid);
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&tuples, (void *)&n, (void *)&q.table, (void *)&q.pane_ts};
-  return cudaLaunchKernel(p1_kernel(p), dim3(g), dim3(kP1Threads), args, (size_t)p1_smem_bytes(p), st);
+  // the fast count kernel keeps CTA-relative positions and panes in 32 bits
+  void *k = p1_cnt(p);
+  if (!k || (n / g + stage_t + p.g) >= (1ll << 30)) k = p1_generic(p);
+  return cudaLaunchKernel(k, dim3(g), dim3(kP1Threads), args, (size_t)p1_smem_bytes(p), st);
 }
 
 }  // namespace sb

@@ -415,12 +415,13 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
 }
 
 // ---------------------------------------------------------------------------
-// Few keys (C <= 32, one slab): a warp holds 32/Cp windows side by side, lane =
-// (window, key slot), Cp = C rounded up to a power of two, so no lane idles on a
-// 4-key GROUP BY or a GLOBAL aggregate.  Row order is window-major, key order
-// inside a window, exactly as k_win_fused.  One ballot per (pass, warp) gives
-// every window's row count and every row's offset.
-constexpr int kPackU = 4;     // window passes per warp per chunk
+// Few keys (C <= 256, one slab): Cp = C rounded up to a power of two.  Cp <= 32:
+// a warp pass holds 32/Cp windows side by side, lane = (window, key slot), so no
+// lane idles on a 4-key GROUP BY or a GLOBAL aggregate; Cp > 32: a window takes
+// NB = Cp/32 consecutive passes of 32 slots.  Row order is window-major, key
+// order inside a window, exactly as k_win_fused.  One ballot per (pass, warp)
+// gives every window's row count and every row's offset.
+constexpr int kPackU = 8;     // ballot passes per warp per chunk
 
 template <bool F>
 __device__ __forceinline__ bool win_value(const Plan &p, const uint64_t *__restrict__ pre,
@@ -450,27 +451,32 @@ k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ 
   __shared__ int64_t s_base;
   __shared__ int s_t;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int WPW = 32 >> cshift;                       // windows per warp pass
-  const int wsub = lane >> cshift, slot = lane & ((1 << cshift) - 1);
-  const unsigned seg_lt = (1u << (wsub << cshift)) - 1u;            // lanes of earlier windows
-  const unsigned seg = cshift == 5 ? kFull : (((1u << (1 << cshift)) - 1u) << (wsub << cshift));
+  const int cs = cshift < 5 ? cshift : 5, nbs = cshift - cs;     // NB = 1 << nbs passes per window
+  const int WPW = 32 >> cs;                                       // windows per warp pass
+  const int wsub = lane >> cs, sl = lane & ((1 << cs) - 1);
+  const unsigned seg_lt = (1u << (wsub << cs)) - 1u;              // lanes of earlier windows
+  const unsigned seg = cs == 5 ? kFull : (((1u << (1 << cs)) - 1u) << (wsub << cs));
   const unsigned lt = (1u << lane) - 1u;
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
   if (nw <= 0) return;
   const uint64_t epoch = (uint64_t)st->tile_epoch;
-  const int WC = 8 * kPackU * WPW;
+  const int WW = (kPackU >> nbs) * WPW;                           // windows per warp per chunk
+  const int WC = 8 * WW;
   const int64_t nchunks = (nw + WC - 1) / WC;
+  auto win_of = [&](int u) { return (int64_t)((u >> nbs) * WPW + wsub); };
+  auto slot_of = [&](int u) { return ((u & ((1 << nbs) - 1)) << 5) + sl; };
   for (;;) {
     if (threadIdx.x == 0) s_t = atomicAdd(ticket, 1);
     __syncthreads();
     const int64_t t = s_t;
     if (t >= nchunks) break;
-    const int64_t wb = J0 + t * WC + (int64_t)warp * kPackU * WPW + wsub;
+    const int64_t wb = J0 + t * WC + (int64_t)warp * WW;
     unsigned bal[kPackU];
     int wtot = 0;
 #pragma unroll
     for (int u = 0; u < kPackU; ++u) {
-      const int64_t j = wb + u * WPW;
+      const int64_t j = wb + win_of(u);
+      const int slot = slot_of(u);
       bool present = false;
       if (j < J1 && slot < p.C) {
         int64_t c;
@@ -509,16 +515,22 @@ k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ 
     }
     __syncthreads();
     int64_t r = s_base + s_wcnt[warp];
+    int64_t w_off = 0;
+    int w_rows = 0;
 #pragma unroll
     for (int u = 0; u < kPackU; ++u) {
-      const int64_t j = wb + u * WPW;
+      const int64_t j = wb + win_of(u);
+      const int slot = slot_of(u);
+      const int part = u & ((1 << nbs) - 1);
+      if (part == 0) { w_off = r + __popc(bal[u] & seg_lt); w_rows = 0; }
+      w_rows += __popc(bal[u] & seg);
       if (j < J1) {
-        if (slot == 0) {
+        if (sl == 0 && part == (1 << nbs) - 1) {
           WinHdr h;
           h.window_id = j;
           h.ts = (p.win_kind == WK_TIME) ? p.T0 + j * p.l : pane_ts[(j * p.L) & (p.R - 1)];
-          h.row_offset = r + __popc(bal[u] & seg_lt);
-          h.nrows = __popc(bal[u] & seg);
+          h.row_offset = w_off;
+          h.nrows = w_rows;
           h.flags = 0;
           hdr[j - J0] = h;
         }
@@ -748,7 +760,7 @@ cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev
   if (p.K > 64 && p.slot_words < 64) k_vh_build_long<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   else if (p.K > 64) k_vh_build_warp<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   else k_vh_build<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
-  if (p.S == 1 && p.C <= 32) {
+  if (p.S == 1 && p.C <= 256) {
     int cshift = 0;
     while ((1 << cshift) < p.C) ++cshift;
     k_win_packed<<<grid, 256, 0, st>>>(p, q.st, q.vh_pre, q.vh_suf, q.pane_ts, (WinHdr *)s.hdr, s.rows,

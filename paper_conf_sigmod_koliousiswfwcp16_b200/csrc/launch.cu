@@ -10,7 +10,7 @@ cudaError_t set_kernel_attributes(const Plan &p) {
   cudaError_t e = cudaSuccess;
   if (p.nagg == 0) return cudaFuncSetAttribute(sel_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem_bytes());
   if (p.nagg > 0) {
-    e = cudaFuncSetAttribute(p1_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p1_smem_bytes(p));
+    e = p1_set_attributes(p);
     if (e) return e;
     if (p.p2_smem > 0) e = cudaFuncSetAttribute(p2_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
     if (e) return e;

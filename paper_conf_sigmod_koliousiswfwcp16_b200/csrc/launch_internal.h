@@ -16,6 +16,7 @@ cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, 
 cudaError_t launch_carry(const Plan &p, const QueryDev &q, const void *tuples, cudaStream_t st);
 // k_pane.cu
 void *p1_kernel(const Plan &p);
+cudaError_t p1_set_attributes(const Plan &p);
 cudaError_t launch_pane_agg(const Plan &p, const QueryDev &q, const void *tuples, int64_t n, int grid,
                             cudaStream_t st);
 // k_window.cu

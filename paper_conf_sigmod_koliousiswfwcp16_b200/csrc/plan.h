@@ -47,7 +47,8 @@ struct Plan {
   int32_t win_kind, pad0;
   int64_t s, l, T0, g, K, L;
   double g_inv;                   // 1/g for the reciprocal division in K1
-  int32_t g_shift, pad7;          // log2(g) if g is a power of two, else -1
+  int32_t g_shift, g_mshift;      // log2(g) if g is a power of two, else -1; magic shift
+  uint64_t g_magic;               // floor(x/g) = (x·g_magic) >> g_mshift for 0 <= x < 2^30, g < 2^28
   // σ
   int32_t npred, pad1;
   Pred pred[kMaxPred];

@@ -170,6 +170,16 @@ static saber_status build_plan(saber_query *q, const saber_schema *sc, const sab
   if ((p.g & (p.g - 1)) == 0)
     for (int b = 0; b < 63; ++b)
       if ((1ll << b) == p.g) p.g_shift = b;
+  // division by the invariant g (Granlund-Montgomery): l = ceil(log2 g),
+  // m = floor(2^(32+l)/g) + 1 gives floor(x/g) = floor(x·m / 2^(32+l)) for x < 2^32
+  p.g_magic = 0;
+  p.g_mshift = 0;
+  if (p.g < (1ll << 28)) {
+    int lg = 0;
+    while ((1ll << lg) < p.g) ++lg;
+    p.g_mshift = 32 + lg;
+    p.g_magic = (uint64_t)((((unsigned __int128)1) << p.g_mshift) / (unsigned __int128)p.g) + 1;
+  }
 
   p.npred = op->npred;
   for (int i = 0; i < op->npred; ++i) {
