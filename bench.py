@@ -91,48 +91,63 @@ def workload(args):
 
 # --------------------------------------------------------------------------- utils
 class Clocks:
-    """nvidia-smi sampling during the timed region (the recipe's clocks line)."""
+    """SM clocks and clock-event reasons sampled DURING the timed region (the
+    recipe's clocks line).  NVML is polled every ~2 ms from a thread (the timed
+    region of a step is milliseconds, too short for `nvidia-smi -lms`); samples
+    are tagged with whether a timed step was in flight (``clk.timed = True``).
+    Every sample is also written to ``path`` as CSV."""
+
+    REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "hw_power_brake_slowdown": 0x80, "sw_power_cap": 0x4}
 
     def __init__(self, index, path):
-        self.path = path
-        self.proc = None
-        self.index = index
+        self.index, self.path = index, path
+        self.rows, self.timed, self._stop = [], False, False
+        self.thread = None
+
+    def _run(self):
+        import pynvml
+        pynvml.nvmlInit()
+        h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+        mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+        while not self._stop:
+            sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+            rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+            self.rows.append((time.perf_counter(), self.timed, sm, mx, int(rs)))
+            time.sleep(0.002)
+        pynvml.nvmlShutdown()
 
     def __enter__(self):
         try:
-            self.f = open(self.path, "w")
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", str(self.index), "--query-gpu=index,clocks.sm,clocks.max.sm,power.draw,"
-                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
-                stdout=self.f, stderr=subprocess.DEVNULL)
+            import pynvml  # noqa: F401
+            self.thread = threading.Thread(target=self._run, daemon=True)
+            self.thread.start()
         except Exception:
-            self.proc = None
+            self.thread = None
         return self
 
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except Exception:
-                self.proc.kill()
-            self.f.close()
+        self._stop = True
+        if self.thread:
+            self.thread.join(timeout=5)
+        try:
+            with open(self.path, "w") as f:
+                f.write("t,timed,sm_mhz,sm_max_mhz,reasons\n")
+                for r in self.rows:
+                    f.write(f"{r[0]:.6f},{int(r[1])},{r[2]},{r[3]},{r[4]:#x}\n")
+        except Exception:
+            pass
 
     def summary(self):
-        try:
-            rows = [r.split(", ") for r in open(self.path).read().strip().splitlines() if r.strip()]
-        except Exception:
-            rows = []
+        rows = [r for r in self.rows if r[1]]
+        where = "timed region"
+        if not rows:
+            rows, where = self.rows, "whole run (no sample fell inside a timed step)"
         if not rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
-        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in rows for i in range(4) if len(r) > 5 + i and r[5 + i].strip() == "Active"})
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(rows)}
+        reasons = sorted({n for r in rows for n, bit in self.REASONS.items() if r[4] & bit})
+        return {"sm_mhz": statistics.median(r[2] for r in rows), "sm_max_mhz": max(r[3] for r in rows),
+                "reasons": reasons, "samples": len(rows), "sampled": where, "source": "NVML, ~2 ms poll"}
 
 
 def measured_peaks():
@@ -312,6 +327,7 @@ def main():
             torch.cuda.synchronize()
             ev0 = torch.cuda.Event(enable_timing=True)
             ev1 = torch.cuda.Event(enable_timing=True)
+            clk.timed = it >= args.warmup
             ev0.record(stream)
             pieces = []
             if world > 1:
@@ -325,6 +341,7 @@ def main():
             while q.stats()["tasks_pending"] > 0:     # already complete once ev1 is
                 drain_one()
             torch.cuda.synchronize()
+            clk.timed = False
             ms = ev0.elapsed_time(ev1)
             st = q.stats()
             if it >= args.warmup:
