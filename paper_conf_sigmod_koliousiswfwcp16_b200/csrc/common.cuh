@@ -82,6 +82,24 @@ __device__ __forceinline__ uint64_t field_value(const Field &f, const uint32_t (
   }
 }
 
+// field access straight from the shared-memory tuple (runtime byte offsets)
+__device__ __forceinline__ int64_t s_int(const unsigned char *t, int word, int type) {
+  return type == T_I32 ? (int64_t) * (const int32_t *)(t + 4 * word) : *(const int64_t *)(t + 4 * word);
+}
+__device__ __forceinline__ double s_flt(const unsigned char *t, int word, int type) {
+  return type == T_F32 ? (double)*(const float *)(t + 4 * word) : *(const double *)(t + 4 * word);
+}
+
+__device__ __forceinline__ bool s_preds(const Plan &p, const unsigned char *t) {
+  bool ok = true;
+  for (int i = 0; i < p.npred; ++i) {
+    const Pred &pr = p.pred[i];
+    if (pr.type == T_F32 || pr.type == T_F64) ok &= cmp_op(s_flt(t, pr.word, pr.type), pr.op, pr.fval);
+    else ok &= cmp_op(s_int(t, pr.word, pr.type), pr.op, pr.ival);
+  }
+  return ok;
+}
+
 __device__ __forceinline__ int64_t cnt_off(const Plan &p) { return p.key_mode == KM_HASH ? p.C : 0; }
 __device__ __forceinline__ int64_t fld_off(const Plan &p, int f) { return cnt_off(p) + (int64_t)(1 + f) * p.C; }
 

@@ -125,7 +125,8 @@ __global__ void k_zero_panes(const Plan p, const State *st, uint64_t *table) {
     int64_t pane = lo + i / p.slot_words;
     int64_t w = i % p.slot_words;
     uint64_t v;
-    if (w < co) v = kEmpty;                               // hash keys
+    if (p.bucket_mode) v = 0;                             // bucket fill counters
+    else if (w < co) v = kEmpty;                               // hash keys
     else if (w < co + p.C) v = 0;                         // counts
     else v = field_identity(p.field[(w - co - p.C) / p.C].kind);
     table[(pane & (p.R - 1)) * p.slot_words + w] = v;

@@ -29,6 +29,7 @@ struct QueryDev {
   unsigned char *carry[2];  // IStream raw tail
   int64_t carry_cap;        // tuples
   int *tile_ctr;
+  unsigned char *bkt;       // bucket mode: [R][S][g] u16 key offsets, then [R][S][nf][g] f32 values
 };
 
 // one task of an aggregation (RStream) query
@@ -49,6 +50,7 @@ int p1_smem_bytes(const Plan &p);
 int p1_blocks_per_sm(const Plan &p);
 int p2_blocks_per_sm(const Plan &p);
 int sel_blocks_per_sm(const Plan &p);
+int bk_scan_blocks_per_sm(const Plan &p);
 cudaError_t set_kernel_attributes(const Plan &p);
 
 }  // namespace sb

@@ -9,6 +9,7 @@ namespace sb {
 cudaError_t set_kernel_attributes(const Plan &p) {
   cudaError_t e = cudaSuccess;
   if (p.nagg == 0) return cudaFuncSetAttribute(sel_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem_bytes());
+  if (p.bucket_mode) return bk_set_attributes(p);
   if (p.nagg > 0) {
     e = p1_set_attributes(p);
     if (e) return e;
@@ -29,6 +30,7 @@ cudaError_t set_kernel_attributes(const Plan &p) {
 
 int p2_blocks_per_sm(const Plan &p) {
   int b = 0;
+  if (p.bucket_mode) return 1;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, p.slab_mode ? slab_kernel(true) : p2_kernel(p), 256, p.p2_smem);
   return b > 0 ? b : 1;
 }
@@ -47,11 +49,16 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
   *launches = 2;
   if (evs) cudaEventRecord(evs[0], st);
   if (n > 0) {
-    if ((e = launch_pane_agg(p, q, tuples, n, p1_grid, st))) return e;
+    if (p.bucket_mode) e = launch_bucket_scan(p, q, tuples, n, p1_grid, st);
+    else e = launch_pane_agg(p, q, tuples, n, p1_grid, st);
+    if (e) return e;
     *launches += 1;
   }
   if (evs) cudaEventRecord(evs[1], st);
-  if (p.slab_mode) {
+  if (p.bucket_mode) {
+    if ((e = launch_bucket_windows(p, q, s, p2_grid, st))) return e;
+    *launches += 3;
+  } else if (p.slab_mode) {
     if ((e = launch_windows_slab(p, q, s, false, p2_grid, win_chunk, st))) return e;
     if ((e = launch_win_scan(p, q, s, st))) return e;
     if ((e = launch_windows_slab(p, q, s, true, p2_grid, win_chunk, st))) return e;
@@ -64,7 +71,7 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
     if ((e = launch_windows_fused(p, q, s, p2_grid, st))) return e;
   }
   if ((e = launch_task_end(p, q, s, st))) return e;
-  *launches += p.key_mode == KM_HASH ? 4 : 3;
+  *launches += p.bucket_mode ? 1 : p.key_mode == KM_HASH ? 4 : 3;
   if (evs) cudaEventRecord(evs[2], st);
   return cudaGetLastError();
 }

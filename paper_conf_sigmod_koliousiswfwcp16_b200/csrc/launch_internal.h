@@ -28,6 +28,12 @@ cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev
 cudaError_t launch_windows_slab(const Plan &p, const QueryDev &q, const SlotDev &s, bool emit, int grid, int W,
                                 cudaStream_t st);
 void *slab_kernel(bool emit);
+// k_bucket.cu
+cudaError_t bk_set_attributes(const Plan &p);
+int bk_scan_blocks_per_sm(const Plan &p);
+cudaError_t launch_bucket_scan(const Plan &p, const QueryDev &q, const void *tuples, int64_t n, int grid,
+                               cudaStream_t st);
+cudaError_t launch_bucket_windows(const Plan &p, const QueryDev &q, const SlotDev &s, int nsm, cudaStream_t st);
 // k_select.cu
 void *sel_kernel(const Plan &p);
 int sel_smem_bytes();

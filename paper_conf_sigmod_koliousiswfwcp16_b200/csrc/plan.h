@@ -91,6 +91,13 @@ struct Plan {
   int64_t win_cap;                // windows per result slot
   int64_t first_window;           // windows < first_window are not emitted
   int64_t carry_cap;              // IStream: raw tail tuples kept between tasks
+  // bucket mode (count windows, one radix key with a large declared domain, fp64
+  // sums of f32 columns, no HAVING): the scan writes every tuple's (key offset,
+  // values) into a per-(pane, key slab) bucket; window assembly slides a dense
+  // per-slab state over the buckets (k_bucket.cu)
+  int32_t bucket_mode, bk_shift;  // SB = 1 << bk_shift keys per slab (S = p.S slabs)
+  int32_t bk_W, bk_threads;       // windows per assembly chunk, threads per assembly CTA
+  int64_t bk_vals;                // byte offset of the value section in the bucket store
 };
 
 // Per-query device state, updated only by kernels on the query's stream.

@@ -13,6 +13,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -51,6 +52,11 @@ struct Stage {
   bool used = false;
 };
 
+constexpr int64_t kDenseMaxPlan = 8192;   // declared key domains up to this use dense pane tables
+bool getenv_flag(const char *name) {
+  const char *v = std::getenv(name);
+  return v && *v && *v != '0';
+}
 int64_t gcd64(int64_t a, int64_t b) { while (b) { int64_t t = a % b; a = b; b = t; } return a; }
 int64_t next_pow2(int64_t x) { int64_t p = 1; while (p < x) p <<= 1; return p; }
 int64_t floor_pow2(int64_t x) { int64_t p = 1; while (p * 2 <= x) p <<= 1; return p; }
@@ -66,6 +72,7 @@ struct saber_query {
   saber_window win{};
   saber_config cfg{};
   int device = 0, nsm = 148;
+  int nsm_hint = 148;           // SM count known at planning time
   cudaStream_t cs = nullptr, h2d = nullptr, d2h = nullptr;
   QueryDev qd{};
   std::vector<Slot> slots;
@@ -248,7 +255,7 @@ static saber_status build_plan(saber_query *q, const saber_schema *sc, const sab
     prod *= (long double)(k.domain > 0 ? k.domain : 1);
     use(k.col);
   }
-  const int64_t kDenseMax = 8192;
+  const int64_t kDenseMax = kDenseMaxPlan;
   if (op->nkeys == 0) {
     p.key_mode = KM_GLOBAL; p.key_pack = KP_RADIX; p.G = 1;
   } else if (all_dom && prod < 4.0e18L) {
@@ -398,6 +405,34 @@ static saber_status size_plan(saber_query *q) {
         }
       }
     }
+    // bucket mode: count windows, one int32 key with a large declared domain,
+    // fp64 sums of f32 columns, no HAVING (k_bucket.cu).  SB keys per slab so
+    // that the slab state (u32 count + nf fp64 sums per key) fits one CTA.
+    if (p.win_kind == WK_COUNT && p.key_mode == KM_HASH && p.key_pack == KP_RADIX && p.nkeys == 1 &&
+        p.fast_path && p.nhave == 0 && p.nagg <= 4 && p.G > kDenseMaxPlan && p.G <= (1ll << 18) && p.g_magic != 0 &&
+        p.g <= 65536 && !getenv_flag("SABER_NO_BUCKET")) {
+      int64_t sb = std::min<int64_t>(16384, floor_pow2((224 * 1024) / (6 + 8 * p.nf)));
+      sb = std::min<int64_t>(sb, next_pow2(p.G));
+      const int64_t S = (p.G + sb - 1) / sb;
+      const int64_t st_max = 16384 / p.tuple_bytes;           // tuples per scan stage
+      if (S <= 16 && (st_max / p.g + 2) * S <= 1024) {
+        p.bucket_mode = 1;
+        p.slab_mode = 0;
+        p.SB = (int)sb;
+        p.S = (int)S;
+        p.bk_shift = 0;
+        while ((1ll << p.bk_shift) < sb) ++p.bk_shift;
+        p.C = S;
+        p.slot_words = S;                                      // per-(pane, slab) fill counters
+        p.bk_threads = 512;
+        // windows per assembly chunk: about one chunk per SM and slab per task
+        const int64_t nwt = std::max<int64_t>(1, T / p.l);
+        const int64_t per_slab = std::max<int64_t>(1, q->nsm_hint / S);
+        p.bk_W = (int)std::max<int64_t>(16, std::min<int64_t>(1024, (nwt + per_slab - 1) / per_slab));
+        p.bk_vals = ((p.R * S * p.g * 2) + 255) & ~255ll;
+        p.p2_smem = 0;
+      }
+    }
     // output columns (keys then aggregates)
     p.ncols = p.nkeys + p.nagg;
     p.row_bytes = 0;
@@ -405,6 +440,7 @@ static saber_status size_plan(saber_query *q) {
     for (int a = 0; a < p.nagg; ++a) { p.col_bytes[p.nkeys + a] = 8; p.row_bytes += 8; }
     p.win_cap = p.win_kind == WK_COUNT ? T / p.l + 4 : p.R / p.L + 4;
     int64_t rows_per_win = p.key_mode == KM_GLOBAL ? 1 : p.key_mode == KM_DENSE ? p.G
+                           : p.bucket_mode ? std::min<int64_t>(p.s, p.G)
                            : (p.win_kind == WK_COUNT ? std::min<int64_t>(p.s, p.C * p.K) : p.C * p.K);
     int64_t rb = c.result_bytes;
     if (rb <= 0) {
@@ -451,6 +487,9 @@ static saber_status alloc_query(saber_query *q) {
       CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
       CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
     }
+    if (p.bucket_mode) {
+      CK(cudaMalloc(&q->qd.bkt, (size_t)p.bk_vals + (size_t)p.R * p.S * p.nf * p.g * 4 + 256));
+    }
     if (p.slab_mode) {
       CK(cudaMalloc(&q->qd.clist, (size_t)p.R * p.C * (1 + p.nf) * 8));
       CK(cudaMalloc(&q->qd.coff, (size_t)p.R * (p.S + 1) * 4));
@@ -492,7 +531,10 @@ static saber_status alloc_query(saber_query *q) {
     CK(set_kernel_attributes(pl));
     q->p1_grid_lane = p1_blocks_per_sm(pl) * q->nsm;
   }
-  if (p.nagg > 0) {
+  if (p.bucket_mode) {
+    q->p1_grid = bk_scan_blocks_per_sm(p) * q->nsm;
+    q->p2_grid = q->nsm;
+  } else if (p.nagg > 0) {
     q->p1_grid = p1_blocks_per_sm(p) * q->nsm;
     q->p2_grid = p2_blocks_per_sm(p) * q->nsm * 2;
   } else {
@@ -592,6 +634,8 @@ saber_status saber_query_create(const saber_schema *schema, const saber_operator
   else cudaGetDevice(&q->device);
   if (q->device >= ndev) { delete q; return fail(nullptr, SABER_EINVAL, "device ordinal"); }
   q->win = *window;
+  cudaDeviceGetAttribute(&q->nsm_hint, cudaDevAttrMultiProcessorCount, q->device);
+  if (q->nsm_hint <= 0) q->nsm_hint = 148;
   saber_status st = build_plan(q, schema, op, window);
   if (st == SABER_OK) st = size_plan(q);
   if (st == SABER_OK) st = alloc_query(q);
@@ -622,7 +666,7 @@ void saber_query_destroy(saber_query *q) {
   for (auto &r : q->registered)
     if (std::find(q->prereg.begin(), q->prereg.end(), r.first) == q->prereg.end()) cudaHostUnregister(r.first);
   cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.vh_pre); cudaFree(q->qd.vh_suf);
-  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.sel_stage); cudaFree(q->qd.cta_cnt); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
+  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.bkt); cudaFree(q->qd.sel_stage); cudaFree(q->qd.cta_cnt); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
   cudaFree(q->qd.carry[0]); cudaFree(q->qd.carry[1]); cudaFree(q->qd.tile_ctr); cudaFree(q->d_tmp);
   if (q->cs) cudaStreamDestroy(q->cs);
   if (q->h2d) cudaStreamDestroy(q->h2d);

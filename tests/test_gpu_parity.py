@@ -110,6 +110,41 @@ def test_c3_groupby(saber, oracle_lib, groups, dom):
     check(saber, oracle_lib, spec, data, task_bytes=(4 << 20))
 
 
+# bucket mode (k_bucket.cu): count windows, one int32 key with a large declared
+# domain; ragged task sizes, several key slabs, σ, 0/1/2 accumulator fields
+@pytest.mark.parametrize("case", ["g64k_ragged", "g20000_sigma", "g100000_tumbling", "cm_two_fields", "count_only"])
+def test_bucket_mode(saber, oracle_lib, case):
+    if case == "g64k_ragged":
+        spec, g = workloads.c3(groups=65536)
+        data = gen.generate("syn", 1 << 19, g["seed"], rate=1, groups=65536)
+        tb = (4 << 20) + 32 * 77
+    elif case == "g20000_sigma":
+        spec, _ = workloads.c3(groups=20000)
+        spec["window"] = workloads.count_window(4096, 512)
+        spec["aggs"] = [("count", None), ("sum", "a1"), ("avg", "a1")]
+        spec["where"] = [("a3", "<", int(0.7 * 2 ** 31))]
+        data = gen.generate("syn", 200000, 11, rate=1, groups=20000)
+        tb = (1 << 20) + 32 * 5
+    elif case == "g100000_tumbling":
+        spec, _ = workloads.c3(groups=100000)
+        spec["window"] = workloads.count_window(2048, 2048)
+        data = gen.generate("syn", 300000, 12, rate=1, groups=100000)
+        tb = 777 * 32
+    elif case == "cm_two_fields":
+        spec, _ = workloads.c4(gcat=32768)
+        spec["window"] = workloads.count_window(3000, 1000)
+        spec["aggs"] = [("sum", "cpu"), ("avg", "ram"), ("count", None)]
+        data = gen.generate("cm", 150000, 13, rate=64, groups=32768)
+        tb = (2 << 20) + 64 * 3
+    else:
+        spec, _ = workloads.c3(groups=50000)
+        spec["window"] = workloads.count_window(1500, 300)
+        spec["aggs"] = [("count", None)]
+        data = gen.generate("syn", 100000, 14, rate=1, groups=50000)
+        tb = 1 << 20
+    check(saber, oracle_lib, spec, data, task_bytes=tb)
+
+
 @pytest.mark.parametrize("rate", [64, 4096])
 def test_c4_cm1(saber, oracle_lib, rate):
     spec, g = workloads.c4(rate=rate)
