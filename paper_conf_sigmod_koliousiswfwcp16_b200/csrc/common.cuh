@@ -153,6 +153,19 @@ __device__ __forceinline__ int64_t global_insert(const Plan &p, State *st, uint6
 }
 
 
+// decoupled look-back status words: epoch (24 bits) | flag (2: 1 aggregate, 2 inclusive) | value (38 bits)
+__device__ __forceinline__ uint64_t lb_ld(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void lb_st(uint64_t *p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v));
+}
+__device__ __forceinline__ uint64_t lb_pack(uint64_t epoch, uint64_t flag, uint64_t v) {
+  return ((epoch & 0xffffffull) << 40) | (flag << 38) | (v & ((1ull << 38) - 1));
+}
+
 // --------------------------------------------------------------------------
 // window assembly helpers
 struct AggVal { uint64_t bits; bool isf; };

@@ -188,16 +188,17 @@ k_pane_bucket(const Plan p, State *__restrict__ st, const unsigned char *__restr
 // (and, in k_bkt_emit, while window j is written), so the global-load latency
 // of a step is hidden behind the previous one; kPF entries per thread and
 // direction are prefetched, anything beyond is loaded in place.
-constexpr int kPF = 2;
+constexpr int kPF = 4;                // k_bkt_count: 256 threads
+constexpr int kEmitPF = 2;           // k_bkt_emit: 512 threads, two entries per thread and direction
 
 template <int NF>
 struct BkVals { float v[NF > 0 ? NF : 1]; };
-template <int NF>
+template <int NF, int PF = kPF>
 struct BkStep {
   int nl, ne;                          // entries leaving / entering (this slab)
   int64_t bl, be;                      // bucket index of the leaving / entering pane
-  uint32_t kl[kPF], ke[kPF];           // prefetched keys
-  BkVals<NF> vl[kPF], ve[kPF];
+  uint32_t kl[PF], ke[PF];             // prefetched keys
+  BkVals<NF> vl[PF], ve[PF];
 };
 
 // bucket fill counts of step j (leave pane j, enter pane j+K; L = 1)
@@ -207,10 +208,10 @@ __device__ __forceinline__ void bk_counts(const Plan &p, const unsigned long lon
   nl = (int)__ldg(bcnt + (j & Rm) * p.S + s);
   ne = (int)__ldg(bcnt + ((j + p.K) & Rm) * p.S + s);
 }
-template <int NF, bool VALS>
+template <int NF, bool VALS, int PF>
 __device__ __forceinline__ void bk_prefetch(const Plan &p, const uint16_t *__restrict__ keys,
                                             const float *__restrict__ vals, int64_t j, int s, int nl, int ne,
-                                            BkStep<NF> &x) {
+                                            BkStep<NF, PF> &x) {
   const int64_t Rm = p.R - 1;
   const int S = p.S, g = (int)p.g, tid = threadIdx.x, nt = blockDim.x;
   x.bl = (j & Rm) * S + s;
@@ -218,7 +219,7 @@ __device__ __forceinline__ void bk_prefetch(const Plan &p, const uint16_t *__res
   x.nl = nl;
   x.ne = ne;
 #pragma unroll
-  for (int u = 0; u < kPF; ++u) {
+  for (int u = 0; u < PF; ++u) {
     const int e = tid + u * nt;
     if (e < x.nl) {
       x.kl[u] = __ldg(keys + x.bl * g + e);
@@ -235,14 +236,15 @@ __device__ __forceinline__ void bk_prefetch(const Plan &p, const uint16_t *__res
   }
 }
 
-// window assembly, pass 1: rows per (window, slab) = keys with a non-zero count
-__global__ void __launch_bounds__(512)
+// window assembly, pass 1: rows per (window, slab) = keys with a non-zero count;
+// chunks of about a third of the emission chunk (3 CTAs per SM)
+__global__ void __launch_bounds__(256, 3)
 k_bkt_count(const Plan p, const State *__restrict__ st, const unsigned long long *__restrict__ bcnt,
             const unsigned char *__restrict__ bkt, int64_t *__restrict__ counts) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int dn[3];
   uint32_t *cnt = (uint32_t *)smem;
-  const int S = p.S, SB = 1 << p.bk_shift, W = p.bk_W, g = (int)p.g;
+  const int S = p.S, SB = 1 << p.bk_shift, W = p.bk_W > 48 ? (p.bk_W + 2) / 3 : 16, g = (int)p.g;
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
   if (nw <= 0) return;
   const int64_t nitems = ((nw + W - 1) / W) * S;
@@ -418,7 +420,7 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
     };
     auto pane_b = [&](int64_t q) { return (q & Rm) * S + s; };
     for (int64_t q = ja * p.L; q < ja * p.L + p.K; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), true);
-    BkStep<NF> A, B;
+    BkStep<NF, kEmitPF> A, B;
     int cnl = 0, cne = 0;                 // bucket counts of the step after the prefetched one
     if (pipe && ja + 1 < jb) {
       int nl, ne;
@@ -498,13 +500,13 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
       // ---- slide to window j+1
       if (pipe) {
 #pragma unroll
-        for (int u = 0; u < kPF; ++u) {
+        for (int u = 0; u < kEmitPF; ++u) {
           const int e = tid + u * nt;
           if (e < A.nl) upd(A.kl[u], false, A.vl[u]);
           if (e < A.ne) upd(A.ke[u], true, A.ve[u]);
         }
-        visit(A.bl, kPF * nt, A.nl, false);
-        visit(A.be, kPF * nt, A.ne, true);
+        visit(A.bl, kEmitPF * nt, A.nl, false);
+        visit(A.be, kEmitPF * nt, A.ne, true);
       } else {
         for (int64_t q = j * p.L; q < (j + 1) * p.L; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), false);
         for (int64_t q = j * p.L + p.K; q < (j + 1) * p.L + p.K; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), true);
@@ -514,13 +516,13 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
       // with count > 0 only, so no barrier separates them
       if (pipe) {
 #pragma unroll
-        for (int u = 0; u < kPF; ++u) {
+        for (int u = 0; u < kEmitPF; ++u) {
           const int e = tid + u * nt;
           if (e < A.nl && cnt[A.kl[u]] == 0u)
 #pragma unroll
             for (int f = 0; f < NF; ++f) sum[f * SB + A.kl[u]] = 0.0;
         }
-        zero_fix(A.bl, kPF * nt, A.nl);
+        zero_fix(A.bl, kEmitPF * nt, A.nl);
         A = B;
       } else {
         for (int64_t q = j * p.L; q < (j + 1) * p.L; ++q) zero_fix(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)));
@@ -574,7 +576,7 @@ cudaError_t launch_bucket_scan(const Plan &p, const QueryDev &q, const void *tup
 
 cudaError_t launch_bucket_windows(const Plan &p, const QueryDev &q, const SlotDev &s, int nsm, cudaStream_t st) {
   const unsigned long long *bc = (const unsigned long long *)q.table;
-  k_bkt_count<<<nsm * 2, 512, bk_count_smem(p), st>>>(p, q.st, bc, q.bkt, s.counts);
+  k_bkt_count<<<nsm * 3, 256, bk_count_smem(p), st>>>(p, q.st, bc, q.bkt, s.counts);
   cudaError_t e = launch_win_scan(p, q, s, st);
   if (e) return e;
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&bc, (void *)&q.bkt, (void *)&s.counts, (void *)&s.rows};

@@ -133,65 +133,106 @@ __global__ void k_zero_panes(const Plan p, const State *st, uint64_t *table) {
   }
 }
 
-__global__ void __launch_bounds__(1024)
+// Window headers and row offsets of a task from its per-(window, slab) row
+// counts (HASH / slab / bucket modes): tiles of kScanTW windows take tickets,
+// scan their counts in the CTA, get the tile's base by decoupled look-back over
+// earlier tiles (st->tile_epoch keeps stale status words of earlier tasks out),
+// then rewrite counts as exclusive row offsets and write the headers.
+constexpr int kScanThreads = 256, kScanPer = 4, kScanTW = kScanThreads * kScanPer;
+
+__global__ void __launch_bounds__(kScanThreads)
 k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t *__restrict__ counts,
-           WinHdr *__restrict__ hdr, SlotMeta *meta) {
-  __shared__ int64_t wsum[32];
+           WinHdr *__restrict__ hdr, SlotMeta *meta, uint64_t *__restrict__ status, int *__restrict__ ticket) {
+  __shared__ int64_t wsum[kScanThreads / 32];
+  __shared__ int64_t s_base;
+  __shared__ int s_t;
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  const uint64_t epoch = (uint64_t)st->tile_epoch;
   const int S = p.S;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const int64_t per = (nw + blockDim.x - 1) / blockDim.x;
-  const int64_t a = (int64_t)tid * per, b = (a + per < nw) ? a + per : nw;
-  int64_t local = 0;
-  if (S == 1 && per <= 16) {
-    int64_t v[16];                           // issue all loads before summing (one latency)
-#pragma unroll
-    for (int k = 0; k < 16; ++k) v[k] = (a + k < b) ? counts[a + k] : 0;
-#pragma unroll
-    for (int k = 0; k < 16; ++k) local += v[k];
-  } else {
-    for (int64_t j = a; j < b; ++j)
-      for (int s = 0; s < S; ++s) local += counts[j * S + s];
+  const int64_t ntiles = (nw + kScanTW - 1) / kScanTW;
+  if (nw <= 0) {
+    if (blockIdx.x == 0 && tid == 0) { meta->nrows = 0; st->sel_rows = 0; }
+    return;
   }
-  int64_t x = local;
+  for (;;) {
+    if (tid == 0) s_t = atomicAdd(ticket, 1);
+    __syncthreads();
+    const int64_t t = s_t;
+    if (t >= ntiles) break;
+    const int64_t a = t * kScanTW + (int64_t)tid * kScanPer;
+    int64_t wt[kScanPer];
+    int64_t local = 0;
 #pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    int64_t y = (int64_t)__shfl_up_sync(kFull, (unsigned long long)x, o);
-    if (lane >= o) x += y;
-  }
-  if (lane == 31) wsum[wid] = x;
-  __syncthreads();
-  if (wid == 0) {
-    int64_t w = wsum[lane], s = w;
+    for (int k = 0; k < kScanPer; ++k) {
+      wt[k] = 0;
+      if (a + k < nw)
+        for (int s = 0; s < S; ++s) wt[k] += counts[(a + k) * S + s];
+      local += wt[k];
+    }
+    int64_t x = local;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      int64_t y = (int64_t)__shfl_up_sync(kFull, (unsigned long long)s, o);
-      if (lane >= o) s += y;
+      const int64_t y = (int64_t)__shfl_up_sync(kFull, (unsigned long long)x, o);
+      if (lane >= o) x += y;
     }
-    wsum[lane] = s - w;
-  }
-  __syncthreads();
-  int64_t run = wsum[wid] + x - local;
-  for (int64_t j = a; j < b; ++j) {
-    WinHdr h;
-    h.window_id = J0 + j;
-    h.ts = (p.win_kind == WK_TIME) ? p.T0 + (J0 + j) * p.l : pane_ts[((J0 + j) * p.L) & (p.R - 1)];
-    h.row_offset = run;
-    int64_t nr = 0;
-    for (int s = 0; s < S; ++s) {
-      int64_t c = counts[j * S + s];
-      counts[j * S + s] = run;
-      run += c;
-      nr += c;
+    if (lane == 31) wsum[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      const int64_t w = lane < kScanThreads / 32 ? wsum[lane] : 0;
+      int64_t y = w;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t z = (int64_t)__shfl_up_sync(kFull, (unsigned long long)y, o);
+        if (lane >= o) y += z;
+      }
+      if (lane < kScanThreads / 32) wsum[lane] = y - w;
+      if (lane == 31) {                           // y = the tile total: look back for the tile's base
+        const uint64_t total = (uint64_t)y;
+        int64_t excl = 0;
+        if (t == 0) {
+          lb_st(&status[0], lb_pack(epoch, 2, total));
+        } else {
+          lb_st(&status[t], lb_pack(epoch, 1, total));
+          for (int64_t i = t - 1;;) {
+            const uint64_t sv = lb_ld(&status[i]);
+            const uint64_t flag = (sv >> 38) & 3ull;
+            if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
+            excl += (int64_t)(sv & ((1ull << 38) - 1));
+            if (flag == 2) break;
+            --i;
+          }
+          lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
+        }
+        s_base = excl;
+        if (t == ntiles - 1) {
+          const int64_t rows = excl + (int64_t)total;
+          meta->nrows = rows;
+          st->sel_rows = rows;
+          if (rows > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+        }
+      }
     }
-    h.nrows = (int32_t)nr;
-    h.flags = 0;
-    hdr[j] = h;
-  }
-  if (tid == blockDim.x - 1) {
-    meta->nrows = run;
-    st->sel_rows = run;
-    if (run > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+    __syncthreads();
+    int64_t run = s_base + wsum[wid] + x - local;
+#pragma unroll
+    for (int k = 0; k < kScanPer; ++k) {
+      const int64_t j = a + k;
+      if (j >= nw) break;
+      WinHdr h;
+      h.window_id = J0 + j;
+      h.ts = (p.win_kind == WK_TIME) ? p.T0 + (J0 + j) * p.l : pane_ts[((J0 + j) * p.L) & (p.R - 1)];
+      h.row_offset = run;
+      h.nrows = (int32_t)wt[k];
+      h.flags = 0;
+      hdr[j] = h;
+      for (int s = 0; s < S; ++s) {
+        const int64_t c = counts[j * S + s];
+        counts[j * S + s] = run;
+        run += c;
+      }
+    }
+    __syncthreads();
   }
 }
 
@@ -288,7 +329,10 @@ cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st)
   return cudaGetLastError();
 }
 cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st) {
-  k_win_scan<<<1, 1024, 0, st>>>(p, q.st, q.pane_ts, s.counts, (WinHdr *)s.hdr, s.meta);
+  // reset the ticket counter (k_task_begin already did for this task; the slab
+  // and hash paths launch no other ticketed kernel before this one)
+  k_win_scan<<<148 * 2, kScanThreads, 0, st>>>(p, q.st, q.pane_ts, s.counts, (WinHdr *)s.hdr, s.meta,
+                                               q.tile_status, q.tile_ctr);
   return cudaGetLastError();
 }
 cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st) {

@@ -213,18 +213,6 @@ k_vh_build_warp(const Plan p, const State *__restrict__ st, const uint64_t *__re
 // chunks in ticket order, count the rows of every (window, slab) item, obtain
 // the chunk's output offset by decoupled look-back over earlier chunks, write
 // the window headers and then the rows.  Replaces count pass + scan + emit pass.
-__device__ __forceinline__ uint64_t lb_ld(const uint64_t *p) {
-  uint64_t v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
-  return v;
-}
-__device__ __forceinline__ void lb_st(uint64_t *p, uint64_t v) {
-  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v));
-}
-__device__ __forceinline__ uint64_t lb_pack(uint64_t epoch, uint64_t flag, uint64_t v) {
-  return ((epoch & 0xffffffull) << 40) | (flag << 38) | (v & ((1ull << 38) - 1));
-}
-
 constexpr int kFusedMaxItems = 256;
 
 template <int GS>

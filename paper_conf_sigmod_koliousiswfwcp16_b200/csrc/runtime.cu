@@ -482,11 +482,11 @@ static saber_status alloc_query(saber_query *q) {
     if (p.key_mode != KM_HASH) {
       CK(cudaMalloc(&q->qd.vh_pre, (size_t)p.R * p.slot_words * 8));
       CK(cudaMalloc(&q->qd.vh_suf, (size_t)p.R * p.slot_words * 8));
-      // look-back status of the fused window pass: one entry per window chunk
-      q->qd.tile_status_cap = p.win_cap + 16;
-      CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
-      CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
     }
+    // look-back status of the fused window pass / the window scan: one entry per window chunk
+    q->qd.tile_status_cap = p.win_cap + 16;
+    CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
+    CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
     if (p.bucket_mode) {
       CK(cudaMalloc(&q->qd.bkt, (size_t)p.bk_vals + (size_t)p.R * p.S * p.nf * p.g * 4 + 256));
     }
