@@ -94,6 +94,14 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
   uint32_t hi = __shfl_sync(kFull, (uint32_t)(v >> 32), src);
   return ((uint64_t)hi << 32) | lo;
 }
+__device__ __forceinline__ uint64_t shfl_up64(uint64_t v, int d = 1) {
+  const uint32_t lo = __shfl_up_sync(kFull, (uint32_t)v, d), hi = __shfl_up_sync(kFull, (uint32_t)(v >> 32), d);
+  return ((uint64_t)hi << 32) | lo;
+}
+__device__ __forceinline__ uint64_t shfl_down64(uint64_t v, int d) {
+  const uint32_t lo = __shfl_down_sync(kFull, (uint32_t)v, d), hi = __shfl_down_sync(kFull, (uint32_t)(v >> 32), d);
+  return ((uint64_t)hi << 32) | lo;
+}
 __device__ __forceinline__ uint64_t shfl_xor64(uint64_t v, int m) {
   uint32_t lo = __shfl_xor_sync(kFull, (uint32_t)v, m);
   uint32_t hi = __shfl_xor_sync(kFull, (uint32_t)(v >> 32), m);

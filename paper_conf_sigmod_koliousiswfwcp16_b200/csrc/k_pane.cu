@@ -52,10 +52,6 @@ __device__ __forceinline__ int64_t fdiv(int64_t x, int64_t d, double inv) {
 __device__ __forceinline__ int64_t pdiv(const Plan &p, int64_t x) {
   return p.g_shift >= 0 ? (x >> p.g_shift) : fdiv(x, p.g, p.g_inv);
 }
-__device__ __forceinline__ uint64_t shfl_up64(uint64_t v) {
-  const uint32_t lo = __shfl_up_sync(kFull, (uint32_t)v, 1), hi = __shfl_up_sync(kFull, (uint32_t)(v >> 32), 1);
-  return ((uint64_t)hi << 32) | lo;
-}
 
 __device__ __forceinline__ uint64_t s_key(const Plan &p, const unsigned char *t, bool &valid, int &err) {
   if (p.key_mode == KM_GLOBAL) return 0;
@@ -482,7 +478,19 @@ __device__ __forceinline__ int divg(const Plan &p, int x) {     // floor(x / g),
 
 enum { KK_GLOBAL = 1, KK_RADIX = 2 };
 
-template <int MODE, int NF, int KK>
+__device__ __forceinline__ uint4 lds_v4(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint32_t sel4(const uint4 &v, int w) {
+  return w == 0 ? v.x : w == 1 ? v.y : w == 2 ? v.z : v.w;
+}
+
+// ONECH: τ, the key and every field lie in one 16-byte chunk of the tuple (Syn:
+// chunk 0), so a tuple costs one 128-bit shared load instead of one 8-way
+// bank-conflicted 32-bit load per field
+template <int MODE, int NF, int KK, bool ONECH>
 __global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? 3 : 2)
 k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
            uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
@@ -538,6 +546,11 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   uint32_t foff[NF];
 #pragma unroll
   for (int f = 0; f < NF; ++f) foff[f] = 4u * p.field[f].word;      // fast path: NF == p.nf
+  // ONECH: word indices inside the shared 16-byte chunk
+  const int ch = p.ts_word >> 2, tw = p.ts_word & 3, kw = KK == KK_RADIX ? p.key[0].word & 3 : 0;
+  int fw[NF];
+#pragma unroll
+  for (int f = 0; f < NF; ++f) fw[f] = p.field[f].word & 3;
   const int64_t Rm = p.R - 1;
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(stages);
   int err = 0;
@@ -574,10 +587,12 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         const uint32_t t = sb + (uint32_t)((valid ? i : ib) * tb);
         const int rel = R0 + xs + i;
         const int q = divg(p, rel);
+        uint4 v4 = make_uint4(0, 0, 0, 0);
+        if (ONECH) v4 = lds_v4(t + 16u * (uint32_t)ch);
         if (first_round) {
           // K1: τ non-decreasing (L347-349) and non-negative (L349-350)
           // (lane 0 reads its predecessor from the stage, or the previous stage's last)
-          const int64_t tau = lds_s64(t + tsoff);
+          const int64_t tau = ONECH ? (int64_t)(((uint64_t)sel4(v4, tw + 1) << 32) | sel4(v4, tw)) : lds_s64(t + tsoff);
           int64_t up = (int64_t)shfl_up64((uint64_t)tau);
           if (lane == 0) up = i > 0 ? lds_s64(t - tb + tsoff) : prev_last;
           if (valid & (tau < up)) err |= ERR_ORDER;
@@ -588,7 +603,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         if (!all_in) valid &= (po >= lo_ofs) & (po < PL);
         uint32_t key = 0;
         if (KK == KK_RADIX) {
-          key = lds_u32(t + koff);
+          key = ONECH ? sel4(v4, kw) : lds_u32(t + koff);
           if (key >= dom) {
             if (valid) err |= ERR_KEY;
             valid = false;
@@ -597,7 +612,8 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         if (valid) {
           double fv[NF];
 #pragma unroll
-          for (int f = 0; f < NF; ++f) fv[f] = (double)__uint_as_float(lds_u32(t + foff[f]));  // NF == nf
+          for (int f = 0; f < NF; ++f)                                   // NF == nf
+            fv[f] = (double)__uint_as_float(ONECH ? sel4(v4, fw[f]) : lds_u32(t + foff[f]));
           if (MODE == TM_LANE) {
             const int e = (po * C + (int)key) * 32 + lane;
             tcnt[e] += 1u;
@@ -661,10 +677,23 @@ static void *p1_mode(const Plan &p) {
 static void *p1_generic(const Plan &p) {
   return p.win_kind == WK_COUNT ? p1_mode<WK_COUNT>(p) : p1_mode<WK_TIME>(p);
 }
+// τ, the key and all fields in one 16-byte chunk (τ must not straddle chunks)
+static bool one_chunk(const Plan &p) {
+  const int ch = p.ts_word >> 2;
+  if ((p.ts_word & 3) == 3) return false;
+  if (p.key_mode != KM_GLOBAL && (p.key[0].word >> 2) != ch) return false;
+  for (int f = 0; f < p.nf; ++f)
+    if ((p.field[f].word >> 2) != ch) return false;
+  return true;
+}
+template <int M, bool OC>
+static void *p1_cnt_nf2(const Plan &p, int kk) {
+  if (kk == KK_GLOBAL) return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_GLOBAL, OC> : (void *)k_pane_cnt<M, 2, KK_GLOBAL, OC>;
+  return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_RADIX, OC> : (void *)k_pane_cnt<M, 2, KK_RADIX, OC>;
+}
 template <int M>
 static void *p1_cnt_nf(const Plan &p, int kk) {
-  if (kk == KK_GLOBAL) return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_GLOBAL> : (void *)k_pane_cnt<M, 2, KK_GLOBAL>;
-  return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_RADIX> : (void *)k_pane_cnt<M, 2, KK_RADIX>;
+  return one_chunk(p) ? p1_cnt_nf2<M, true>(p, kk) : p1_cnt_nf2<M, false>(p, kk);
 }
 // count-window fast kernel, or nullptr when the plan needs the generic one
 static void *p1_cnt(const Plan &p) {

@@ -115,21 +115,27 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
 }
 
 // --------------------------------------------------------------------------
-__global__ void k_zero_panes(const Plan p, const State *st, uint64_t *table) {
+// initialise the pane slots [zero_lo, zero_hi) of the ring: one CTA per slot at a
+// time, one contiguous segment (hash keys, counts, each field) after the other,
+// so no per-word division decides the identity value
+__global__ void __launch_bounds__(256) k_zero_panes(const Plan p, const State *st, uint64_t *table) {
   const int64_t lo = st->zero_lo, hi = st->zero_hi;
   if (hi <= lo) return;
-  const int64_t words = (hi - lo) * p.slot_words;
-  const int64_t co = cnt_off(p);
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < words;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    int64_t pane = lo + i / p.slot_words;
-    int64_t w = i % p.slot_words;
-    uint64_t v;
-    if (p.bucket_mode) v = 0;                             // bucket fill counters
-    else if (w < co) v = kEmpty;                               // hash keys
-    else if (w < co + p.C) v = 0;                         // counts
-    else v = field_identity(p.field[(w - co - p.C) / p.C].kind);
-    table[(pane & (p.R - 1)) * p.slot_words + w] = v;
+  const int64_t W = p.slot_words;
+  for (int64_t pane = lo + blockIdx.x; pane < hi; pane += gridDim.x) {
+    uint64_t *slot = table + (pane & (p.R - 1)) * W;
+    if (p.bucket_mode) {
+      for (int64_t w = threadIdx.x; w < W; w += blockDim.x) slot[w] = 0;
+      continue;
+    }
+    const int64_t co = cnt_off(p);
+    for (int64_t w = threadIdx.x; w < co; w += blockDim.x) slot[w] = kEmpty;          // hash keys
+    for (int64_t w = threadIdx.x; w < p.C; w += blockDim.x) slot[co + w] = 0;         // counts
+    for (int f = 0; f < p.nf; ++f) {
+      const uint64_t v = field_identity(p.field[f].kind);
+      uint64_t *d = slot + fld_off(p, f);
+      for (int64_t w = threadIdx.x; w < p.C; w += blockDim.x) d[w] = v;
+    }
   }
 }
 

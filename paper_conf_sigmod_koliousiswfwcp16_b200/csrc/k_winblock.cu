@@ -1,0 +1,312 @@
+// k_winblock.cu -- window assembly for short windows over few keys (DENSE /
+// GLOBAL keys, K <= 64 panes per window, a pane slot of at most a few hundred
+// words): C1, C3 at G = 64, C4.  One kernel, no van Herk arrays in HBM/L2.
+//
+// The batch operator f_b (§3) combines the K pane partials of
+// each window.  A CTA takes, in ticket order, NB consecutive K-aligned pane
+// blocks; the windows starting in them need panes [b0·K, (b0+NB+1)·K - 1).  It
+// stages those pane slots in shared memory with 1-D TMA bulk copies, and per
+// (block, table word) computes the van Herk / Gil-Werman decomposition in place:
+//   S[a] = ⊕ partial[a .. end of a's block]      (suffix, backward)
+//   V[a] = S[a] ⊕ P[a+K-1],  P = ⊕ partial[start of the next block .. a+K-1]
+// (V[a] = S[a] when a is block-aligned): one combine per window and word for
+// count/sum/min/max alike, the same decomposition as k_vh_build + k_win_packed
+// but without writing and re-reading the prefix/suffix arrays.  Then it counts
+// the rows of its windows (ballots), obtains its output offset by decoupled
+// look-back over earlier tickets and writes headers and rows (window-major,
+// key order inside a window).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "launch_internal.h"
+#include "tma.cuh"
+
+namespace sb {
+
+constexpr int kWbThreads = 256;
+constexpr int kWbMaxWin = 512;          // windows per item (row counts in shared memory)
+constexpr int kWbMaxRounds = 256;       // (window, key) rounds of 256 per item
+
+__device__ __forceinline__ uint64_t wb_combine(int kind, uint64_t a, uint64_t b) {
+  return kind < 0 ? a + b : field_combine(kind, a, b);
+}
+
+template <int NF>
+__global__ void __launch_bounds__(kWbThreads)
+k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table,
+            const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
+            uint64_t *__restrict__ status, int *__restrict__ ticket, int NB) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ uint64_t bar;
+  __shared__ int s_t;
+  __shared__ int64_t s_base;
+  __shared__ int s_wcnt[kWbMaxWin];           // rows per window of the item
+  __shared__ int s_roff[kWbMaxRounds * 8];    // rows per (round, warp) → exclusive offsets
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  const int64_t W = p.slot_words;             // C·(1+nf) words per pane slot
+  const int64_t K = p.K, L = p.L, C = p.C, Rm = p.R - 1;
+  const uint64_t epoch = (uint64_t)st->tile_epoch;
+  const int64_t qlo = J0 * L, qhi = (J1 - 1) * L + K - 1;   // panes read by the task's windows
+  const int64_t bfirst = qlo / K;
+  const int64_t nitems = (qhi / K - bfirst + NB) / NB;       // items covering the blocks of window starts
+  const int NP = (int)((NB + 1) * K - 1);                     // staged panes per item
+  uint64_t *raw = (uint64_t *)smem;                           // [NP][W]
+  // window values: in place over block b0's rows when NB == 1 (the prefix reads
+  // only block b0+1), a separate [NB·K][W] array otherwise
+  uint64_t *V = NB == 1 ? raw : raw + (int64_t)NP * W;
+  const unsigned lt = (1u << lane) - 1u;
+  if (tid == 0) { mbar_init(&bar, 1); fence_mbar_init(); }
+  __syncthreads();
+  uint32_t phase = 0;
+  for (;;) {
+    if (tid == 0) s_t = atomicAdd(ticket, 1);
+    __syncthreads();
+    const int64_t t = s_t;
+    if (t >= nitems) break;
+    const int64_t b0 = bfirst + t * NB;
+    const int64_t q0 = b0 * K;                                // first staged pane
+    // windows of this item: j with j·L in [max(q0, qlo), (b0+NB)·K), j < J1
+    int64_t ja = (q0 + L - 1) / L;
+    if (ja < J0) ja = J0;
+    int64_t jb = ((b0 + NB) * K + L - 1) / L;
+    if (jb > J1) jb = J1;
+    const int nwin = jb > ja ? (int)(jb - ja) : 0;
+    // ---- stage panes [max(q0, qlo), min(q0+NP, qhi+1)) with bulk copies (ring-contiguous runs)
+    const int64_t sa = q0 > qlo ? q0 : qlo;
+    const int64_t se = (q0 + NP) < (qhi + 1) ? (q0 + NP) : (qhi + 1);
+    if (tid == 0) {
+      uint32_t bytes = 0;
+      for (int64_t q = sa; q < se;) {
+        const int64_t run = ((q | Rm) + 1 - q) < (se - q) ? ((q | Rm) + 1 - q) : (se - q);   // up to the ring wrap
+        int64_t done = 0;
+        while (done < run) {
+          const int64_t n = (run - done) * W * 8 < (1 << 20) ? (run - done) : ((1 << 20) / (W * 8));
+          bytes += (uint32_t)(n * W * 8);
+          done += n;
+        }
+        q += run;
+      }
+      mbar_expect_tx(&bar, bytes);
+      for (int64_t q = sa; q < se;) {
+        const int64_t run = ((q | Rm) + 1 - q) < (se - q) ? ((q | Rm) + 1 - q) : (se - q);
+        int64_t done = 0;
+        while (done < run) {
+          const int64_t n = (run - done) * W * 8 < (1 << 20) ? (run - done) : ((1 << 20) / (W * 8));
+          bulk_g2s(raw + (q + done - q0) * W, table + ((q + done) & Rm) * W, (uint32_t)(n * W * 8), &bar);
+          done += n;
+        }
+        q += run;
+      }
+    }
+    for (int i = tid; i < nwin; i += kWbThreads) s_wcnt[i] = 0;
+    mbar_wait(&bar, phase);
+    phase ^= 1u;
+    // ---- van Herk / Gil-Werman per table word (threads over consecutive words,
+    // so shared-memory accesses are conflict-free)
+    if (NB == 1) {
+      // in place: (A) suffix of block b0 into its own rows and prefix of block
+      // b0+1 into its own rows, one thread per (word, direction); (B) V[a] =
+      // S[a] ⊕ P[a+K-1] for a > b0·K, in parallel over (pane, word)
+      const int64_t bs = q0, be = (bs + K - 1) < qhi ? (bs + K - 1) : qhi;
+      const int64_t lo = bs > qlo ? bs : qlo;
+      const int64_t pe = (bs + 2 * K - 2) < qhi ? (bs + 2 * K - 2) : qhi;   // last prefix pane needed
+      for (int64_t x = tid; x < 2 * W; x += kWbThreads) {
+        const bool suffix = x < W;
+        const int64_t w = suffix ? x : x - W;
+        const int f = (int)(w / C) - 1;                       // -1: count word
+        const int kind = f < 0 ? -1 : p.field[f].kind;
+        uint64_t acc = kind < 0 ? 0ull : field_identity(kind);
+        if (suffix) {
+          for (int64_t q = be; q >= lo; --q) {
+            uint64_t *r = raw + (q - q0) * W + w;
+            acc = wb_combine(kind, acc, *r);
+            *r = acc;
+          }
+        } else {
+          for (int64_t q = bs + K; q <= pe; ++q) {
+            uint64_t *r = raw + (q - q0) * W + w;
+            acc = wb_combine(kind, acc, *r);
+            *r = acc;
+          }
+        }
+      }
+      __syncthreads();
+      const int64_t a0 = lo > bs ? lo : bs + 1;                // windows starting at a0..be need a prefix
+      const int64_t a1 = (pe - K + 1) < be ? (pe - K + 1) : be;
+      const int64_t nvals = a1 >= a0 ? (a1 - a0 + 1) * W : 0;
+      for (int64_t x = tid; x < nvals; x += kWbThreads) {
+        const int64_t a = a0 + x / W, w = x % W;
+        const int f = (int)(w / C) - 1;
+        const int kind = f < 0 ? -1 : p.field[f].kind;
+        uint64_t *r = raw + (a - q0) * W + w;
+        *r = wb_combine(kind, *r, raw[(a + K - 1 - q0) * W + w]);
+      }
+    } else {
+      // separate V: one thread per (block, word): suffix into V, then the prefix
+      // of the next block completes the windows starting inside the block
+      for (int64_t x = tid; x < (int64_t)NB * W; x += kWbThreads) {
+        const int bi = (int)(x / W);
+        const int64_t w = x - (int64_t)bi * W;
+        const int f = (int)(w / C) - 1;
+        const int kind = f < 0 ? -1 : p.field[f].kind;
+        const uint64_t id = kind < 0 ? 0ull : field_identity(kind);
+        const int64_t bs = q0 + (int64_t)bi * K;
+        const int64_t lo = bs > qlo ? bs : qlo;
+        if (lo > qhi || lo >= bs + K) continue;
+        const int64_t be = (bs + K - 1) < qhi ? (bs + K - 1) : qhi;
+        uint64_t acc = id;
+        for (int64_t q = be; q >= lo; --q) {
+          acc = wb_combine(kind, acc, raw[(q - q0) * W + w]);
+          V[(q - q0) * W + w] = acc;
+        }
+        acc = id;
+        for (int64_t a = bs + 1; a <= be; ++a) {
+          const int64_t e = a + K - 1;
+          if (e > qhi) break;
+          acc = wb_combine(kind, acc, raw[(e - q0) * W + w]);
+          if (a >= lo) V[(a - q0) * W + w] = wb_combine(kind, V[(a - q0) * W + w], acc);
+        }
+      }
+    }
+    __syncthreads();
+    // ---- rows: (window, key) items in window-major order, 256 per round
+    const int nitem = nwin * (int)C;
+    const int nrounds = (nitem + kWbThreads - 1) / kWbThreads;
+    auto value = [&](int it, int64_t &c, uint64_t (&fv)[kMaxField]) -> bool {
+      const int wi = it / (int)C, key = it - wi * (int)C;
+      const uint64_t *v = V + ((ja + wi) * L - q0) * W;
+      c = (int64_t)v[key];
+      if (c <= 0) return false;
+#pragma unroll
+      for (int f = 0; f < NF; ++f)
+        if (f < p.nf) fv[f] = v[(1 + f) * C + key];
+      return !p.nhave || having_ok(p, c, fv);
+    };
+    for (int r = 0; r < nrounds; ++r) {
+      const int it = r * kWbThreads + tid;
+      int64_t c;
+      uint64_t fv[kMaxField];
+      const bool pres = it < nitem && value(it, c, fv);
+      const unsigned bal = __ballot_sync(kFull, pres);
+      if (lane == 0) s_roff[r * 8 + warp] = __popc(bal);
+      if (pres) atomicAdd(&s_wcnt[it / (int)C], 1);
+    }
+    __syncthreads();
+    if (warp == 0) {                                          // exclusive scan of (round, warp) counts
+      const int n = nrounds * 8;
+      int run = 0;
+      for (int b = 0; b < n; b += 32) {
+        const int v = b + lane < n ? s_roff[b + lane] : 0;
+        int y = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int z = __shfl_up_sync(kFull, y, o);
+          if (lane >= o) y += z;
+        }
+        if (b + lane < n) s_roff[b + lane] = run + y - v;
+        run += __shfl_sync(kFull, y, 31);
+      }
+      if (lane == 0) {
+        const uint64_t total = (uint64_t)run;
+        int64_t excl = 0;
+        if (t == 0) {
+          lb_st(&status[0], lb_pack(epoch, 2, total));
+        } else {
+          lb_st(&status[t], lb_pack(epoch, 1, total));
+          for (int64_t i = t - 1;;) {
+            const uint64_t sv = lb_ld(&status[i]);
+            const uint64_t flag = (sv >> 38) & 3ull;
+            if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
+            excl += (int64_t)(sv & ((1ull << 38) - 1));
+            if (flag == 2) break;
+            --i;
+          }
+          lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
+        }
+        s_base = excl;
+        if (t == nitems - 1) {
+          st->sel_rows = excl + (int64_t)total;
+          if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+        }
+      }
+    }
+    __syncthreads();
+    const int64_t base = s_base;
+    // headers: a window's first row is the offset of its first (window, key) item
+    for (int wi = tid; wi < nwin; wi += kWbThreads) {
+      const int it = wi * (int)C;
+      const int r = it / kWbThreads, ln = it % kWbThreads;
+      int before = 0;                                         // present items of round r before lane ln
+      for (int i = r * kWbThreads + (ln & ~31); i < it; ++i) {
+        int64_t c;
+        uint64_t fv[kMaxField];
+        before += value(i, c, fv);
+      }
+      const int64_t j = ja + wi;
+      WinHdr h;
+      h.window_id = j;
+      h.ts = (p.win_kind == WK_TIME) ? p.T0 + j * p.l : pane_ts[(j * L) & Rm];
+      h.row_offset = base + s_roff[r * 8 + (ln >> 5)] + before;
+      h.nrows = s_wcnt[wi];
+      h.flags = 0;
+      hdr[j - J0] = h;
+    }
+    for (int r = 0; r < nrounds; ++r) {
+      const int it = r * kWbThreads + tid;
+      int64_t c = 0;
+      uint64_t fv[kMaxField];
+#pragma unroll
+      for (int f = 0; f < kMaxField; ++f) fv[f] = 0;
+      const bool pres = it < nitem && value(it, c, fv);
+      const unsigned bal = __ballot_sync(kFull, pres);
+      if (pres) {
+        int64_t kv[kMaxKey];
+        decode_key(p, (uint64_t)(it % (int)C), kv);
+        write_row(p, rows, base + s_roff[r * 8 + warp] + __popc(bal & lt), kv, c, fv);
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------------------
+// host side: usable when an item's staged panes + window values fit in shared
+// memory and its windows / rounds fit the per-item arrays
+static int wb_nb(const Plan &p) {
+  int nb = (int)((32 * p.L + p.K - 1) / p.K);     // about 32 windows per item
+  return nb < 1 ? 1 : nb;
+}
+int wb_smem(const Plan &p) {
+  const int nb = wb_nb(p);
+  return (int)(((nb + 1) * p.K - 1 + (nb == 1 ? 0 : nb * p.K)) * p.slot_words * 8);
+}
+bool wb_usable(const Plan &p) {
+  if (p.key_mode == KM_HASH || p.nagg == 0 || p.K > 64 || (p.slot_words & 1)) return false;   // 16-B bulk copies
+  const int nb = wb_nb(p);
+  const int64_t nwin = (nb * p.K + p.L - 1) / p.L + 1;
+  if (nwin > kWbMaxWin || (nwin * p.C + kWbThreads - 1) / kWbThreads > kWbMaxRounds) return false;
+  return wb_smem(p) <= 96 * 1024;
+}
+static void *wb_kernel(const Plan &p) {
+  return p.nf <= 1 ? (void *)k_win_block<1> : p.nf <= 2 ? (void *)k_win_block<2>
+       : p.nf <= 4 ? (void *)k_win_block<4> : (void *)k_win_block<8>;
+}
+cudaError_t wb_set_attributes(const Plan &p) {
+  return cudaFuncSetAttribute(wb_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, wb_smem(p));
+}
+int wb_blocks_per_sm(const Plan &p) {
+  int b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, wb_kernel(p), kWbThreads, wb_smem(p));
+  return b > 0 ? b : 1;
+}
+cudaError_t launch_windows_block(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st) {
+  const int nb = wb_nb(p);
+  void *args[] = {(void *)&p, (void *)&q.st, (void *)&q.table, (void *)&q.pane_ts, (void *)&s.hdr, (void *)&s.rows,
+                  (void *)&q.tile_status, (void *)&q.tile_ctr, (void *)&nb};
+  return cudaLaunchKernel(wb_kernel(p), dim3(grid), dim3(kWbThreads), args, (size_t)wb_smem(p), st);
+}
+
+}  // namespace sb

@@ -54,23 +54,33 @@ k_vh_build(const Plan p, const State *__restrict__ st, const uint64_t *__restric
     const int kind = f < 0 ? -1 : p.field[f].kind;
     const int64_t bs = b * p.K, be = (bs + p.K - 1 < hi) ? bs + p.K - 1 : hi;
     uint64_t acc = kind < 0 ? 0ull : field_identity(kind);
+    // eight loads in flight per thread, then the dependent combines
+    constexpr int U = 8;
     if (prefix) {
       if (bs < lo) continue;                             // prefixes are only read for blocks starting >= lo
-#pragma unroll 4
-      for (int64_t q = bs; q <= be; ++q) {
-        const int64_t r = (q & Rm) * words + w;
-        const uint64_t v = table[r];
-        acc = kind < 0 ? acc + v : field_combine(kind, acc, v);
-        pre[r] = acc;
+      for (int64_t q0 = bs; q0 <= be; q0 += U) {
+        uint64_t v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = q0 + u <= be ? table[((q0 + u) & Rm) * words + w] : 0ull;
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          if (q0 + u > be) break;
+          acc = kind < 0 ? acc + v[u] : field_combine(kind, acc, v[u]);
+          pre[((q0 + u) & Rm) * words + w] = acc;
+        }
       }
     } else {
       const int64_t qlo = bs > lo ? bs : lo;
-#pragma unroll 4
-      for (int64_t q = be; q >= qlo; --q) {
-        const int64_t r = (q & Rm) * words + w;
-        const uint64_t v = table[r];
-        acc = kind < 0 ? acc + v : field_combine(kind, acc, v);
-        suf[r] = acc;
+      for (int64_t q0 = be; q0 >= qlo; q0 -= U) {
+        uint64_t v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = q0 - u >= qlo ? table[((q0 - u) & Rm) * words + w] : 0ull;
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          if (q0 - u < qlo) break;
+          acc = kind < 0 ? acc + v[u] : field_combine(kind, acc, v[u]);
+          suf[((q0 - u) & Rm) * words + w] = acc;
+        }
       }
     }
   }
@@ -409,9 +419,9 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
 // NB = Cp/32 consecutive passes of 32 slots.  Row order is window-major, key
 // order inside a window, exactly as k_win_fused.  One ballot per (pass, warp)
 // gives every window's row count and every row's offset.
-constexpr int kPackU = 8;     // ballot passes per warp per chunk
+constexpr int kPackU = 16;    // ballot passes per warp per chunk
 
-template <bool F>
+template <bool F, int NF = kMaxField>
 __device__ __forceinline__ bool win_value(const Plan &p, const uint64_t *__restrict__ pre,
                                           const uint64_t *__restrict__ suf, int64_t j, int s, int64_t &c,
                                           uint64_t (&fv)[kMaxField]) {
@@ -422,15 +432,18 @@ __device__ __forceinline__ bool win_value(const Plan &p, const uint64_t *__restr
   c = (int64_t)sa[s] + (aligned ? 0 : (int64_t)pb[s]);
   if (c <= 0) return false;
   if constexpr (F) {
-    FOR_F(f) {
-      const uint64_t x = sa[vh_off(p, f) + s];
-      fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
-    }
+#pragma unroll
+    for (int f = 0; f < NF; ++f)
+      if (f < p.nf) {
+        const uint64_t x = sa[vh_off(p, f) + s];
+        fv[f] = aligned ? x : field_combine(p.field[f].kind, x, pb[vh_off(p, f) + s]);
+      }
     return !p.nhave || having_ok(p, c, fv);
   }
   return true;
 }
 
+template <int NF>
 __global__ void __launch_bounds__(256)
 k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre, const uint64_t *__restrict__ suf,
              const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
@@ -469,7 +482,7 @@ k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ 
       if (j < J1 && slot < p.C) {
         int64_t c;
         uint64_t fv[kMaxField];
-        present = p.nhave ? win_value<true>(p, pre, suf, j, slot, c, fv) : win_value<false>(p, pre, suf, j, slot, c, fv);
+        present = p.nhave ? win_value<true, NF>(p, pre, suf, j, slot, c, fv) : win_value<false, NF>(p, pre, suf, j, slot, c, fv);
       }
       bal[u] = __ballot_sync(kFull, present);
       wtot += __popc(bal[u]);
@@ -525,7 +538,9 @@ k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ 
         if ((bal[u] >> lane) & 1u) {
           int64_t c;
           uint64_t fv[kMaxField];
-          win_value<true>(p, pre, suf, j, slot, c, fv);
+          win_value<true, NF>(p, pre, suf, j, slot, c, fv);
+#pragma unroll
+          for (int f = NF; f < kMaxField; ++f) fv[f] = 0;
           int64_t kv[kMaxKey];
           decode_key(p, (uint64_t)slot, kv);
           write_row(p, rows, r + __popc(bal[u] & lt), kv, c, fv);
@@ -751,8 +766,11 @@ cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev
   if (p.S == 1 && p.C <= 256) {
     int cshift = 0;
     while ((1 << cshift) < p.C) ++cshift;
-    k_win_packed<<<grid, 256, 0, st>>>(p, q.st, q.vh_pre, q.vh_suf, q.pane_ts, (WinHdr *)s.hdr, s.rows,
-                                       q.tile_status, q.tile_ctr, cshift);
+    void (*k)(const Plan, State *, const uint64_t *, const uint64_t *, const int64_t *, WinHdr *, unsigned char *,
+              uint64_t *, int *, int) = p.nf <= 1 ? k_win_packed<1> : p.nf <= 2 ? k_win_packed<2>
+                                     : p.nf <= 4 ? k_win_packed<4> : k_win_packed<8>;
+    k<<<grid, 256, 0, st>>>(p, q.st, q.vh_pre, q.vh_suf, q.pane_ts, (WinHdr *)s.hdr, s.rows, q.tile_status,
+                            q.tile_ctr, cshift);
     return cudaGetLastError();
   }
   const int gpb = 256 / p.GS;

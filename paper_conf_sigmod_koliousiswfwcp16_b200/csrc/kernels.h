@@ -51,6 +51,8 @@ int p1_blocks_per_sm(const Plan &p);
 int p2_blocks_per_sm(const Plan &p);
 int sel_blocks_per_sm(const Plan &p);
 int bk_scan_blocks_per_sm(const Plan &p);
+bool wb_usable(const Plan &p);
+int wb_blocks_per_sm(const Plan &p);
 cudaError_t set_kernel_attributes(const Plan &p);
 
 }  // namespace sb

@@ -15,6 +15,7 @@ cudaError_t set_kernel_attributes(const Plan &p) {
     if (e) return e;
     if (p.p2_smem > 0) e = cudaFuncSetAttribute(p2_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
     if (e) return e;
+    if (p.win_block && (e = wb_set_attributes(p))) return e;
     if (p.key_mode == KM_HASH) {
       e = cudaFuncSetAttribute(p2_kernel_count(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
       if (e) return e;
@@ -67,6 +68,8 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
     if ((e = launch_windows(p, q, s, false, p2_grid, win_chunk, st))) return e;
     if ((e = launch_win_scan(p, q, s, st))) return e;
     if ((e = launch_windows(p, q, s, true, p2_grid, win_chunk, st))) return e;
+  } else if (p.win_block) {
+    if ((e = launch_windows_block(p, q, s, p.wb_grid, st))) return e;
   } else {
     if ((e = launch_windows_fused(p, q, s, p2_grid, st))) return e;
   }

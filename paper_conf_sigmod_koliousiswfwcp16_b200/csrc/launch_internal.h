@@ -34,6 +34,11 @@ int bk_scan_blocks_per_sm(const Plan &p);
 cudaError_t launch_bucket_scan(const Plan &p, const QueryDev &q, const void *tuples, int64_t n, int grid,
                                cudaStream_t st);
 cudaError_t launch_bucket_windows(const Plan &p, const QueryDev &q, const SlotDev &s, int nsm, cudaStream_t st);
+// k_winblock.cu
+bool wb_usable(const Plan &p);
+cudaError_t wb_set_attributes(const Plan &p);
+int wb_blocks_per_sm(const Plan &p);
+cudaError_t launch_windows_block(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st);
 // k_select.cu
 void *sel_kernel(const Plan &p);
 int sel_smem_bytes();

@@ -98,6 +98,7 @@ struct Plan {
   int32_t bucket_mode, bk_shift;  // SB = 1 << bk_shift keys per slab (S = p.S slabs)
   int32_t bk_W, bk_threads;       // windows per assembly chunk, threads per assembly CTA
   int64_t bk_vals;                // byte offset of the value section in the bucket store
+  int32_t win_block, wb_grid;     // short windows over few keys: k_win_block (k_winblock.cu), its grid
 };
 
 // Per-query device state, updated only by kernels on the query's stream.

@@ -519,8 +519,10 @@ static saber_status alloc_query(saber_query *q) {
     if (q->cfg.profile)
       for (auto &e : s.prof) CK(cudaEventCreate(&e));
   }
-  CK(set_kernel_attributes(p));
   CK(cudaDeviceGetAttribute(&q->nsm, cudaDevAttrMultiProcessorCount, q->device));
+  if (p.nagg > 0 && !p.bucket_mode && wb_usable(p) && !getenv_flag("SABER_NO_WINBLOCK")) p.win_block = 1;
+  CK(set_kernel_attributes(p));
+  if (p.win_block) p.wb_grid = wb_blocks_per_sm(p) * q->nsm;
   if (p.lane_alt) {
     Plan &pl = q->plan_lane;
     pl = p;
