@@ -122,6 +122,20 @@ __global__ void __launch_bounds__(256) k_zero_panes(const Plan p, const State *s
   const int64_t lo = st->zero_lo, hi = st->zero_hi;
   if (hi <= lo) return;
   const int64_t W = p.slot_words;
+  bool flat = p.bucket_mode || (p.key_mode != KM_HASH && !p.has_minmax);
+  if (flat && (W & 1) == 0) {
+    // every word's identity is 0: 16-byte stores over the ring-contiguous runs
+    const int64_t Rm = p.R - 1;
+    const int64_t s0 = lo & Rm, n = hi - lo;
+    const int64_t n1 = (s0 + n <= p.R) ? n : p.R - s0;         // panes before the ring wrap
+    uint4 *d1 = (uint4 *)(table + s0 * W), *d2 = (uint4 *)table;
+    const int64_t v1 = n1 * W / 2, v2 = (n - n1) * W / 2;
+    const uint4 z = make_uint4(0, 0, 0, 0);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < v1 + v2; i += (int64_t)gridDim.x * blockDim.x) {
+      if (i < v1) d1[i] = z; else d2[i - v1] = z;
+    }
+    return;
+  }
   for (int64_t pane = lo + blockIdx.x; pane < hi; pane += gridDim.x) {
     uint64_t *slot = table + (pane & (p.R - 1)) * W;
     if (p.bucket_mode) {

@@ -286,6 +286,9 @@ int wb_smem(const Plan &p) {
 bool wb_usable(const Plan &p) {
   if (p.key_mode == KM_HASH || p.nagg == 0 || p.K > 64 || (p.slot_words & 1)) return false;   // 16-B bulk copies
   const int nb = wb_nb(p);
+  // the van Herk phase runs one thread per (block, word) and direction: too few
+  // words leave the CTA idle (C4's 4 keys), those plans keep k_vh_build + k_win_packed
+  if ((nb == 1 ? 2 * p.slot_words : nb * p.slot_words) < 64) return false;
   const int64_t nwin = (nb * p.K + p.L - 1) / p.L + 1;
   if (nwin > kWbMaxWin || (nwin * p.C + kWbThreads - 1) / kWbThreads > kWbMaxRounds) return false;
   return wb_smem(p) <= 96 * 1024;

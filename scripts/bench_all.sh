@@ -6,8 +6,8 @@ run --config C1 --task-mb 32
 run --config C2 --sel 0.5 --task-mb 1024
 run --config C3 --groups 64 --task-mb 1024
 run --config C3 --groups 1024 --task-mb 1024
-run --config C3 --groups 16384 --task-mb 128
-run --config C3 --groups 65536 --task-mb 64
+run --config C3 --groups 16384 --task-mb 512
+run --config C3 --groups 65536 --task-mb 256
 run --config C4 --rate 64 --task-mb 1024
 run --config C4 --rate 4096 --task-mb 1024
 run --config C5a --task-mb 1024
