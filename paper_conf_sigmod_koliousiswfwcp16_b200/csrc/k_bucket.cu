@@ -459,6 +459,14 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
         uint16_t *sl_w = slist + wid * RS;
         const uint4 *cw = (const uint4 *)(cnt + wid * RS) + lane;
         int n = 0;
+        if (RS & 127) {                                       // small slabs: 32 slots per round
+          for (int o = 0; o < RS; o += 32) {
+            const uint32_t c = cnt[wid * RS + o + lane];
+            const unsigned bal = __ballot_sync(kFull, c != 0u);
+            if (c) sl_w[n + __popc(bal & lt)] = (uint16_t)(o + lane);
+            n += __popc(bal);
+          }
+        } else
 #pragma unroll 2
         for (int o = 0; o < RS; o += 128) {
           const uint4 c4 = cw[o >> 2];

@@ -408,8 +408,11 @@ static saber_status size_plan(saber_query *q) {
     // bucket mode: count windows, one int32 key with a large declared domain,
     // fp64 sums of f32 columns, no HAVING (k_bucket.cu).  SB keys per slab so
     // that the slab state (u32 count + nf fp64 sums per key) fits one CTA.
-    if (p.win_kind == WK_COUNT && p.key_mode == KM_HASH && p.key_pack == KP_RADIX && p.nkeys == 1 &&
-        p.fast_path && p.nhave == 0 && p.nagg <= 4 && p.G > kDenseMaxPlan && p.G <= (1ll << 18) && p.g_magic != 0 &&
+    // Also for mid-size declared domains (256 <= G <= 8192) when a pane has at least
+    // G/4 tuples: dense pane tables would then be about as large as the input.
+    const bool mid = p.key_mode == KM_DENSE && p.G >= 256 && p.g * 4 >= p.G;
+    if (p.win_kind == WK_COUNT && (p.key_mode == KM_HASH || mid) && p.key_pack == KP_RADIX && p.nkeys == 1 &&
+        p.fast_path && p.nhave == 0 && p.nagg <= 4 && p.G >= 256 && p.G <= (1ll << 18) && p.g_magic != 0 &&
         p.g <= 65536 && !getenv_flag("SABER_NO_BUCKET")) {
       int64_t sb = std::min<int64_t>(16384, floor_pow2((224 * 1024) / (6 + 8 * p.nf)));
       sb = std::min<int64_t>(sb, next_pow2(p.G));
@@ -424,7 +427,8 @@ static saber_status size_plan(saber_query *q) {
         while ((1ll << p.bk_shift) < sb) ++p.bk_shift;
         p.C = S;
         p.slot_words = S;                                      // per-(pane, slab) fill counters
-        p.bk_threads = 512;
+        p.bk_threads = (int)std::min<int64_t>(512, sb / 2);      // >= 64 slots per warp
+        p.key_mode = KM_HASH;                                    // no dense pane tables
         // windows per assembly chunk: about one chunk per SM and slab per task
         const int64_t nwt = std::max<int64_t>(1, T / p.l);
         const int64_t per_slab = std::max<int64_t>(1, q->nsm_hint / S);

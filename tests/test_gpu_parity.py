@@ -102,7 +102,7 @@ def test_c2_select_project(saber, oracle_lib, sel):
     check(saber, oracle_lib, spec, data, task_bytes=(4 << 20) + 32 * 77)
 
 
-@pytest.mark.parametrize("groups,dom", [(64, True), (64, False), (200, True), (1024, True), (16384, True), (65536, False)])
+@pytest.mark.parametrize("groups,dom", [(64, True), (64, False), (200, True), (300, True), (1024, True), (4096, True), (16384, True), (65536, False)])
 def test_c3_groupby(saber, oracle_lib, groups, dom):
     spec, g = workloads.c3(groups=groups, declare_domain=dom)
     n = 1 << 19
