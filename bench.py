@@ -369,7 +369,8 @@ def main():
     traffic = ncu_traffic(key)
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": (achieved / peak) if achieved else None, "traffic": traffic,
-                "kernel": "k_select" if not spec["aggs"] else "k_pane_agg",
+                "kernel": saber.SCAN_KERNELS[stats_acc[-1]["scan_kind"]] if stats_acc else None,
+                "window_kernels": saber.WINDOW_KERNELS[stats_acc[-1]["window_kind"]] if stats_acc else None,
                 "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,
                 "launches_per_step": scan_launches / max(1, len(stats_acc)), "peak_source": peak_src,
                 "share_of_step": (scan_ms / max(1, len(stats_acc))) / ms_rank if ms_rank else None}

@@ -226,6 +226,10 @@ typedef struct {
   int64_t kernel_launches;
   int64_t scan_launches;        /* launches of the fused scan kernel (pane or select) */
   double scan_ms, assemble_ms;
+  /* kernels the plan runs: scan 0 k_select, 1 k_pane_agg, 2 k_pane_cnt,
+   * 3 k_pane_bucket; window assembly 0 none (σ/π), 1 k_vh_build + k_win_packed/fused,
+   * 2 k_win_block, 3 bucket (k_bkt_count + k_win_scan + k_bkt_emit), 4 hash, 5 slab */
+  int32_t scan_kind, window_kind;
 } saber_stats;
 saber_status saber_query_stats(const saber_query *q, saber_stats *out);
 

@@ -709,6 +709,7 @@ static void *p1_cnt(const Plan &p) {
     default: return nullptr;
   }
 }
+bool p1_is_cnt(const Plan &p) { return p1_cnt(p) != nullptr; }
 void *p1_kernel(const Plan &p) {
   void *k = p1_cnt(p);
   return k ? k : p1_generic(p);

@@ -218,6 +218,68 @@ k_vh_build_warp(const Plan p, const State *__restrict__ st, const uint64_t *__re
   }
 }
 
+// Long windows, many table words: one CTA per (block, direction, group of 32
+// consecutive words).  Lane = word (each warp load is 256 contiguous bytes of a
+// pane slot), warp = one of 8 chunks of the block's panes: chunk totals, a scan
+// of the 8 totals per word in shared memory, then each warp re-walks its chunk.
+__global__ void __launch_bounds__(256)
+k_vh_build_cta(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
+               uint64_t *__restrict__ pre, uint64_t *__restrict__ suf) {
+  __shared__ uint64_t s_tot[8][32];
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t lo = J0 * p.L, hi = (J1 - 1) * p.L + p.K - 1;
+  const int64_t b0 = lo / p.K, b1 = hi / p.K;
+  const int64_t words = p.slot_words, groups = (words + 31) / 32;
+  const int64_t items = (b1 - b0 + 1) * 2 * groups;
+  const int64_t Rm = p.R - 1;
+  for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const int64_t grp = it % groups, rest = it / groups;
+    const bool prefix = rest & 1;
+    const int64_t b = b0 + (rest >> 1);
+    const int64_t w = grp * 32 + lane;
+    const bool live = w < words;
+    const int f = live ? (int)(w / p.C) - 1 : -1;
+    const int kind = f < 0 ? -1 : p.field[f].kind;
+    const uint64_t id = kind < 0 ? 0ull : field_identity(kind);
+    const int64_t bs = b * p.K, be = (bs + p.K - 1 < hi) ? bs + p.K - 1 : hi;
+    if (prefix && bs < lo) continue;                                 // uniform across the CTA
+    const int64_t qa = prefix ? bs : (bs > lo ? bs : lo);
+    const int64_t len = be - qa + 1;
+    const int64_t ch = (len + 7) / 8;
+    const int64_t c0 = warp * ch, c1 = (c0 + ch < len) ? c0 + ch : len;
+    auto pane_of = [&](int64_t k) { return prefix ? qa + k : be - k; };
+    auto ld = [&](int64_t k) { return live ? table[(pane_of(k) & Rm) * words + w] : 0ull; };
+    constexpr int U = 8;
+    uint64_t acc = id;
+    for (int64_t k0 = c0; k0 < c1; k0 += U) {
+      uint64_t v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) v[u] = k0 + u < c1 ? ld(k0 + u) : id;
+#pragma unroll
+      for (int u = 0; u < U; ++u) acc = kind < 0 ? acc + v[u] : field_combine(kind, acc, v[u]);
+    }
+    s_tot[warp][lane] = acc;
+    __syncthreads();
+    uint64_t run = id;                                                // combine of the chunks before this warp's
+    for (int c = 0; c < warp; ++c) run = kind < 0 ? run + s_tot[c][lane] : field_combine(kind, run, s_tot[c][lane]);
+    uint64_t *dst = prefix ? pre : suf;
+    for (int64_t k0 = c0; k0 < c1; k0 += U) {
+      uint64_t v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) v[u] = k0 + u < c1 ? ld(k0 + u) : id;
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (k0 + u >= c1) break;
+        run = kind < 0 ? run + v[u] : field_combine(kind, run, v[u]);
+        if (live) dst[(pane_of(k0 + u) & Rm) * words + w] = run;
+      }
+    }
+    __syncthreads();
+  }
+}
+
 // ---------------------------------------------------------------------------
 // Single pass over the windows closed by a task (DENSE/GLOBAL): CTAs take window
 // chunks in ticket order, count the rows of every (window, slab) item, obtain
@@ -761,7 +823,7 @@ cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev
   // long windows: a CTA per (block, word) when there are few words (no GROUP BY),
   // a warp per (block, word) otherwise; short windows: a thread per (block, word)
   if (p.K > 64 && p.slot_words < 64) k_vh_build_long<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
-  else if (p.K > 64) k_vh_build_warp<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  else if (p.K > 64) k_vh_build_cta<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   else k_vh_build<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   if (p.S == 1 && p.C <= 256) {
     int cshift = 0;

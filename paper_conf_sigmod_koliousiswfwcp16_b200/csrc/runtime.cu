@@ -938,6 +938,10 @@ saber_status saber_query_stats(const saber_query *q, saber_stats *out) {
   if (!q || !out) return SABER_EINVAL;
   *out = q->stats;
   out->tasks_pending = q->next_task - q->next_poll;
+  const Plan &p = q->plan;
+  out->scan_kind = p.nagg == 0 ? 0 : p.bucket_mode ? 3 : p1_is_cnt(p) ? 2 : 1;
+  out->window_kind = p.nagg == 0 ? 0 : p.bucket_mode ? 3 : p.slab_mode ? 5 : p.key_mode == KM_HASH ? 4
+                     : p.win_block ? 2 : 1;
   return SABER_OK;
 }
 
