@@ -159,6 +159,28 @@ def measured_peaks():
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
+def host_link(dev, nbytes=256 << 20, reps=10):
+    """Pinned host<->device copy bandwidth of this GPU, measured in the same run
+    (SURVEY.md §8(d) D5): best of `reps` cudaMemcpyAsync of 256 MiB each way."""
+    import torch
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    out = {}
+    for name, dst, src in (("h2d_gbs", d, h), ("d2h_gbs", h, d)):
+        best = None
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            dst.copy_(src, non_blocking=True)
+            e1.record()
+            e1.synchronize()
+            ms = e0.elapsed_time(e1)
+            best = ms if best is None else min(best, ms)
+        out[name] = nbytes / (best / 1e3) / 1e9
+    del h, d
+    return out
+
+
 def ncu_traffic(config_key):
     """Per-launch DRAM bytes of the dominant kernel from a committed ncu --set full capture."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -373,6 +395,8 @@ def main():
                 "window_kernels": saber.WINDOW_KERNELS[stats_acc[-1]["window_kind"]] if stats_acc else None,
                 "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,
                 "launches_per_step": scan_launches / max(1, len(stats_acc)), "peak_source": peak_src,
+                "scan_grid": stats_acc[-1]["scan_grid"] if stats_acc else None,
+                "window_grid": stats_acc[-1]["window_grid"] if stats_acc else None,
                 "share_of_step": (scan_ms / max(1, len(stats_acc))) / ms_rank if ms_rank else None}
 
     # ---------------- end-to-end through the C ABI from pinned host memory
@@ -427,9 +451,14 @@ def main():
                 d2h_bytes = got_bytes
         q.close()
         e_s = max_over_ranks(statistics.median(e_times))
+        link = host_link(dev)
+        in_gbs = n * tb / e_s / 1e9                          # per GPU
         e2e = {"value": total_tuples / e_s, "unit": "tuples/s", "h2d_bytes_per_step": n * tb,
                "d2h_bytes_per_step": d2h_bytes, "s_per_step": e_s,
-               "input_gbs": total_tuples * tb / e_s / 1e9}
+               "input_gbs": total_tuples * tb / e_s / 1e9,
+               "host_link": {"bound": "h2d", "achieved": in_gbs, "peak": link["h2d_gbs"], "unit": "GB/s",
+                             "frac": in_gbs / link["h2d_gbs"], "d2h_peak": link["d2h_gbs"],
+                             "peak_source": "measured in this run: pinned cudaMemcpyAsync of 256 MiB, best of 10, per GPU"}}
 
     # ---------------- CPU oracle baseline (rank 0, N = 1)
     cpu = None

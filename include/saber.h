@@ -230,6 +230,10 @@ typedef struct {
    * 3 k_pane_bucket; window assembly 0 none (σ/π), 1 k_vh_build + k_win_packed/fused,
    * 2 k_win_block, 3 bucket (k_bkt_count + k_win_scan + k_bkt_emit), 4 hash, 5 slab */
   int32_t scan_kind, window_kind;
+  /* CTAs per launch of the scan kernel and of the main window-assembly kernel */
+  int32_t scan_grid, window_grid;
+  /* 1 if window assembly of a task overlaps the next task's scan (SABER_OVERLAP=1) */
+  int32_t overlap, reserved;
 } saber_stats;
 saber_status saber_query_stats(const saber_query *q, saber_stats *out);
 

@@ -49,6 +49,17 @@ __device__ __forceinline__ int64_t fdiv(int64_t x, int64_t d, double inv) {
   return x / d;
 }
 // pane division: shift for power-of-two pane lengths, reciprocal otherwise
+// trunc(v / d) for int32 v and 0 < d < 2^31 (C semantics), via the double
+// reciprocal inv = 1/d and one exact integer correction
+__device__ __forceinline__ int32_t div_trunc32(int32_t v, int32_t d, double inv) {
+  const uint32_t a = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
+  uint32_t q = (uint32_t)((double)a * inv);
+  const int64_t r = (int64_t)a - (int64_t)q * d;
+  if (r < 0) --q;
+  else if (r >= d) ++q;
+  return v < 0 ? -(int32_t)q : (int32_t)q;
+}
+
 __device__ __forceinline__ int64_t pdiv(const Plan &p, int64_t x) {
   return p.g_shift >= 0 ? (x >> p.g_shift) : fdiv(x, p.g, p.g_inv);
 }
@@ -355,17 +366,27 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         if (FAST) {
           // all fields are fp64 sums of f32 columns; at most one int32 key column, div 1
           if (p.key_mode == KM_GLOBAL) key = 0;
-          else {
-            const int32_t v = *(const int32_t *)(t + 4 * p.key[0].word);
-            if (p.key_pack == KP_RADIX) {
-              if ((uint32_t)v >= (uint32_t)p.key[0].domain) {     // domain < 2^31 on the fast path
-                if (valid) err |= ERR_KEY;
-                valid = false;
+          else if (p.key_pack == KP_RADIX) {
+            // radix-packed int32 key columns, each col / div (C truncation, A17)
+            uint64_t kk = 0;
+            bool bad = false;
+#pragma unroll
+            for (int kc = 0; kc < kMaxKey; ++kc) {
+              if (kc < p.nkeys) {
+                int32_t v = *(const int32_t *)(t + 4 * p.key[kc].word);
+                if (p.key[kc].div != 1) v = div_trunc32(v, p.key[kc].div, p.key[kc].inv);
+                bad |= (uint32_t)v >= (uint32_t)p.key[kc].domain;     // domain < 2^31 on the fast path
+                kk += (uint64_t)(uint32_t)v * (uint64_t)p.key[kc].stride;
               }
-              key = (uint64_t)(uint32_t)v;
-            } else {
-              key = (uint64_t)(int64_t)v ^ 0x8000000000000000ull;
             }
+            if (bad) {
+              if (valid) err |= ERR_KEY;
+              valid = false;
+            }
+            key = kk;
+          } else {
+            const int32_t v = *(const int32_t *)(t + 4 * p.key[0].word);
+            key = (uint64_t)(int64_t)v ^ 0x8000000000000000ull;
           }
 #pragma unroll
           for (int f = 0; f < NF; ++f)
@@ -666,7 +687,7 @@ static void *p1_nf(int nf, bool fast) {
 }
 template <int WK>
 static void *p1_mode(const Plan &p) {
-  const bool f = p.fast_path;
+  const bool f = p.fast_keys;
   switch (p.local_mode) {
     case TM_LANE: return p1_nf<TM_LANE, WK>(p.nf, f);
     case TM_DIRECT: return p1_nf<TM_DIRECT, WK>(p.nf, f);

@@ -51,8 +51,9 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
     if (J1 < J0) J1 = J0;
     st->pos_next = pos0 + n;
     st->J1 = J1;
-    // pane ring: slots of panes [J0·L, phi] must coexist during this task
-    int64_t live_lo = J0 * p.L;
+    // pane ring: slots of panes [J0·L, phi] must coexist during this task (from
+    // the previous task's J0 when its window phase may still be running)
+    int64_t live_lo = (p.overlap ? st->live_J0 : J0) * p.L;
     int64_t zlo = st->zeroed_hi > live_lo ? st->zeroed_hi : live_lo;
     int64_t zhi = zlo;
     if (phi >= 0 && p.nagg > 0) {
@@ -271,14 +272,25 @@ __global__ void k_task_end(const Plan p, State *st, SlotMeta *meta) {
     st->carry_sel ^= 1;
     st->zero_lo = st->zero_hi = 0;
   } else {
-    meta->nrows = st->sel_rows;     // written by the window pass (fused) or k_win_scan
+    if (!p.overlap) meta->nrows = st->sel_rows;     // written by the window pass (fused) or k_win_scan
     meta->ntuples = 0;
   }
   if (p.slab_mode && st->J1 > st->J0) {
     const int64_t c = (st->J1 - 1) * p.L + p.K;
     if (c > st->compacted_hi) st->compacted_hi = c;
   }
+  st->live_J0 = st->J0;
   st->J0 = st->J1;
+}
+
+// overlap plans: close the window phase of a slot that ran on its State snapshot
+__global__ void k_win_end(State *st, const State *wst, SlotMeta *meta) {
+  if (threadIdx.x) return;
+  meta->nrows = wst->sel_rows;
+  if (wst->error) {
+    meta->error |= wst->error;
+    atomicOr(&st->error, wst->error);
+  }
 }
 
 __global__ void k_carry(const Plan p, const State *st, const uint4 *task, const uint4 *carry0,
@@ -308,6 +320,7 @@ __global__ void k_init_state(State *st, int64_t base_index, int64_t first_window
   s.first_task = 1;
   s.carry_pos = base_index;
   s.compacted_hi = first_window * L;
+  s.live_J0 = first_window;
   *st = s;
 }
 
@@ -357,6 +370,10 @@ cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, 
 }
 cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st) {
   k_task_end<<<1, 32, 0, st>>>(p, q.st, s.meta);
+  return cudaGetLastError();
+}
+cudaError_t launch_win_end(const QueryDev &q, const SlotDev &s, cudaStream_t st) {
+  k_win_end<<<1, 32, 0, st>>>(q.st, s.wst, s.meta);
   return cudaGetLastError();
 }
 cudaError_t launch_carry(const Plan &p, const QueryDev &q, const void *tuples, cudaStream_t st) {

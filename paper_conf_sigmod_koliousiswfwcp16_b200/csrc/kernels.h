@@ -12,6 +12,8 @@ struct SlotDev {
   void *hdr;                // saber_win_hdr[win_cap]
   int64_t *counts;          // per (window, slab) row counts → offsets
   SlotMeta *meta;
+  State *wst;               // overlap: State snapshot the slot's window kernels run on
+  int *ticket;              // overlap: the slot's work-ticket counter
 };
 
 struct QueryDev {
@@ -41,6 +43,12 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
 cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
                                int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
                                int sel_grid, cudaStream_t st, cudaEvent_t *evs, int *launches);
+// overlap plans: the task's scan on `cs`, its window phase on `ws` (after
+// `scan_done`, which the caller's next tasks order against)
+cudaError_t launch_agg_task_overlap(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
+                                    int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
+                                    int p1_grid, int p2_grid, cudaStream_t cs, cudaStream_t ws,
+                                    cudaEvent_t scan_done, cudaEvent_t *evs, int *launches);
 cudaError_t launch_init_state(const Plan &p, const QueryDev &q, int64_t base_index, int64_t epoch0, cudaStream_t st);
 cudaError_t launch_partition_plan(int ts_word, int tuple_words, int win_kind, int64_t s, int64_t l,
                                   int64_t T0, const void *tuples, int64_t begin, int64_t n,

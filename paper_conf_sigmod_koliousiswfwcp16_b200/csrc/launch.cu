@@ -79,6 +79,44 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
   return cudaGetLastError();
 }
 
+// Overlap plans (dense/global pane tables, see Plan::overlap).  On `cs`: task
+// prologue, pane-slot initialisation, the scan, a snapshot of State into the
+// slot (the window kernels' J0/J1/epoch) and the task epilogue, which advances
+// J0 so the next task's prologue can run at once.  On `ws`, after `scan_done`:
+// the window phase on the snapshot with the slot's own ticket counter, then
+// k_win_end (row count, window-phase errors).  The caller keeps `cs` at most one
+// task ahead of `ws` (the pane ring keeps [live_J0·L, ...) intact for that).
+cudaError_t launch_agg_task_overlap(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples,
+                                    int64_t n, int final_, int has_wm, int64_t wm, int emit_on_finish,
+                                    int p1_grid, int p2_grid, cudaStream_t cs, cudaStream_t ws,
+                                    cudaEvent_t scan_done, cudaEvent_t *evs, int *launches) {
+  cudaError_t e;
+  if ((e = launch_task_begin(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, cs))) return e;
+  if ((e = launch_zero_panes(p, q, cs))) return e;
+  *launches = 2;
+  if (evs) cudaEventRecord(evs[0], cs);
+  if (n > 0) {
+    if ((e = launch_pane_agg(p, q, tuples, n, p1_grid, cs))) return e;
+    *launches += 1;
+  }
+  if (evs) cudaEventRecord(evs[1], cs);
+  if ((e = cudaMemcpyAsync(s.wst, q.st, sizeof(State), cudaMemcpyDeviceToDevice, cs))) return e;
+  if ((e = cudaMemsetAsync(s.ticket, 0, sizeof(int), cs))) return e;
+  if ((e = launch_task_end(p, q, s, cs))) return e;
+  if ((e = cudaEventRecord(scan_done, cs))) return e;
+  if ((e = cudaStreamWaitEvent(ws, scan_done, 0))) return e;
+  QueryDev qw = q;
+  qw.st = s.wst;
+  qw.tile_ctr = s.ticket;
+  if (p.win_block) e = launch_windows_block(p, qw, s, p.wb_grid, ws);
+  else e = launch_windows_fused(p, qw, s, p2_grid, ws);
+  if (e) return e;
+  if ((e = launch_win_end(q, s, ws))) return e;
+  *launches += p.win_block ? 3 : 4;
+  if (evs) cudaEventRecord(evs[2], ws);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
                                int final_, int has_wm, int64_t wm, int emit_on_finish, int sel_grid, cudaStream_t st,
                                cudaEvent_t *evs, int *launches) {

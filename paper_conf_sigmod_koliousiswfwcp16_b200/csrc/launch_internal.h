@@ -12,6 +12,7 @@ cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s
                               int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st);
 cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st);
 cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);
+cudaError_t launch_win_end(const QueryDev &q, const SlotDev &s, cudaStream_t st);
 cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);
 cudaError_t launch_carry(const Plan &p, const QueryDev &q, const void *tuples, cudaStream_t st);
 // k_pane.cu

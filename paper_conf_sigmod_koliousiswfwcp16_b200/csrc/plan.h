@@ -35,7 +35,7 @@ enum {
 };
 
 struct Pred { int32_t word, type, op, pad; int64_t ival; double fval; };
-struct Key  { int32_t word, type, div, pad; int64_t domain, stride; };
+struct Key  { int32_t word, type, div, pad; int64_t domain, stride; double inv; };   // inv = 1/div
 struct Field { int32_t kind, word, type, pad; };
 struct AggOut { int32_t fn, field, is_float_col, out_float; };
 struct Have { int32_t agg, op, pad0, pad1; int64_t ival; double fval; };
@@ -78,6 +78,7 @@ struct Plan {
   int32_t lane_alt;               // DIRECT plan that may switch to LANE per task (time windows)
   int32_t lane_pl, lane_entries, lane_bytes;
   int32_t fast_path, pad6;        // all fields fp64 sums of f32 columns, <= 1 int32 key (div 1), nf <= 2
+  int32_t fast_keys, pad7;        // k_pane_agg fast path: as fast_path but up to kMaxKey radix int32 keys, div > 0
   // phase-2 window assembly
   int32_t S, SB, GS, pad5;        // key slabs, slots per slab, threads per slab group
   int32_t state_cap, p2_smem;     // hash state entries per CTA, dynamic smem bytes
@@ -99,6 +100,10 @@ struct Plan {
   int32_t bk_W, bk_threads;       // windows per assembly chunk, threads per assembly CTA
   int64_t bk_vals;                // byte offset of the value section in the bucket store
   int32_t win_block, wb_grid;     // short windows over few keys: k_win_block (k_winblock.cu), its grid
+  // window phase of task i on a second stream, concurrent with the scan of task
+  // i+1 (dense/global pane tables): window kernels read a per-slot snapshot of
+  // State, and the pane ring keeps the previous task's windows live
+  int32_t overlap, pad9;
 };
 
 // Per-query device state, updated only by kernels on the query's stream.
@@ -122,6 +127,7 @@ struct State {
   int64_t sel_rows;               // rows written by the compaction kernel
   int64_t tile_epoch;             // look-back epoch
   int64_t compacted_hi;           // slab mode: panes < compacted_hi have bucketed lists
+  int64_t live_J0;                // overlap: first window of the task whose window phase may still run
 };
 
 // Per result slot metadata, copied to the host after a task.

@@ -38,6 +38,7 @@ struct Slot {
   saber_win_hdr *h_hdr = nullptr;
   SlotMeta *h_meta = nullptr;
   cudaEvent_t done = nullptr;
+  cudaEvent_t scan_done = nullptr;      // overlap plans: the task's scan + epilogue on cs
   cudaEvent_t prof[3] = {nullptr, nullptr, nullptr};
   bool profiled = false, scanned = false;
   int64_t task_id = -1;
@@ -74,6 +75,7 @@ struct saber_query {
   int device = 0, nsm = 148;
   int nsm_hint = 148;           // SM count known at planning time
   cudaStream_t cs = nullptr, h2d = nullptr, d2h = nullptr;
+  cudaStream_t ws = nullptr;    // overlap plans: window phases (Plan::overlap)
   QueryDev qd{};
   std::vector<Slot> slots;
   std::vector<Stage> stages;
@@ -250,6 +252,7 @@ static saber_status build_plan(saber_query *q, const saber_schema *sc, const sab
     p.key[i].word = sc->offsets[k.col] / 4;
     p.key[i].type = sc->types[k.col];
     p.key[i].div = k.div;
+    p.key[i].inv = 1.0 / (double)k.div;
     p.key[i].domain = k.domain;
     all_dom &= k.domain > 0;
     prod *= (long double)(k.domain > 0 ? k.domain : 1);
@@ -367,6 +370,16 @@ static saber_status size_plan(saber_query *q) {
         fast &= p.key[0].type == T_I32 && p.key[0].div == 1 &&
                 ((p.key_pack == KP_RADIX && p.key[0].domain < (1ll << 31)) || p.key_pack == KP_BIASED64);
       p.fast_path = fast ? 1 : 0;
+      // generic scan: several radix-packed int32 keys (C5a's plug/household/house,
+      // C5b's highway/direction/position÷5280) on the same fast path
+      bool fk = p.nf <= 2;
+      for (int f = 0; f < p.nf; ++f) fk &= p.field[f].kind == FK_SUM_F && p.field[f].type == T_F32;
+      if (p.nkeys > 0 && p.key_pack == KP_RADIX)
+        for (int i = 0; i < p.nkeys; ++i)
+          fk &= p.key[i].type == T_I32 && p.key[i].div > 0 && p.key[i].domain < (1ll << 31);
+      else if (p.nkeys > 0)
+        fk &= p.fast_path != 0;
+      p.fast_keys = (fk || p.fast_path) ? 1 : 0;
     }
     // phase-2 geometry
     const int smem_budget = 96 * 1024;
@@ -437,6 +450,12 @@ static saber_status size_plan(saber_query *q) {
         p.p2_smem = 0;
       }
     }
+    // dense / global count-window plans overlap the window phase of a task with the
+    // next task's scan (Plan::overlap): the ring then holds two tasks' panes
+    if (!p.bucket_mode && !p.slab_mode && p.key_mode != KM_HASH && p.win_kind == WK_COUNT && c.max_panes <= 0) {
+      const int64_t R2 = next_pow2(2 * ((T + p.g - 1) / p.g + 2) + p.K + p.L + 2);
+      if (R2 > p.R && R2 * slot_bytes <= (1ll << 30)) p.R = R2;
+    }
     // output columns (keys then aggregates)
     p.ncols = p.nkeys + p.nagg;
     p.row_bytes = 0;
@@ -477,6 +496,7 @@ static saber_status alloc_query(saber_query *q) {
   CK(cudaStreamCreateWithFlags(&q->cs, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&q->h2d, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&q->d2h, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&q->ws, cudaStreamNonBlocking));
   CK(cudaMalloc(&q->qd.st, sizeof(State)));
   CK(cudaMalloc(&q->qd.tile_ctr, 64));
   CK(cudaMalloc(&q->d_tmp, 64));
@@ -514,6 +534,9 @@ static saber_status alloc_query(saber_query *q) {
     CK(cudaMalloc(&s.dev.hdr, (size_t)p.win_cap * sizeof(saber_win_hdr)));
     CK(cudaMalloc(&s.dev.counts, (size_t)p.win_cap * std::max(1, p.S) * 8));
     CK(cudaMalloc(&s.dev.meta, sizeof(SlotMeta)));
+    CK(cudaMalloc(&s.dev.wst, sizeof(State)));
+    CK(cudaMalloc(&s.dev.ticket, 64));
+    CK(cudaEventCreateWithFlags(&s.scan_done, cudaEventDisableTiming));
     CK(cudaMallocHost(&s.h_meta, sizeof(SlotMeta)));
     if (q->cfg.result_mode == SABER_RESULTS_HOST) {
       CK(cudaMallocHost(&s.h_rows, rows_bytes ? rows_bytes : 16));
@@ -527,6 +550,34 @@ static saber_status alloc_query(saber_query *q) {
   if (p.nagg > 0 && !p.bucket_mode && wb_usable(p) && !getenv_flag("SABER_NO_WINBLOCK")) p.win_block = 1;
   CK(set_kernel_attributes(p));
   if (p.win_block) p.wb_grid = wb_blocks_per_sm(p) * q->nsm;
+  // overlap the window phase of task i with the scan of task i+1 (dense / global
+  // pane tables): the ring must hold the panes of two tasks' windows at once
+  // (opt-in: measured on B200, the concurrent window kernel slows the scan more
+  // than it hides -- C3 G=64 3.00 -> 2.84 ms, C4/C5/SG1 10-35% slower)
+  if (p.nagg > 0 && !p.bucket_mode && !p.slab_mode && p.key_mode != KM_HASH && getenv_flag("SABER_OVERLAP")) {
+    const int64_t T = q->task_tuples;
+    const bool fits = p.win_kind == WK_COUNT ? p.R >= 2 * ((T + p.g - 1) / p.g + 2) + p.K + p.L + 2
+                                             : q->cfg.max_panes <= 0;
+    if (fits) p.overlap = 1;
+  }
+  if (p.overlap) {
+    // the scan leaves room on every SM for the previous task's window kernel
+    const char *sb = std::getenv("SABER_OVL_SCAN_BPS"), *wb = std::getenv("SABER_OVL_WIN_BPS");
+    const int bps = p1_blocks_per_sm(p);
+    const int scan_bps = sb ? std::max(1, std::atoi(sb)) : std::max(1, bps - 1);
+    const int win_bps = wb ? std::max(1, std::atoi(wb)) : 1;
+    q->p1_grid = std::min(bps, scan_bps) * q->nsm;
+    q->p2_grid = win_bps * q->nsm;
+    if (p.win_block) p.wb_grid = std::min(wb_blocks_per_sm(p), win_bps) * q->nsm;
+  } else if (p.bucket_mode) {
+    q->p1_grid = bk_scan_blocks_per_sm(p) * q->nsm;
+    q->p2_grid = q->nsm;
+  } else if (p.nagg > 0) {
+    q->p1_grid = p1_blocks_per_sm(p) * q->nsm;
+    q->p2_grid = p2_blocks_per_sm(p) * q->nsm * 2;
+  } else {
+    q->sel_grid = sel_blocks_per_sm(p) * q->nsm;
+  }
   if (p.lane_alt) {
     Plan &pl = q->plan_lane;
     pl = p;
@@ -535,16 +586,8 @@ static saber_status alloc_query(saber_query *q) {
     pl.local_entries = p.lane_entries;
     pl.local_bytes = p.lane_bytes;
     CK(set_kernel_attributes(pl));
-    q->p1_grid_lane = p1_blocks_per_sm(pl) * q->nsm;
-  }
-  if (p.bucket_mode) {
-    q->p1_grid = bk_scan_blocks_per_sm(p) * q->nsm;
-    q->p2_grid = q->nsm;
-  } else if (p.nagg > 0) {
-    q->p1_grid = p1_blocks_per_sm(p) * q->nsm;
-    q->p2_grid = p2_blocks_per_sm(p) * q->nsm * 2;
-  } else {
-    q->sel_grid = sel_blocks_per_sm(p) * q->nsm;
+    const int lbps = p1_blocks_per_sm(pl);
+    q->p1_grid_lane = (p.overlap ? std::max(1, lbps - 1) : lbps) * q->nsm;
   }
   CK(launch_init_state(p, q->qd, q->cfg.base_index, 0, q->cs));
   CK(cudaStreamSynchronize(q->cs));
@@ -571,7 +614,19 @@ static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuple
   cudaError_t e;
   int launches = 0;
   cudaEvent_t *evs = q->cfg.profile ? s.prof : nullptr;
-  if (p.nagg > 0)
+  cudaStream_t done_stream = q->cs;
+  if (p.overlap) {
+    // cs runs at most one task ahead of ws: task k's pane-slot initialisation may
+    // reuse slots that the window phase of task k-2 read
+    if (q->next_task >= 2) {
+      Slot &o = q->slots[(q->next_task - 2) % (int64_t)q->slots.size()];
+      CK(cudaStreamWaitEvent(q->cs, o.done, 0));
+    }
+    e = launch_agg_task_overlap(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish,
+                                lane ? q->p1_grid_lane : q->p1_grid, q->p2_grid, q->cs, q->ws, s.scan_done,
+                                evs, &launches);
+    done_stream = q->ws;
+  } else if (p.nagg > 0)
     e = launch_agg_task(p, q->qd, s.dev, dev, ntuples, final_, has_wm, wm, q->cfg.emit_on_finish,
                         lane ? q->p1_grid_lane : q->p1_grid,
                         q->p2_grid, q->win_chunk, q->cs, evs, &launches);
@@ -583,8 +638,8 @@ static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuple
   s.scanned = (p.nagg == 0) || ntuples > 0;
   if (s.scanned) q->stats.scan_launches += 1;
   if (e != cudaSuccess) return fail(q, SABER_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e));
-  CK(cudaMemcpyAsync(s.h_meta, s.dev.meta, sizeof(SlotMeta), cudaMemcpyDeviceToHost, q->cs));
-  CK(cudaEventRecord(s.done, q->cs));
+  CK(cudaMemcpyAsync(s.h_meta, s.dev.meta, sizeof(SlotMeta), cudaMemcpyDeviceToHost, done_stream));
+  CK(cudaEventRecord(s.done, done_stream));
   s.state = SLOT_BUSY;
   s.task_id = q->next_task++;
   q->stats.tasks += 1;
@@ -659,8 +714,11 @@ void saber_query_destroy(saber_query *q) {
   cudaSetDevice(q->device);
   if (q->cs) cudaStreamSynchronize(q->cs);
   if (q->h2d) cudaStreamSynchronize(q->h2d);
+  if (q->ws) cudaStreamSynchronize(q->ws);
   for (auto &s : q->slots) {
     cudaFree(s.dev.rows); cudaFree(s.dev.hdr); cudaFree(s.dev.counts); cudaFree(s.dev.meta);
+    cudaFree(s.dev.wst); cudaFree(s.dev.ticket);
+    if (s.scan_done) cudaEventDestroy(s.scan_done);
     cudaFreeHost(s.h_meta); cudaFreeHost(s.h_rows); cudaFreeHost(s.h_hdr);
     if (s.done) cudaEventDestroy(s.done);
     for (auto e : s.prof) if (e) cudaEventDestroy(e);
@@ -677,6 +735,7 @@ void saber_query_destroy(saber_query *q) {
   if (q->cs) cudaStreamDestroy(q->cs);
   if (q->h2d) cudaStreamDestroy(q->h2d);
   if (q->d2h) cudaStreamDestroy(q->d2h);
+  if (q->ws) cudaStreamDestroy(q->ws);
   cudaGetLastError();
   delete q;
 }
@@ -942,6 +1001,9 @@ saber_status saber_query_stats(const saber_query *q, saber_stats *out) {
   out->scan_kind = p.nagg == 0 ? 0 : p.bucket_mode ? 3 : p1_is_cnt(p) ? 2 : 1;
   out->window_kind = p.nagg == 0 ? 0 : p.bucket_mode ? 3 : p.slab_mode ? 5 : p.key_mode == KM_HASH ? 4
                      : p.win_block ? 2 : 1;
+  out->scan_grid = p.nagg == 0 ? q->sel_grid : (p.lane_alt && q->use_lane) ? q->p1_grid_lane : q->p1_grid;
+  out->window_grid = p.win_block ? p.wb_grid : q->p2_grid;
+  out->overlap = p.overlap;
   return SABER_OK;
 }
 
@@ -953,6 +1015,7 @@ saber_status saber_query_reset(saber_query *q, int64_t base_index, int64_t first
   CK(cudaSetDevice(q->device));
   CK(cudaStreamSynchronize(q->h2d));
   CK(cudaStreamSynchronize(q->cs));
+  CK(cudaStreamSynchronize(q->ws));
   for (auto &s : q->slots) { s.state = SLOT_FREE; s.task_id = -1; s.profiled = false; }
   for (auto &g : q->stages) g.used = false;
   q->cfg.base_index = base_index;
@@ -976,6 +1039,7 @@ saber_status saber_query_sync(saber_query *q) {
   if (!q) return SABER_EINVAL;
   CK(cudaSetDevice(q->device));
   CK(cudaStreamSynchronize(q->cs));
+  CK(cudaStreamSynchronize(q->ws));
   return SABER_OK;
 }
 
@@ -986,6 +1050,8 @@ saber_status saber_query_record(saber_query *q, void *cuda_stream) {
   cudaEvent_t ev;
   CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
   CK(cudaEventRecord(ev, q->cs));
+  CK(cudaStreamWaitEvent((cudaStream_t)cuda_stream, ev, 0));
+  CK(cudaEventRecord(ev, q->ws));
   CK(cudaStreamWaitEvent((cudaStream_t)cuda_stream, ev, 0));
   CK(cudaEventDestroy(ev));
   return SABER_OK;

@@ -357,3 +357,57 @@ def test_partitioned_queries_match_single_gpu(saber, oracle_lib, cfg, parts):
               "vals": [np.concatenate([s["vals"][i] for s in slices]) for i in range(len(slices[0]["vals"]))],
               "tuples": b"".join(s["tuples"] for s in slices)}
     compare(spec, merged, exp)
+
+
+# ------------------------------------------------- overlapped window phase --
+@pytest.mark.parametrize("case", ["c3_g64", "c3_minmax_ragged", "c4_time", "sg_long", "c1_tumbling"])
+def test_overlap_window_phase(saber, oracle_lib, case, monkeypatch):
+    """Plan::overlap (SABER_OVERLAP=1): the window phase of task i runs on a second
+    stream on a State snapshot while task i+1 scans; results must equal the oracle
+    (many small tasks, ragged sizes, fewer result slots than tasks)."""
+    monkeypatch.setenv("SABER_OVERLAP", "1")
+    if case == "c3_g64":
+        spec, g = workloads.c3(groups=64)
+        spec["window"] = workloads.count_window(4096, 1024)
+        data = gen.generate("syn", 1 << 18, g["seed"], groups=64)
+        tb = 1 << 20
+    elif case == "c3_minmax_ragged":
+        spec, g = workloads.c3(groups=32)
+        spec["window"] = workloads.count_window(2048, 256)
+        spec["aggs"] = [("min", "a1"), ("max", "a3"), ("count", None), ("sum", "a4")]
+        data = gen.generate("syn", 300000, 21, groups=32)
+        tb = 32 * 20011
+    elif case == "c4_time":
+        spec, g = workloads.c4(rate=64)
+        data = gen.generate("cm", 1 << 18, g["seed"], rate=64, groups=g["groups"])
+        tb = 64 * 7001
+    elif case == "sg_long":
+        spec, g = workloads.c5a()
+        spec["window"]["size"] = 120
+        data = gen.generate("sg", 1 << 19, g["seed"], rate=512)
+        tb = 32 * 50000
+    else:
+        spec, g = workloads.c1()
+        data = gen.generate("syn", 1 << 18, g["seed"])
+        tb = 32 * 3000
+    check(saber, oracle_lib, spec, data, task_bytes=tb, result_slots=3)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_radix_keys_with_divisors(saber, oracle_lib, seed):
+    """k_pane_agg fast path for several radix-packed int32 keys (Plan::fast_keys):
+    key = (k, v / d) with C truncation (reading A17) -- negative v in (-d, 0) map to
+    key 0 -- and sums/averages of the f32 column, count and time windows."""
+    rng = np.random.default_rng(500 + seed)
+    n = 20000
+    d = int(rng.choice([3, 7, 5280 // 64]))
+    v = rng.integers(-d + 1, 40 * d, size=n)
+    x = rng.integers(0, 1 << 12, size=n) / 64.0
+    k = rng.integers(0, 5, size=n)
+    for kind in ("count", "time"):
+        tau = np.arange(n) if kind == "count" else np.cumsum(rng.choice([0, 1, 1, 3], size=n))
+        w = {"kind": kind, "size": 64, "slide": 8, "origin": 0}
+        sp = tspec(w, aggs=[("avg", "x"), ("sum", "x"), ("count", None)],
+                   group_by=[("k", 1, 5), ("v", d, 40), ("o", 1, 2)])
+        data = stream(v=v, tau=tau, x=x, k=k, n=n)
+        check(saber, oracle_lib, sp, data, task_bytes=32 * int(rng.choice([777, 5000, 20000])))
