@@ -228,7 +228,8 @@ typedef struct {
   double scan_ms, assemble_ms;
   /* kernels the plan runs: scan 0 k_select, 1 k_pane_agg, 2 k_pane_cnt,
    * 3 k_pane_bucket; window assembly 0 none (σ/π), 1 k_vh_build + k_win_packed/fused,
-   * 2 k_win_block, 3 bucket (k_bkt_count + k_win_scan + k_bkt_emit), 4 hash, 5 slab */
+   * 2 k_win_block, 3 bucket (k_bkt_count + k_win_scan + k_bkt_emit), 4 hash, 5 slab,
+   * 6 k_vh_build + k_win_wide */
   int32_t scan_kind, window_kind;
   /* CTAs per launch of the scan kernel and of the main window-assembly kernel */
   int32_t scan_grid, window_grid;

@@ -279,6 +279,11 @@ __global__ void k_task_end(const Plan p, State *st, SlotMeta *meta) {
     const int64_t c = (st->J1 - 1) * p.L + p.K;
     if (c > st->compacted_hi) st->compacted_hi = c;
   }
+  // the window ends of this task had their block prefixes built (k_vh_build_tile)
+  if (p.nagg > 0 && st->J1 > st->J0) {
+    const int64_t e = (st->J1 - 1) * p.L + p.K;
+    if (e > st->vh_pre_hi) st->vh_pre_hi = e;
+  }
   st->live_J0 = st->J0;
   st->J0 = st->J1;
 }

@@ -280,6 +280,99 @@ k_vh_build_cta(const Plan p, const State *__restrict__ st, const uint64_t *__res
   }
 }
 
+// Long windows, many table words, built only where the task's windows read them
+// and in one pass: items are (block, direction, group of 32 consecutive words),
+// lane = word.  Suffixes S[a] are needed for the window starts a in [a0, a1]
+// (walk each start block backward from its end down to max(block start, a0));
+// prefixes P[e] for the ends e = a+K-1 in [e0, e1] of non-aligned windows, in
+// blocks starting after a0, and only from vh_pre_hi on: the previous task built
+// the prefixes below it, so a block's walk continues from P[start-1].  A CTA walks
+// its range in tiles of 8 warps × kVhU panes: per-lane register scans, warp
+// totals through shared memory, a running carry; the next tile's loads are
+// issued before the current tile is combined.  One table read and one write per
+// (pane, word) and direction (k_vh_build_cta read every word twice, for both
+// directions over the whole pane range of the task).
+constexpr int kVhU = 8;
+
+__global__ void __launch_bounds__(256)
+k_vh_build_tile(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
+                uint64_t *__restrict__ pre, uint64_t *__restrict__ suf) {
+  __shared__ uint64_t s_tot[8][32];
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t K = p.K, Rm = p.R - 1, words = p.slot_words, groups = (words + 31) / 32;
+  const int64_t a0 = J0 * p.L, a1 = (J1 - 1) * p.L, e0 = a0 + K - 1, e1 = a1 + K - 1;
+  const int64_t sb0 = a0 / K, nS = a1 / K - sb0 + 1;             // suffix blocks
+  const int64_t pb0 = a0 / K + 1, nP = e1 / K >= pb0 ? e1 / K - pb0 + 1 : 0;   // prefix blocks (start > a0)
+  const int64_t pdone = st->vh_pre_hi;
+  const int64_t items = (nS + nP) * groups;
+  (void)e0;
+  for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const int64_t grp = it % groups, seg = it / groups;
+    const bool prefix = seg >= nS;
+    const int64_t b = prefix ? pb0 + (seg - nS) : sb0 + seg;
+    const int64_t bs = b * K, be = bs + K - 1;
+    int64_t start, len;                                           // walk: pane(k) = start ± k
+    if (prefix) {
+      start = bs > pdone ? bs : pdone;
+      const int64_t end = be < e1 ? be : e1;
+      len = end - start + 1;
+    } else {
+      start = be;
+      len = be - (bs > a0 ? bs : a0) + 1;
+    }
+    if (len <= 0) continue;                                       // uniform across the CTA
+    const int64_t w = grp * 32 + lane;
+    const bool live = w < words;
+    const int f = live ? (int)(w / p.C) - 1 : -1;
+    const int kind = f < 0 ? -1 : p.field[f].kind;
+    const uint64_t id = kind < 0 ? 0ull : field_identity(kind);
+    uint64_t carry = id;
+    if (prefix && start > bs && live) carry = pre[((start - 1) & Rm) * words + w];
+    uint64_t *dst = prefix ? pre : suf;
+    auto pane_of = [&](int64_t k) { return prefix ? start + k : start - k; };
+    uint64_t v[kVhU], vn[kVhU];
+    auto load = [&](int64_t k0, uint64_t (&x)[kVhU]) {
+#pragma unroll
+      for (int u = 0; u < kVhU; ++u) {
+        const int64_t k = k0 + warp * kVhU + u;
+        x[u] = (live && k < len) ? table[(pane_of(k) & Rm) * words + w] : id;
+      }
+    };
+    load(0, vn);
+    for (int64_t k0 = 0; k0 < len; k0 += 8 * kVhU) {
+#pragma unroll
+      for (int u = 0; u < kVhU; ++u) v[u] = vn[u];
+      if (k0 + 8 * kVhU < len) load(k0 + 8 * kVhU, vn);
+      uint64_t acc = id;
+#pragma unroll
+      for (int u = 0; u < kVhU; ++u) {
+        acc = kind < 0 ? acc + v[u] : field_combine(kind, acc, v[u]);
+        v[u] = acc;
+      }
+      s_tot[warp][lane] = acc;
+      __syncthreads();
+      uint64_t run = carry, all = carry;
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        const uint64_t x = s_tot[c][lane];
+        if (c < warp) run = kind < 0 ? run + x : field_combine(kind, run, x);
+        all = kind < 0 ? all + x : field_combine(kind, all, x);
+      }
+      carry = all;
+      if (live) {
+#pragma unroll
+        for (int u = 0; u < kVhU; ++u) {
+          const int64_t k = k0 + warp * kVhU + u;
+          if (k < len) dst[(pane_of(k) & Rm) * words + w] = kind < 0 ? run + v[u] : field_combine(kind, run, v[u]);
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------
 // Single pass over the windows closed by a task (DENSE/GLOBAL): CTAs take window
 // chunks in ticket order, count the rows of every (window, slab) item, obtain
@@ -823,8 +916,10 @@ cudaError_t launch_windows_fused(const Plan &p, const QueryDev &q, const SlotDev
   // long windows: a CTA per (block, word) when there are few words (no GROUP BY),
   // a warp per (block, word) otherwise; short windows: a thread per (block, word)
   if (p.K > 64 && p.slot_words < 64) k_vh_build_long<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  else if (p.K > 64 && p.win_wide) k_vh_build_tile<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   else if (p.K > 64) k_vh_build_cta<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
   else k_vh_build<<<148 * 8, 256, 0, st>>>(p, q.st, q.table, q.vh_pre, q.vh_suf);
+  if (p.win_wide) return launch_windows_wide(p, q, s, p.ww_grid, st);
   if (p.S == 1 && p.C <= 256) {
     int cshift = 0;
     while ((1 << cshift) < p.C) ++cshift;

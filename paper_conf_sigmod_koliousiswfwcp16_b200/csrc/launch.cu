@@ -16,6 +16,7 @@ cudaError_t set_kernel_attributes(const Plan &p) {
     if (p.p2_smem > 0) e = cudaFuncSetAttribute(p2_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
     if (e) return e;
     if (p.win_block && (e = wb_set_attributes(p))) return e;
+    if (p.win_wide && (e = ww_set_attributes(p))) return e;
     if (p.key_mode == KM_HASH) {
       e = cudaFuncSetAttribute(p2_kernel_count(p), cudaFuncAttributeMaxDynamicSharedMemorySize, p.p2_smem);
       if (e) return e;

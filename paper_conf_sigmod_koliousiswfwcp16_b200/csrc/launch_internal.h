@@ -40,6 +40,11 @@ bool wb_usable(const Plan &p);
 cudaError_t wb_set_attributes(const Plan &p);
 int wb_blocks_per_sm(const Plan &p);
 cudaError_t launch_windows_block(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st);
+// k_winwide.cu
+bool ww_usable(const Plan &p);
+cudaError_t ww_set_attributes(const Plan &p);
+int ww_blocks_per_sm(const Plan &p);
+cudaError_t launch_windows_wide(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st);
 // k_select.cu
 void *sel_kernel(const Plan &p);
 int sel_smem_bytes();

@@ -104,6 +104,7 @@ struct Plan {
   // i+1 (dense/global pane tables): window kernels read a per-slot snapshot of
   // State, and the pane ring keeps the previous task's windows live
   int32_t overlap, pad9;
+  int32_t win_wide, ww_grid;       // many dense keys (256 < C <= 2048): k_win_wide (k_winwide.cu), its grid
 };
 
 // Per-query device state, updated only by kernels on the query's stream.
@@ -128,6 +129,7 @@ struct State {
   int64_t tile_epoch;             // look-back epoch
   int64_t compacted_hi;           // slab mode: panes < compacted_hi have bucketed lists
   int64_t live_J0;                // overlap: first window of the task whose window phase may still run
+  int64_t vh_pre_hi;              // van Herk block-prefix values are valid for panes < vh_pre_hi (k_vh_build_tile)
 };
 
 // Per result slot metadata, copied to the host after a task.

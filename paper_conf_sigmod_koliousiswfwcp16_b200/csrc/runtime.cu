@@ -548,8 +548,10 @@ static saber_status alloc_query(saber_query *q) {
   }
   CK(cudaDeviceGetAttribute(&q->nsm, cudaDevAttrMultiProcessorCount, q->device));
   if (p.nagg > 0 && !p.bucket_mode && wb_usable(p) && !getenv_flag("SABER_NO_WINBLOCK")) p.win_block = 1;
+  if (p.nagg > 0 && !p.win_block && ww_usable(p) && !getenv_flag("SABER_NO_WINWIDE")) p.win_wide = 1;
   CK(set_kernel_attributes(p));
   if (p.win_block) p.wb_grid = wb_blocks_per_sm(p) * q->nsm;
+  if (p.win_wide) p.ww_grid = ww_blocks_per_sm(p) * q->nsm;
   // overlap the window phase of task i with the scan of task i+1 (dense / global
   // pane tables): the ring must hold the panes of two tasks' windows at once
   // (opt-in: measured on B200, the concurrent window kernel slows the scan more
@@ -1000,9 +1002,9 @@ saber_status saber_query_stats(const saber_query *q, saber_stats *out) {
   const Plan &p = q->plan;
   out->scan_kind = p.nagg == 0 ? 0 : p.bucket_mode ? 3 : p1_is_cnt(p) ? 2 : 1;
   out->window_kind = p.nagg == 0 ? 0 : p.bucket_mode ? 3 : p.slab_mode ? 5 : p.key_mode == KM_HASH ? 4
-                     : p.win_block ? 2 : 1;
+                     : p.win_block ? 2 : p.win_wide ? 6 : 1;
   out->scan_grid = p.nagg == 0 ? q->sel_grid : (p.lane_alt && q->use_lane) ? q->p1_grid_lane : q->p1_grid;
-  out->window_grid = p.win_block ? p.wb_grid : q->p2_grid;
+  out->window_grid = p.win_block ? p.wb_grid : p.win_wide ? p.ww_grid : q->p2_grid;
   out->overlap = p.overlap;
   return SABER_OK;
 }

@@ -94,7 +94,7 @@ class Stats(C.Structure):
 
 SCAN_KERNELS = ["k_select", "k_pane_agg", "k_pane_cnt", "k_pane_bucket"]
 WINDOW_KERNELS = ["none", "k_vh_build+k_win_packed/k_win_fused", "k_win_block", "k_bkt_count+k_win_scan+k_bkt_emit",
-                  "k_win_hash", "k_win_slab"]
+                  "k_win_hash", "k_win_slab", "k_vh_build+k_win_wide"]
 
 
 # every function declared in include/saber.h: name -> (restype, argtypes)

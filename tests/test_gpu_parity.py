@@ -411,3 +411,29 @@ def test_radix_keys_with_divisors(saber, oracle_lib, seed):
                    group_by=[("k", 1, 5), ("v", d, 40), ("o", 1, 2)])
         data = stream(v=v, tau=tau, x=x, k=k, n=n)
         check(saber, oracle_lib, sp, data, task_bytes=32 * int(rng.choice([777, 5000, 20000])))
+
+
+@pytest.mark.parametrize("case", ["minmax_having", "avg_two_keys_time", "g2048_tumbling"])
+def test_win_wide(saber, oracle_lib, case):
+    """k_win_wide (256 < C <= 2048 dense keys): one window per ticket, rows in key
+    order, look-back per window; HAVING, min/max, ragged tasks."""
+    if case == "minmax_having":
+        spec, _ = workloads.c3(groups=700)
+        spec["window"] = workloads.count_window(640, 64)
+        spec["aggs"] = [("min", "a1"), ("max", "a3"), ("count", None)]
+        spec["having"] = [(2, ">=", 2)]
+        data = gen.generate("syn", 150000, 31, groups=700)
+        tb = 32 * 9973
+    elif case == "avg_two_keys_time":
+        spec, g = workloads.c5b()
+        spec["window"]["size"] = 20
+        spec["window"]["slide"] = 2
+        data = gen.generate("lrb", 1 << 18, 32, rate=512)
+        tb = 32 * 30011
+    else:
+        spec, _ = workloads.c3(groups=2048)
+        spec["window"] = workloads.count_window(512, 512)
+        spec["aggs"] = [("avg", "a1"), ("sum", "a4")]
+        data = gen.generate("syn", 1 << 17, 33, groups=2048)
+        tb = 1 << 20
+    check(saber, oracle_lib, spec, data, task_bytes=tb, result_slots=3)
