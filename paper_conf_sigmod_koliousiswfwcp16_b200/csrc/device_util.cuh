@@ -89,6 +89,15 @@ __device__ __forceinline__ uint64_t field_combine(int kind, uint64_t a, uint64_t
   }
 }
 
+// field_combine without branches (op = FK_*; counts use FK_SUM_I), for loops
+// whose field kind varies across the lanes of a warp
+__device__ __forceinline__ uint64_t field_combine_sel(int op, uint64_t a, uint64_t b) {
+  const uint64_t si = a + b;
+  const uint64_t sf = (uint64_t)__double_as_longlong(__longlong_as_double((long long)a) + __longlong_as_double((long long)b));
+  const uint64_t mn = a < b ? a : b, mx = a < b ? b : a;
+  return op == FK_SUM_F ? sf : op == FK_SUM_I ? si : op == FK_MIN ? mn : mx;
+}
+
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
   uint32_t lo = __shfl_sync(kFull, (uint32_t)v, src);
   uint32_t hi = __shfl_sync(kFull, (uint32_t)(v >> 32), src);

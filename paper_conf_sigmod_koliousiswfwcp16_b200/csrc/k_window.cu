@@ -294,7 +294,7 @@ k_vh_build_cta(const Plan p, const State *__restrict__ st, const uint64_t *__res
 // directions over the whole pane range of the task).
 constexpr int kVhU = 8;
 
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(256, 3)
 k_vh_build_tile(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
                 uint64_t *__restrict__ pre, uint64_t *__restrict__ suf) {
   __shared__ uint64_t s_tot[8][32];
@@ -326,8 +326,8 @@ k_vh_build_tile(const Plan p, const State *__restrict__ st, const uint64_t *__re
     const int64_t w = grp * 32 + lane;
     const bool live = w < words;
     const int f = live ? (int)(w / p.C) - 1 : -1;
-    const int kind = f < 0 ? -1 : p.field[f].kind;
-    const uint64_t id = kind < 0 ? 0ull : field_identity(kind);
+    const int op = f < 0 ? FK_SUM_I : p.field[f].kind;             // count words add as integers
+    const uint64_t id = field_identity(op);
     uint64_t carry = id;
     if (prefix && start > bs && live) carry = pre[((start - 1) & Rm) * words + w];
     uint64_t *dst = prefix ? pre : suf;
@@ -348,7 +348,7 @@ k_vh_build_tile(const Plan p, const State *__restrict__ st, const uint64_t *__re
       uint64_t acc = id;
 #pragma unroll
       for (int u = 0; u < kVhU; ++u) {
-        acc = kind < 0 ? acc + v[u] : field_combine(kind, acc, v[u]);
+        acc = field_combine_sel(op, acc, v[u]);
         v[u] = acc;
       }
       s_tot[warp][lane] = acc;
@@ -357,15 +357,15 @@ k_vh_build_tile(const Plan p, const State *__restrict__ st, const uint64_t *__re
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
         const uint64_t x = s_tot[c][lane];
-        if (c < warp) run = kind < 0 ? run + x : field_combine(kind, run, x);
-        all = kind < 0 ? all + x : field_combine(kind, all, x);
+        if (c < warp) run = field_combine_sel(op, run, x);
+        all = field_combine_sel(op, all, x);
       }
       carry = all;
       if (live) {
 #pragma unroll
         for (int u = 0; u < kVhU; ++u) {
           const int64_t k = k0 + warp * kVhU + u;
-          if (k < len) dst[(pane_of(k) & Rm) * words + w] = kind < 0 ? run + v[u] : field_combine(kind, run, v[u]);
+          if (k < len) dst[(pane_of(k) & Rm) * words + w] = field_combine_sel(op, run, v[u]);
         }
       }
       __syncthreads();

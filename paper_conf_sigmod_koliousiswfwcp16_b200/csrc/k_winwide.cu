@@ -62,23 +62,26 @@ k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pr
     int64_t c[RR];
     uint64_t fv[RR][NF];
     unsigned bal[RR];
+    // all loads of the window first (RR·(1+NF)·2 independent 8-byte loads per thread)
+    uint64_t xs[RR][1 + NF], xp[RR][1 + NF];
 #pragma unroll
     for (int r = 0; r < RR; ++r) {
       const int s = r * kWwThreads + tid;
-      bool pres = false;
-      c[r] = 0;
+      const bool in = s < C;
 #pragma unroll
-      for (int f = 0; f < NF; ++f) fv[r][f] = 0;
-      if (s < C) {
-        c[r] = (int64_t)__ldg(&sa[s]) + (aligned ? 0 : (int64_t)__ldg(&pb[s]));
-#pragma unroll
-        for (int f = 0; f < NF; ++f) {
-          if (f < p.nf) {
-            const uint64_t x = __ldg(&sa[(int64_t)(1 + f) * C + s]);
-            fv[r][f] = aligned ? x : field_combine(kinds[f], x, __ldg(&pb[(int64_t)(1 + f) * C + s]));
-          }
-        }
+      for (int f = 0; f <= NF; ++f) {
+        const bool use = in && (f == 0 || f <= p.nf);
+        xs[r][f] = use ? __ldg(&sa[(int64_t)f * C + s]) : 0ull;
+        xp[r][f] = (use && !aligned) ? __ldg(&pb[(int64_t)f * C + s]) : 0ull;
       }
+    }
+#pragma unroll
+    for (int r = 0; r < RR; ++r) {
+      bool pres = false;
+      c[r] = (int64_t)xs[r][0] + (int64_t)xp[r][0];
+#pragma unroll
+      for (int f = 0; f < NF; ++f)
+        fv[r][f] = aligned ? xs[r][1 + f] : field_combine(kinds[f], xs[r][1 + f], xp[r][1 + f]);
       if (c[r] > 0) {
         uint64_t fa[kMaxField];
 #pragma unroll

@@ -352,8 +352,11 @@ static saber_status size_plan(saber_query *q) {
       p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
     } else if (p.key_mode != KM_HASH && p.C * 2 * ed <= 48 * 1024) {
       // one dense table per CTA, shared atomics (mid-size declared domains)
+      const char *kb = std::getenv("SABER_SHARED_KB");
+      // 24 KiB: one pane of C5a's 2,048 keys, 3 CTAs/SM (48 KiB gave 2: C5a scan 1.98 -> 2.49 TB/s)
+      const int64_t tb = (kb ? std::max(1, std::atoi(kb)) : 24) * 1024;
       p.local_mode = 3;
-      p.local_pl = (int)std::min<int64_t>(1024, (48 * 1024) / (ed * p.C));
+      p.local_pl = (int)std::max<int64_t>(1, std::min<int64_t>(1024, tb / (ed * p.C)));
       p.local_entries = p.local_pl * (int)p.C;
       p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
     } else {
