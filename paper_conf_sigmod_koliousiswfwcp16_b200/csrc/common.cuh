@@ -166,6 +166,43 @@ __device__ __forceinline__ uint64_t lb_pack(uint64_t epoch, uint64_t flag, uint6
   return ((epoch & 0xffffffull) << 40) | (flag << 38) | (v & ((1ull << 38) - 1));
 }
 
+// Decoupled look-back for tile t (called by all 32 lanes of one warp): publishes
+// the tile's aggregate, then inspects 32 predecessors per step (lane i reads
+// tile t-1-i-32·k); the lanes up to the nearest inclusive prefix must all be
+// published before their aggregates are summed.  Returns the exclusive prefix
+// (to every lane) and publishes the inclusive one.  A one-thread walk costs one
+// dependent L2 round trip per predecessor: with hundreds of tiles in flight the
+// chain of a wave's last tile was tens of microseconds.
+__device__ __forceinline__ int64_t lookback_warp(uint64_t *status, int64_t t, uint64_t epoch, uint64_t total) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t ep = epoch & 0xffffffull;
+  const uint64_t vmask = (1ull << 38) - 1;
+  if (t == 0) {
+    if (lane == 0) lb_st(&status[0], lb_pack(epoch, 2, total));
+    return 0;
+  }
+  if (lane == 0) lb_st(&status[t], lb_pack(epoch, 1, total));
+  int64_t excl = 0;
+  for (int64_t i = t - 1;;) {
+    const int64_t idx = i - lane;
+    uint64_t sv = idx >= 0 ? lb_ld(&status[idx]) : lb_pack(epoch, 2, 0);   // before tile 0: inclusive 0
+    const uint64_t flag = (sv >> 38) & 3ull;
+    const bool ok = (sv >> 40) == ep && flag != 0;
+    const unsigned incl = __ballot_sync(kFull, ok && flag == 2);
+    const unsigned bad = __ballot_sync(kFull, !ok);
+    const unsigned need = incl ? (((incl & (0u - incl)) << 1) - 1u) : kFull;   // lanes 0 .. first inclusive
+    if (bad & need) continue;                                                // not all published yet
+    uint64_t v = ((need >> lane) & 1u) ? (sv & vmask) : 0ull;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    excl += (int64_t)v;
+    if (incl) break;
+    i -= 32;
+  }
+  if (lane == 0) lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
+  return excl;
+}
+
 // --------------------------------------------------------------------------
 // window assembly helpers
 struct AggVal { uint64_t bits; bool isf; };

@@ -208,23 +208,9 @@ k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t
         if (lane >= o) y += z;
       }
       if (lane < kScanThreads / 32) wsum[lane] = y - w;
-      if (lane == 31) {                           // y = the tile total: look back for the tile's base
-        const uint64_t total = (uint64_t)y;
-        int64_t excl = 0;
-        if (t == 0) {
-          lb_st(&status[0], lb_pack(epoch, 2, total));
-        } else {
-          lb_st(&status[t], lb_pack(epoch, 1, total));
-          for (int64_t i = t - 1;;) {
-            const uint64_t sv = lb_ld(&status[i]);
-            const uint64_t flag = (sv >> 38) & 3ull;
-            if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
-            excl += (int64_t)(sv & ((1ull << 38) - 1));
-            if (flag == 2) break;
-            --i;
-          }
-          lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
-        }
+      const uint64_t total = (uint64_t)__shfl_sync(kFull, (unsigned long long)y, 31);   // the tile total
+      const int64_t excl = lookback_warp(status, t, epoch, total);
+      if (lane == 31) {
         s_base = excl;
         if (t == ntiles - 1) {
           const int64_t rows = excl + (int64_t)total;

@@ -209,23 +209,9 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
         if (b + lane < n) s_roff[b + lane] = run + y - v;
         run += __shfl_sync(kFull, y, 31);
       }
+      const uint64_t total = (uint64_t)run;
+      const int64_t excl = lookback_warp(status, t, epoch, total);
       if (lane == 0) {
-        const uint64_t total = (uint64_t)run;
-        int64_t excl = 0;
-        if (t == 0) {
-          lb_st(&status[0], lb_pack(epoch, 2, total));
-        } else {
-          lb_st(&status[t], lb_pack(epoch, 1, total));
-          for (int64_t i = t - 1;;) {
-            const uint64_t sv = lb_ld(&status[i]);
-            const uint64_t flag = (sv >> 38) & 3ull;
-            if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
-            excl += (int64_t)(sv & ((1ull << 38) - 1));
-            if (flag == 2) break;
-            --i;
-          }
-          lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
-        }
         s_base = excl;
         if (t == nitems - 1) {
           st->sel_rows = excl + (int64_t)total;

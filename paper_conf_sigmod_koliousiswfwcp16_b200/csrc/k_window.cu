@@ -468,27 +468,15 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
       if (lane == 0) s_total = run;
     }
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (threadIdx.x < 32) {
       const uint64_t total = (uint64_t)s_total;
-      int64_t excl = 0;
-      if (t == 0) {
-        lb_st(&status[0], lb_pack(epoch, 2, total));
-      } else {
-        lb_st(&status[t], lb_pack(epoch, 1, total));
-        for (int64_t i = t - 1;;) {
-          const uint64_t sv = lb_ld(&status[i]);
-          const uint64_t flag = (sv >> 38) & 3ull;
-          if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
-          excl += (int64_t)(sv & ((1ull << 38) - 1));
-          if (flag == 2) break;
-          --i;
+      const int64_t excl = lookback_warp(status, t, epoch, total);
+      if (threadIdx.x == 0) {
+        s_base = excl;
+        if (t == nchunks - 1) {
+          st->sel_rows = excl + (int64_t)total;
+          if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
         }
-        lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
-      }
-      s_base = excl;
-      if (t == nchunks - 1) {
-        st->sel_rows = excl + (int64_t)total;
-        if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
       }
     }
     __syncthreads();
@@ -644,29 +632,24 @@ k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ 
     }
     if (lane == 0) s_wcnt[warp] = wtot;
     __syncthreads();
-    if (threadIdx.x == 0) {
-      int run = 0;
-      for (int w = 0; w < 8; ++w) { const int v = s_wcnt[w]; s_wcnt[w] = run; run += v; }
-      const uint64_t total = (uint64_t)run;
-      int64_t excl = 0;
-      if (t == 0) {
-        lb_st(&status[0], lb_pack(epoch, 2, total));
-      } else {
-        lb_st(&status[t], lb_pack(epoch, 1, total));
-        for (int64_t i = t - 1;;) {
-          const uint64_t sv = lb_ld(&status[i]);
-          const uint64_t flag = (sv >> 38) & 3ull;
-          if ((sv >> 40) != (epoch & 0xffffffull) || flag == 0) continue;
-          excl += (int64_t)(sv & ((1ull << 38) - 1));
-          if (flag == 2) break;
-          --i;
-        }
-        lb_st(&status[t], lb_pack(epoch, 2, (uint64_t)excl + total));
+    if (threadIdx.x < 32) {
+      const int v = lane < 8 ? s_wcnt[lane] : 0;       // exclusive offsets of the 8 warps
+      int x = v;
+#pragma unroll
+      for (int o = 1; o < 8; o <<= 1) {
+        const int y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
       }
-      s_base = excl;
-      if (t == nchunks - 1) {
-        st->sel_rows = excl + (int64_t)total;
-        if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+      const uint64_t total = (uint64_t)__shfl_sync(kFull, x, 7);
+      __syncwarp();
+      if (lane < 8) s_wcnt[lane] = x - v;
+      const int64_t excl = lookback_warp(status, t, epoch, total);
+      if (lane == 0) {
+        s_base = excl;
+        if (t == nchunks - 1) {
+          st->sel_rows = excl + (int64_t)total;
+          if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+        }
       }
     }
     __syncthreads();
