@@ -50,7 +50,12 @@ def parse():
     ap.add_argument("--sel", type=float, default=0.5)
     ap.add_argument("--rate", type=int, default=0)
     ap.add_argument("--tuples-log2", type=int, default=0, help="tuples per GPU (default: the config's)")
-    ap.add_argument("--task-mb", type=int, default=1024, help="query task size φ in MiB")
+    ap.add_argument("--task-mb", type=int, default=4096,
+                    help="query task size φ in MiB (device-resident leg; B200 plateau: DESIGN.md §8 φ sweep)")
+    ap.add_argument("--e2e-task-mb", type=int, default=256,
+                    help="task size φ of the end-to-end leg (finer tasks pipeline H2D with compute)")
+    ap.add_argument("--size", type=int, default=0, help="override the window size (slide sweeps, Fig. 11)")
+    ap.add_argument("--slide", type=int, default=0, help="override the window slide (slide sweeps, Fig. 11)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -76,6 +81,10 @@ def workload(args):
     if args.tuples_log2:
         g["n"] = 1 << args.tuples_log2
     w = spec["window"]
+    if args.size:
+        w["size"] = args.size
+    if args.slide:
+        w["slide"] = args.slide
     desc = {
         "C1": "Syn 32-B, SUM(a1), count w(1024,1024)",
         "C2": f"Syn 32-B, SELECT ts,a1,a2 WHERE a3<sel*2^31 (sel={args.sel}), count w(1024,64), IStream",
@@ -85,6 +94,8 @@ def workload(args):
         "C5b": f"LRB 32-B, AVG(speed) GROUP BY highway,direction,position/5280 HAVING avg<40, time w(300,1), R={g['rate']}/s",
         "SG1": f"SG 32-B, AVG(value), time w(3600,1), R={g['rate']}/s",
     }[c]
+    if args.size or args.slide:
+        desc += f" [window overridden: size {w['size']}, slide {w['slide']}]"
     name = f"{c}: {desc}, 2^{int(np.log2(g['n']))} tuples ({g['n'] * spec['schema']['tuple_bytes'] >> 20} MiB) per GPU"
     return spec, g, name, w
 
@@ -408,7 +419,8 @@ def main():
         host_np = host.numpy()
         e_times = []
         d2h_bytes = 0
-        q = saber.Query(spec, task_bytes=task_bytes, result_mode=saber.RESULTS_HOST, device=local,
+        e2e_task = args.e2e_task_mb << 20
+        q = saber.Query(spec, task_bytes=e2e_task, result_mode=saber.RESULTS_HOST, device=local,
                         base_index=base_index, first_window=first_window, emit_on_finish=(rank == world - 1))
         q.register_host(host_np)
         for it in range(args.warmup + min(args.steps, 3)):
@@ -425,7 +437,7 @@ def main():
             if halo_np is not None:
                 chunks.append(halo_np)
             chunks.append(host_np)
-            per = task_bytes * 7
+            per = e2e_task * 7
             for arr in chunks:
                 off = 0
                 while off < arr.size:
@@ -454,7 +466,7 @@ def main():
         link = host_link(dev)
         in_gbs = n * tb / e_s / 1e9                          # per GPU
         e2e = {"value": total_tuples / e_s, "unit": "tuples/s", "h2d_bytes_per_step": n * tb,
-               "d2h_bytes_per_step": d2h_bytes, "s_per_step": e_s,
+               "d2h_bytes_per_step": d2h_bytes, "s_per_step": e_s, "task_bytes": e2e_task,
                "input_gbs": total_tuples * tb / e_s / 1e9,
                "host_link": {"bound": "h2d", "achieved": in_gbs, "peak": link["h2d_gbs"], "unit": "GB/s",
                              "frac": in_gbs / link["h2d_gbs"], "d2h_peak": link["d2h_gbs"],
