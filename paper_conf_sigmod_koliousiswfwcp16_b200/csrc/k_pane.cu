@@ -31,8 +31,18 @@
 namespace sb {
 
 constexpr int kP1Threads = 256, kP1Warps = kP1Threads / 32;
-constexpr int kStageBytes = 16384;   // 512 32-B tuples: 2 iterations per warp per stage
-constexpr int kStages = 2;
+// stage geometry and DIRECT-table occupancy (compile-time; -D overrides for experiments)
+#ifndef SB_P1_STAGE_KB
+#define SB_P1_STAGE_KB 16
+#endif
+#ifndef SB_P1_STAGES
+#define SB_P1_STAGES 2
+#endif
+#ifndef SB_P1_DIRECT_BPS
+#define SB_P1_DIRECT_BPS 4
+#endif
+constexpr int kStageBytes = SB_P1_STAGE_KB * 1024;   // 16 KiB: 512 32-B tuples, 2 iterations per warp per stage
+constexpr int kStages = SB_P1_STAGES;
 enum { TM_LANE = 0, TM_DIRECT = 1, TM_HASHED = 2, TM_SHARED = 3 };
 
 
@@ -195,7 +205,7 @@ __device__ __forceinline__ void flush_tables(const Plan &p, State *st, uint64_t 
 }
 
 template <int MODE, int WK, int NF, bool FAST>
-__global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? 4 : 2)
+__global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? SB_P1_DIRECT_BPS : 2)
 k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
            uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
   extern __shared__ __align__(128) unsigned char smem[];
@@ -512,7 +522,7 @@ __device__ __forceinline__ uint32_t sel4(const uint4 &v, int w) {
 // chunk 0), so a tuple costs one 128-bit shared load instead of one 8-way
 // bank-conflicted 32-bit load per field
 template <int MODE, int NF, int KK, bool ONECH>
-__global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? 4 : 2)
+__global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? SB_P1_DIRECT_BPS : 2)
 k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
            uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
   extern __shared__ __align__(128) unsigned char smem[];

@@ -16,7 +16,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsaber.so")
+# SABER_LIB: an alternative build of the same sources (tuning experiments, scripts/build_variant.sh)
+LIB_PATH = os.environ.get("SABER_LIB") or os.path.join(_HERE, "libsaber.so")
 
 OK, EINVAL, ENOMEM, EAGAIN = 0, -22, -12, -11
 EORDER, ECUDA, ENCCL, ECLOSED, ETS, EKEY, ECAPACITY = -1001, -1002, -1003, -1004, -1005, -1006, -1007
