@@ -399,9 +399,14 @@ def main():
     per_launch_ms = scan_ms / max(1, scan_launches)
     achieved = per_launch_bytes / (per_launch_ms / 1e3) / 1e9 if per_launch_ms > 0 else None
     key = f"{args.config}_G{args.groups}" if args.config == "C3" else args.config
-    traffic = ncu_traffic(key)
+    traffic, traffic_note = ncu_traffic(key), None
+    if isinstance(traffic, dict):
+        cap_in = traffic["launch_input_bytes"]
+        traffic = traffic["dram_bytes"] * (per_launch_bytes / cap_in) if cap_in else None
+        if cap_in != int(per_launch_bytes):
+            traffic_note = f"scaled from an ncu capture of a {cap_in >> 20} MiB launch"
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+                "frac": (achieved / peak) if achieved else None, "traffic": traffic, "traffic_note": traffic_note,
                 "kernel": saber.SCAN_KERNELS[stats_acc[-1]["scan_kind"]] if stats_acc else None,
                 "window_kernels": saber.WINDOW_KERNELS[stats_acc[-1]["window_kind"]] if stats_acc else None,
                 "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,
