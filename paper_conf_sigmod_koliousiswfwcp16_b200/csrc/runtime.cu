@@ -424,9 +424,11 @@ static saber_status size_plan(saber_query *q) {
     // bucket mode: count windows, one int32 key with a large declared domain,
     // fp64 sums of f32 columns, no HAVING (k_bucket.cu).  SB keys per slab so
     // that the slab state (u32 count + nf fp64 sums per key) fits one CTA.
-    // Also for mid-size declared domains (256 <= G <= 8192) when a pane has at least
+    // Also for mid-size declared domains (1024 <= G <= 8192) when a pane has at least
     // G/4 tuples: dense pane tables would then be about as large as the input.
-    const bool mid = p.key_mode == KM_DENSE && p.G >= 256 && p.g * 4 >= p.G;
+    // (Measured on B200, C3 1 GiB tasks: G = 256 dense 6.3 ms vs bucket 21.9 ms,
+    // G = 512 7.9 vs 13.7, G = 1024 11.5 vs 9.7, G = 2048 21.7 vs 10.5.)
+    const bool mid = p.key_mode == KM_DENSE && p.G >= 1024 && p.g * 4 >= p.G;
     if (p.win_kind == WK_COUNT && (p.key_mode == KM_HASH || mid) && p.key_pack == KP_RADIX && p.nkeys == 1 &&
         p.fast_path && p.nhave == 0 && p.nagg <= 4 && p.G >= 256 && p.G <= (1ll << 18) && p.g_magic != 0 &&
         p.g <= 65536 && !getenv_flag("SABER_NO_BUCKET")) {
