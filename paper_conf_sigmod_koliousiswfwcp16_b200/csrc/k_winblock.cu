@@ -113,36 +113,58 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
       const int64_t bs = q0, be = (bs + K - 1) < qhi ? (bs + K - 1) : qhi;
       const int64_t lo = bs > qlo ? bs : qlo;
       const int64_t pe = (bs + 2 * K - 2) < qhi ? (bs + 2 * K - 2) : qhi;   // last prefix pane needed
-      for (int64_t x = tid; x < 2 * W; x += kWbThreads) {
-        const bool suffix = x < W;
-        const int64_t w = suffix ? x : x - W;
-        const int f = (int)(w / C) - 1;                       // -1: count word
+      // field of table word w (count words first): compares instead of a division
+      auto field_of = [&](int w) {
+        int f = -1;
+#pragma unroll
+        for (int k = 0; k < kMaxField; ++k)
+          if (k < p.nf && w >= (k + 1) * (int)C) f = k;
+        return f;
+      };
+      const int Wi = (int)W;
+      for (int x = tid; x < 2 * Wi; x += kWbThreads) {
+        const bool suffix = x < Wi;
+        const int w = suffix ? x : x - Wi;
+        const int f = field_of(w);
         const int kind = f < 0 ? -1 : p.field[f].kind;
         uint64_t acc = kind < 0 ? 0ull : field_identity(kind);
-        if (suffix) {
-          for (int64_t q = be; q >= lo; --q) {
-            uint64_t *r = raw + (q - q0) * W + w;
-            acc = wb_combine(kind, acc, *r);
-            *r = acc;
-          }
-        } else {
-          for (int64_t q = bs + K; q <= pe; ++q) {
-            uint64_t *r = raw + (q - q0) * W + w;
-            acc = wb_combine(kind, acc, *r);
-            *r = acc;
-          }
+        // 4 loads in flight per step (the combine chain is the only dependency)
+        const int qa = suffix ? (int)(be - q0) : (int)(bs + K - q0);
+        const int qe = suffix ? (int)(lo - q0) : (int)(pe - q0);     // inclusive end of the walk
+        const int n = suffix ? qa - qe + 1 : qe - qa + 1;
+        const int dq = suffix ? -Wi : Wi;
+        uint64_t *r = raw + qa * Wi + w;
+        int k = 0;
+        for (; k + 4 <= n; k += 4) {
+          const uint64_t v0 = r[0], v1 = r[dq], v2 = r[2 * dq], v3 = r[3 * dq];
+          acc = wb_combine(kind, acc, v0); r[0] = acc;
+          acc = wb_combine(kind, acc, v1); r[dq] = acc;
+          acc = wb_combine(kind, acc, v2); r[2 * dq] = acc;
+          acc = wb_combine(kind, acc, v3); r[3 * dq] = acc;
+          r += 4 * dq;
+        }
+        for (; k < n; ++k) {
+          acc = wb_combine(kind, acc, r[0]);
+          r[0] = acc;
+          r += dq;
         }
       }
       __syncthreads();
       const int64_t a0 = lo > bs ? lo : bs + 1;                // windows starting at a0..be need a prefix
       const int64_t a1 = (pe - K + 1) < be ? (pe - K + 1) : be;
-      const int64_t nvals = a1 >= a0 ? (a1 - a0 + 1) * W : 0;
-      for (int64_t x = tid; x < nvals; x += kWbThreads) {
-        const int64_t a = a0 + x / W, w = x % W;
-        const int f = (int)(w / C) - 1;
+      const int nvals = a1 >= a0 ? (int)((a1 - a0 + 1) * W) : 0;
+      // (pane, word) pairs walked incrementally: no division per element
+      const int step_a = kWbThreads / Wi, step_w = kWbThreads % Wi;
+      int ao = tid / Wi, w = tid - (tid / Wi) * Wi;
+      const int base_a = (int)(a0 - q0), Kd = (int)(K - 1) * Wi;
+      for (int x = tid; x < nvals; x += kWbThreads) {
+        const int f = field_of(w);
         const int kind = f < 0 ? -1 : p.field[f].kind;
-        uint64_t *r = raw + (a - q0) * W + w;
-        *r = wb_combine(kind, *r, raw[(a + K - 1 - q0) * W + w]);
+        uint64_t *rr = raw + (base_a + ao) * Wi + w;
+        *rr = wb_combine(kind, *rr, rr[Kd]);
+        ao += step_a;
+        w += step_w;
+        if (w >= Wi) { w -= Wi; ++ao; }
       }
     } else {
       // separate V: one thread per (block, word): suffix into V, then the prefix
@@ -175,8 +197,11 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
     // ---- rows: (window, key) items in window-major order, 256 per round
     const int nitem = nwin * (int)C;
     const int nrounds = (nitem + kWbThreads - 1) / kWbThreads;
+    const int Ci = (int)C;
+    const int cshift = (Ci & (Ci - 1)) == 0 ? __ffs(Ci) - 1 : -1;  // C a power of two: shifts
+    auto win_of = [&](int it) { return cshift >= 0 ? it >> cshift : it / Ci; };
     auto value = [&](int it, int64_t &c, uint64_t (&fv)[kMaxField]) -> bool {
-      const int wi = it / (int)C, key = it - wi * (int)C;
+      const int wi = win_of(it), key = it - wi * Ci;
       const uint64_t *v = V + ((ja + wi) * L - q0) * W;
       c = (int64_t)v[key];
       if (c <= 0) return false;
@@ -192,7 +217,7 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
       const bool pres = it < nitem && value(it, c, fv);
       const unsigned bal = __ballot_sync(kFull, pres);
       if (lane == 0) s_roff[r * 8 + warp] = __popc(bal);
-      if (pres) atomicAdd(&s_wcnt[it / (int)C], 1);
+      if (pres) atomicAdd(&s_wcnt[win_of(it)], 1);
     }
     __syncthreads();
     if (warp == 0) {                                          // exclusive scan of (round, warp) counts
@@ -250,7 +275,7 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
       const unsigned bal = __ballot_sync(kFull, pres);
       if (pres) {
         int64_t kv[kMaxKey];
-        decode_key(p, (uint64_t)(it % (int)C), kv);
+        decode_key(p, (uint64_t)(it - win_of(it) * Ci), kv);
         write_row(p, rows, base + s_roff[r * 8 + warp] + __popc(bal & lt), kv, c, fv);
       }
     }
