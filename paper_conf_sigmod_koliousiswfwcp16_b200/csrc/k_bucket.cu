@@ -588,7 +588,7 @@ cudaError_t launch_bucket_windows(const Plan &p, const QueryDev &q, const SlotDe
   cudaError_t e = launch_win_scan(p, q, s, st);
   if (e) return e;
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&bc, (void *)&q.bkt, (void *)&s.counts, (void *)&s.rows};
-  return cudaLaunchKernel(bk_emit_kernel(p), dim3(nsm), dim3(p.bk_threads), args, (size_t)bk_emit_smem(p), st);
+  return cudaLaunchKernel(bk_emit_kernel(p), dim3(nsm * p.bk_ctas), dim3(p.bk_threads), args, (size_t)bk_emit_smem(p), st);
 }
 
 }  // namespace sb

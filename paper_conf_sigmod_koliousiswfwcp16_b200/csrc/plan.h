@@ -99,6 +99,7 @@ struct Plan {
   int32_t bucket_mode, bk_shift;  // SB = 1 << bk_shift keys per slab (S = p.S slabs)
   int32_t bk_W, bk_threads;       // windows per assembly chunk, threads per assembly CTA
   int64_t bk_vals;                // byte offset of the value section in the bucket store
+  int32_t bk_ctas, pad10;         // emission CTAs per SM
   int32_t win_block, wb_grid;     // short windows over few keys: k_win_block (k_winblock.cu), its grid
   // window phase of task i on a second stream, concurrent with the scan of task
   // i+1 (dense/global pane tables): window kernels read a per-slot snapshot of

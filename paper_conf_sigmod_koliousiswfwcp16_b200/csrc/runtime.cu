@@ -432,7 +432,9 @@ static saber_status size_plan(saber_query *q) {
     if (p.win_kind == WK_COUNT && (p.key_mode == KM_HASH || mid) && p.key_pack == KP_RADIX && p.nkeys == 1 &&
         p.fast_path && p.nhave == 0 && p.nagg <= 4 && p.G >= 256 && p.G <= (1ll << 18) && p.g_magic != 0 &&
         p.g <= 65536 && !getenv_flag("SABER_NO_BUCKET")) {
-      int64_t sb = std::min<int64_t>(16384, floor_pow2((224 * 1024) / (6 + 8 * p.nf)));
+      const char *sbe = std::getenv("SABER_BK_SB");      // tuning: max keys per slab
+      int64_t sb = std::min<int64_t>(sbe ? std::max(256, std::atoi(sbe)) : 16384,
+                                     floor_pow2((224 * 1024) / (6 + 8 * p.nf)));
       sb = std::min<int64_t>(sb, next_pow2(p.G));
       const int64_t S = (p.G + sb - 1) / sb;
       const int64_t st_max = 16384 / p.tuple_bytes;           // tuples per scan stage
@@ -445,11 +447,13 @@ static saber_status size_plan(saber_query *q) {
         while ((1ll << p.bk_shift) < sb) ++p.bk_shift;
         p.C = S;
         p.slot_words = S;                                      // per-(pane, slab) fill counters
-        p.bk_threads = (int)std::min<int64_t>(512, sb / 2);      // >= 64 slots per warp
+        const char *bte = std::getenv("SABER_BK_THREADS"), *bce = std::getenv("SABER_BK_CTAS");
+        p.bk_threads = (int)std::min<int64_t>(bte ? std::atoi(bte) : 512, sb / 2);   // >= 64 slots per warp
+        p.bk_ctas = bce ? std::max(1, std::atoi(bce)) : 1;       // emission CTAs per SM
         p.key_mode = KM_HASH;                                    // no dense pane tables
         // windows per assembly chunk: about one chunk per SM and slab per task
         const int64_t nwt = std::max<int64_t>(1, T / p.l);
-        const int64_t per_slab = std::max<int64_t>(1, q->nsm_hint / S);
+        const int64_t per_slab = std::max<int64_t>(1, q->nsm_hint * p.bk_ctas / S);
         p.bk_W = (int)std::max<int64_t>(16, std::min<int64_t>(1024, (nwt + per_slab - 1) / per_slab));
         p.bk_vals = ((p.R * S * p.g * 2) + 255) & ~255ll;
         p.p2_smem = 0;
