@@ -38,6 +38,9 @@ constexpr int kP1Threads = 256, kP1Warps = kP1Threads / 32;
 #ifndef SB_P1_STAGES
 #define SB_P1_STAGES 2
 #endif
+#ifndef SB_P1_MATCH
+#define SB_P1_MATCH 0
+#endif
 #ifndef SB_P1_DIRECT_BPS
 #define SB_P1_DIRECT_BPS 4
 #endif
@@ -640,11 +643,28 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
             valid = false;
           }
         }
+#if SB_P1_MATCH
+        const unsigned vmask = __ballot_sync(kFull, valid);
+#endif
         if (valid) {
           double fv[NF];
 #pragma unroll
           for (int f = 0; f < NF; ++f)                                   // NF == nf
             fv[f] = (double)__uint_as_float(ONECH ? sel4(v4, fw[f]) : lds_u32(t + foff[f]));
+#if SB_P1_MATCH
+          // warp-private DIRECT table: a lane whose entry no other lane of this
+          // iteration touches updates it with plain loads/stores (no CAS loop)
+          const int em = po * C + (int)key;
+          const bool solo = MODE == TM_DIRECT && __match_any_sync(vmask, em) == (1u << lane);
+          if (solo) {
+            tcnt[em] += 1u;
+#pragma unroll
+            for (int f = 0; f < NF; ++f) {
+              double *a = (double *)&tf[f * TE + em];
+              *a = *a + fv[f];
+            }
+          } else
+#endif
           if (MODE == TM_LANE) {
             const int e = (po * C + (int)key) * 32 + lane;
             tcnt[e] += 1u;
@@ -660,6 +680,9 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
             for (int f = 0; f < NF; ++f) atomicAdd((double *)&tf[f * TE + e], fv[f]);
           }
         }
+#if SB_P1_MATCH
+        __syncwarp();                                        // plain table updates visible to the next iteration
+#endif
       }
       first_round = false;
       if (pl < wend) break;
