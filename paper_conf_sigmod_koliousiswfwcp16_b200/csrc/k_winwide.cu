@@ -17,6 +17,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "common.cuh"
 #include "launch_internal.h"
 
@@ -24,11 +26,11 @@ namespace sb {
 
 constexpr int kWwThreads = 256;
 
-template <int NF, int RR>
+template <int NF, int RR, bool PRE>
 __global__ void __launch_bounds__(kWwThreads)
 k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre, const uint64_t *__restrict__ suf,
            const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
-           uint64_t *__restrict__ status, int *__restrict__ ticket, int ktab) {
+           uint64_t *__restrict__ status, int *__restrict__ ticket, int ktab, const int64_t *__restrict__ offs) {
   extern __shared__ __align__(16) int32_t s_keys[];           // ktab: decoded key columns [nkeys][C]
   __shared__ int s_cnt[RR * 8];                              // rows per (round, warp) -> exclusive offsets
   __shared__ int64_t s_base;
@@ -50,10 +52,10 @@ k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pr
   int kinds[NF];
 #pragma unroll
   for (int f = 0; f < NF; ++f) kinds[f] = f < p.nf ? p.field[f].kind : FK_SUM_I;
-  for (;;) {
-    if (tid == 0) s_t = atomicAdd(ticket, 1);
+  for (int64_t t0 = blockIdx.x;; t0 += gridDim.x) {
+    if (!PRE && tid == 0) s_t = atomicAdd(ticket, 1);
     __syncthreads();
-    const int64_t t = s_t;
+    const int64_t t = PRE ? t0 : (int64_t)s_t;
     if (t >= nw) break;
     const int64_t j = J0 + t, a = j * L;
     const bool aligned = (a % K) == 0;
@@ -111,6 +113,9 @@ k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pr
         run += __shfl_sync(kFull, x, 31);
       }
       const uint64_t total = (uint64_t)run;
+      if (PRE) {                           // offsets from k_win_wide_count + k_win_scan (headers too)
+        if (lane == 0) s_base = offs[t];
+      } else {
       const int64_t excl = lookback_warp(status, t, epoch, total);
       if (lane == 0) {
         s_base = excl;
@@ -125,6 +130,7 @@ k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pr
           st->sel_rows = excl + (int64_t)total;
           if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
         }
+      }
       }
     }
     __syncthreads();
@@ -148,14 +154,88 @@ k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pr
   }
 }
 
+// Row counts per window (keys with count > 0 that pass HAVING) for the
+// look-back-free variant: k_win_scan turns them into offsets + headers, then
+// k_win_wide<.., PRE = true> writes every window independently (grid stride).
+template <int NF, int RR>
+__global__ void __launch_bounds__(kWwThreads)
+k_win_wide_count(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ pre,
+                 const uint64_t *__restrict__ suf, int64_t *__restrict__ counts) {
+  __shared__ int s_w[8];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  const int C = (int)p.C;
+  const int64_t W = p.slot_words, Rm = p.R - 1, K = p.K, L = p.L;
+  int kinds[NF];
+#pragma unroll
+  for (int f = 0; f < NF; ++f) kinds[f] = f < p.nf ? p.field[f].kind : FK_SUM_I;
+  for (int64_t t = blockIdx.x; t < nw; t += gridDim.x) {
+    const int64_t a = (J0 + t) * L;
+    const bool aligned = (a % K) == 0;
+    const uint64_t *sa = suf + (a & Rm) * W;
+    const uint64_t *pb = pre + ((a + K - 1) & Rm) * W;
+    int n = 0;
+#pragma unroll
+    for (int r = 0; r < RR; ++r) {
+      const int s = r * kWwThreads + tid;
+      if (s >= C) continue;
+      const int64_t c = (int64_t)__ldg(&sa[s]) + (aligned ? 0 : (int64_t)__ldg(&pb[s]));
+      bool pres = c > 0;
+      if (pres && p.nhave) {
+        uint64_t fa[kMaxField];
+#pragma unroll
+        for (int f = 0; f < kMaxField; ++f) fa[f] = 0;
+#pragma unroll
+        for (int f = 0; f < NF; ++f) {
+          if (f < p.nf) {
+            const uint64_t x = __ldg(&sa[(int64_t)(1 + f) * C + s]);
+            fa[f] = aligned ? x : field_combine(kinds[f], x, __ldg(&pb[(int64_t)(1 + f) * C + s]));
+          }
+        }
+        pres = having_ok(p, c, fa);
+      }
+      n += pres;
+    }
+    n = __reduce_add_sync(kFull, (unsigned)n);
+    if (lane == 0) s_w[warp] = n;
+    __syncthreads();
+    if (tid == 0) {
+      int tot = 0;
+#pragma unroll
+      for (int w = 0; w < 8; ++w) tot += s_w[w];
+      counts[t] = tot;
+    }
+    __syncthreads();
+  }
+}
+
 // ---------------------------------------------------------------------------
-template <int NF>
+template <int NF, bool PRE>
 static void *ww_rr(int rr) {
-  return rr <= 2 ? (void *)k_win_wide<NF, 2> : rr <= 4 ? (void *)k_win_wide<NF, 4> : (void *)k_win_wide<NF, 8>;
+  return rr <= 2 ? (void *)k_win_wide<NF, 2, PRE> : rr <= 4 ? (void *)k_win_wide<NF, 4, PRE>
+                                                             : (void *)k_win_wide<NF, 8, PRE>;
+}
+template <int NF>
+static void *wc_rr(int rr) {
+  return rr <= 2 ? (void *)k_win_wide_count<NF, 2> : rr <= 4 ? (void *)k_win_wide_count<NF, 4>
+                                                             : (void *)k_win_wide_count<NF, 8>;
+}
+// Plans without HAVING count rows from the count words alone (half the window's
+// words): count + scan + independent emission beats the per-window look-back
+// (C5a 8.85 -> 8.38 ms); with HAVING the count pass re-reads every field and the
+// look-back kernel stays (C5b 5.83 vs 5.89 ms).
+static bool ww_pre(const Plan &p) {
+  const char *v = std::getenv("SABER_WW_LOOKBACK");    // 1: always the single look-back kernel
+  return !(v && *v == '1') && p.nhave == 0;
 }
 static void *ww_kernel(const Plan &p) {
   const int rr = (int)((p.C + kWwThreads - 1) / kWwThreads);
-  return p.nf <= 1 ? ww_rr<1>(rr) : ww_rr<2>(rr);
+  if (ww_pre(p)) return p.nf <= 1 ? ww_rr<1, true>(rr) : ww_rr<2, true>(rr);
+  return p.nf <= 1 ? ww_rr<1, false>(rr) : ww_rr<2, false>(rr);
+}
+static void *wc_kernel(const Plan &p) {
+  const int rr = (int)((p.C + kWwThreads - 1) / kWwThreads);
+  return p.nf <= 1 ? wc_rr<1>(rr) : wc_rr<2>(rr);
 }
 bool ww_usable(const Plan &p) {
   return p.key_mode != KM_HASH && p.C > 256 && p.C <= 8 * kWwThreads && p.nf <= 2 && !p.slab_mode &&
@@ -175,8 +255,18 @@ int ww_blocks_per_sm(const Plan &p) {
 }
 cudaError_t launch_windows_wide(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st) {
   int ktab = ww_smem(p) > 0 ? 1 : 0;
+  const int64_t *offs = s.counts;
+  if (ww_pre(p)) {
+    int b = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, wc_kernel(p), kWwThreads, 0);
+    void *cargs[] = {(void *)&p, (void *)&q.st, (void *)&q.vh_pre, (void *)&q.vh_suf, (void *)&s.counts};
+    cudaError_t e = cudaLaunchKernel(wc_kernel(p), dim3((b > 0 ? b : 1) * 148), dim3(kWwThreads), cargs, 0, st);
+    if (e) return e;
+    if ((e = launch_win_scan(p, q, s, st))) return e;     // offsets + headers + sel_rows
+  }
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&q.vh_pre, (void *)&q.vh_suf, (void *)&q.pane_ts,
-                  (void *)&s.hdr, (void *)&s.rows, (void *)&q.tile_status, (void *)&q.tile_ctr, (void *)&ktab};
+                  (void *)&s.hdr, (void *)&s.rows, (void *)&q.tile_status, (void *)&q.tile_ctr, (void *)&ktab,
+                  (void *)&offs};
   return cudaLaunchKernel(ww_kernel(p), dim3(grid), dim3(kWwThreads), args, (size_t)ww_smem(p), st);
 }
 

@@ -75,7 +75,7 @@ cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, 
     if ((e = launch_windows_fused(p, q, s, p2_grid, st))) return e;
   }
   if ((e = launch_task_end(p, q, s, st))) return e;
-  *launches += p.bucket_mode ? 1 : p.key_mode == KM_HASH ? 4 : 3;
+  *launches += p.bucket_mode ? 1 : p.key_mode == KM_HASH ? 4 : p.win_wide && !p.nhave ? 5 : 3;   // k_win_wide: + count + scan
   if (evs) cudaEventRecord(evs[2], st);
   return cudaGetLastError();
 }
@@ -113,7 +113,7 @@ cudaError_t launch_agg_task_overlap(const Plan &p, const QueryDev &q, const Slot
   else e = launch_windows_fused(p, qw, s, p2_grid, ws);
   if (e) return e;
   if ((e = launch_win_end(q, s, ws))) return e;
-  *launches += p.win_block ? 3 : 4;
+  *launches += p.win_block ? 3 : p.win_wide && !p.nhave ? 6 : 4;
   if (evs) cudaEventRecord(evs[2], ws);
   return cudaGetLastError();
 }
