@@ -307,8 +307,6 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     if (pf < min_pane) pf = min_pane;
     const int ib = wid * per_warp;
     const int ie = ib + per_warp < ntup ? ib + per_warp : ntup;
-    // τ of the tuple before this warp's slice (K1 order check, first round)
-    int64_t carry_tau = (ib > 0 && ib <= ntup) ? *(const int64_t *)(sb + (ib - 1) * tb + 4 * tsw) : prev_last;
     int64_t cur = pf;
     bool first_round = true;
     while (cur <= pl) {
@@ -345,11 +343,9 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         if (first_round) {
           // K1: τ non-decreasing (L347-349) and non-negative (L349-350); the
           // predecessor of lane 0 is the previous iteration's lane 31
-          const int64_t up0 = (int64_t)shfl_up64((uint64_t)tau);
-          const int64_t up = lane == 0 ? carry_tau : up0;
+          const int64_t up = i > 0 ? *(const int64_t *)(t - tb + 4 * tsw) : prev_last;   // predecessor τ
           if (valid & (tau < up)) err |= ERR_ORDER;
           if (valid & (tau < 0)) err |= ERR_TS;
-          carry_tau = (int64_t)shfl64((uint64_t)tau, 31);
         }
         int64_t pane;
         int pw;                                          // this tuple's pane offset from pbase
@@ -624,11 +620,11 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         uint4 v4 = make_uint4(0, 0, 0, 0);
         if (ONECH) v4 = lds_v4(t + 16u * (uint32_t)ch);
         if (first_round) {
-          // K1: τ non-decreasing (L347-349) and non-negative (L349-350)
-          // (lane 0 reads its predecessor from the stage, or the previous stage's last)
+          // K1: τ non-decreasing (L347-349) and non-negative (L349-350); every lane
+          // reads its predecessor's τ from the stage (no shuffles, no lane-0 branch),
+          // the stage's first tuple compares with the previous stage's last
           const int64_t tau = ONECH ? (int64_t)(((uint64_t)sel4(v4, tw + 1) << 32) | sel4(v4, tw)) : lds_s64(t + tsoff);
-          int64_t up = (int64_t)shfl_up64((uint64_t)tau);
-          if (lane == 0) up = i > 0 ? lds_s64(t - tb + tsoff) : prev_last;
+          const int64_t up = i > 0 ? lds_s64(t - tb + tsoff) : prev_last;
           if (valid & (tau < up)) err |= ERR_ORDER;
           if (valid & (tau < 0)) err |= ERR_TS;
           if (valid && rel == q * g && q >= minrel) pane_ts[(P0 + q) & Rm] = tau;
