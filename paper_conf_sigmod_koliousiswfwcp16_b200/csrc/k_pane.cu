@@ -24,6 +24,8 @@
 #include <climits>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "common.cuh"
 #include "launch_internal.h"
 #include "tma.cuh"
@@ -520,10 +522,21 @@ __device__ __forceinline__ uint32_t sel4(const uint4 &v, int w) {
 // ONECH: τ, the key and every field lie in one 16-byte chunk of the tuple (Syn:
 // chunk 0), so a tuple costs one 128-bit shared load instead of one 8-way
 // bank-conflicted 32-bit load per field
-template <int MODE, int NF, int KK, bool ONECH>
+// OC: 0 fields loaded one by one; 1 one 16-byte chunk, word positions chosen at
+// run time; 2 one chunk with τ in words 0-1, the value in word 2 and the key in
+// word 3 (the Syn layout, L1473-1476: ts, a1, a2), selected at compile time
+// (the run-time word selects compile to branch trees in the hot loop)
+template <int W>
+__device__ __forceinline__ uint32_t sel4c(const uint4 &v) {
+  return W == 0 ? v.x : W == 1 ? v.y : W == 2 ? v.z : v.w;
+}
+
+template <int MODE, int NF, int KK, int OC>
 __global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? SB_P1_DIRECT_BPS : 2)
 k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
            uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
+  constexpr bool ONECH = OC != 0;
+  static_assert(OC != 2 || NF == 1, "fixed layout: one value column");
   extern __shared__ __align__(128) unsigned char smem[];
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int tb = p.tuple_bytes;
@@ -623,7 +636,8 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
           // K1: τ non-decreasing (L347-349) and non-negative (L349-350); every lane
           // reads its predecessor's τ from the stage (no shuffles, no lane-0 branch),
           // the stage's first tuple compares with the previous stage's last
-          const int64_t tau = ONECH ? (int64_t)(((uint64_t)sel4(v4, tw + 1) << 32) | sel4(v4, tw)) : lds_s64(t + tsoff);
+          const int64_t tau = OC == 2 ? (int64_t)(((uint64_t)sel4c<1>(v4) << 32) | sel4c<0>(v4))
+                              : ONECH ? (int64_t)(((uint64_t)sel4(v4, tw + 1) << 32) | sel4(v4, tw)) : lds_s64(t + tsoff);
           const int64_t up = i > 0 ? lds_s64(t - tb + tsoff) : prev_last;
           if (valid & (tau < up)) err |= ERR_ORDER;
           if (valid & (tau < 0)) err |= ERR_TS;
@@ -633,7 +647,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         if (!all_in) valid &= (po >= lo_ofs) & (po < PL);
         uint32_t key = 0;
         if (KK == KK_RADIX) {
-          key = ONECH ? sel4(v4, kw) : lds_u32(t + koff);
+          key = OC == 2 ? sel4c<3>(v4) : ONECH ? sel4(v4, kw) : lds_u32(t + koff);
           if (key >= dom) {
             if (valid) err |= ERR_KEY;
             valid = false;
@@ -646,7 +660,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
           double fv[NF];
 #pragma unroll
           for (int f = 0; f < NF; ++f)                                   // NF == nf
-            fv[f] = (double)__uint_as_float(ONECH ? sel4(v4, fw[f]) : lds_u32(t + foff[f]));
+            fv[f] = (double)__uint_as_float(OC == 2 ? sel4c<2>(v4) : ONECH ? sel4(v4, fw[f]) : lds_u32(t + foff[f]));
 #if SB_P1_MATCH
           // warp-private DIRECT table: a lane whose entry no other lane of this
           // iteration touches updates it with plain loads/stores (no CAS loop)
@@ -736,14 +750,21 @@ static bool one_chunk(const Plan &p) {
     if ((p.field[f].word >> 2) != ch) return false;
   return true;
 }
-template <int M, bool OC>
+template <int M, int OC>
 static void *p1_cnt_nf2(const Plan &p, int kk) {
   if (kk == KK_GLOBAL) return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_GLOBAL, OC> : (void *)k_pane_cnt<M, 2, KK_GLOBAL, OC>;
   return p.nf <= 1 ? (void *)k_pane_cnt<M, 1, KK_RADIX, OC> : (void *)k_pane_cnt<M, 2, KK_RADIX, OC>;
 }
+// τ in words 0-1, one value in word 2, the key (if any) in word 3 of one chunk
+static bool syn_layout(const Plan &p, int kk) {
+  return one_chunk(p) && (p.ts_word & 3) == 0 && p.nf == 1 && (p.field[0].word & 3) == 2 &&
+         (kk == KK_GLOBAL || (p.key[0].word & 3) == 3) && !std::getenv("SABER_NO_FIXED_LAYOUT");
+}
 template <int M>
 static void *p1_cnt_nf(const Plan &p, int kk) {
-  return one_chunk(p) ? p1_cnt_nf2<M, true>(p, kk) : p1_cnt_nf2<M, false>(p, kk);
+  if (syn_layout(p, kk))
+    return kk == KK_GLOBAL ? (void *)k_pane_cnt<M, 1, KK_GLOBAL, 2> : (void *)k_pane_cnt<M, 1, KK_RADIX, 2>;
+  return one_chunk(p) ? p1_cnt_nf2<M, 1>(p, kk) : p1_cnt_nf2<M, 0>(p, kk);
 }
 // count-window fast kernel, or nullptr when the plan needs the generic one
 static void *p1_cnt(const Plan &p) {
