@@ -209,7 +209,9 @@ __device__ __forceinline__ void flush_tables(const Plan &p, State *st, uint64_t 
   __syncthreads();
 }
 
-template <int MODE, int WK, int NF, bool FAST>
+// NK >= 0 (FAST plans): exactly NK radix-packed int32 key columns, known at
+// compile time (no per-tuple loop bounds and plan-field branches); -1: run time
+template <int MODE, int WK, int NF, bool FAST, int NK = -1>
 __global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? SB_P1_DIRECT_BPS : 2)
 k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
            uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
@@ -376,14 +378,14 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
         uint64_t fv[NF];
         if (FAST) {
           // all fields are fp64 sums of f32 columns; at most one int32 key column, div 1
-          if (p.key_mode == KM_GLOBAL) key = 0;
-          else if (p.key_pack == KP_RADIX) {
+          if (NK == 0 || (NK < 0 && p.key_mode == KM_GLOBAL)) key = 0;
+          else if (NK > 0 || p.key_pack == KP_RADIX) {
             // radix-packed int32 key columns, each col / div (C truncation, A17)
             uint64_t kk = 0;
             bool bad = false;
 #pragma unroll
-            for (int kc = 0; kc < kMaxKey; ++kc) {
-              if (kc < p.nkeys) {
+            for (int kc = 0; kc < (NK > 0 ? NK : kMaxKey); ++kc) {
+              if (NK > 0 || kc < p.nkeys) {
                 int32_t v = *(const int32_t *)(t + 4 * p.key[kc].word);
                 if (p.key[kc].div != 1) v = div_trunc32(v, p.key[kc].div, p.key[kc].inv);
                 bad |= (uint32_t)v >= (uint32_t)p.key[kc].domain;     // domain < 2^31 on the fast path
@@ -718,9 +720,26 @@ int p1_smem_bytes(const Plan &p) {
   return kStages * kStageBytes + 2 * kStages * 8 + (p.local_mode == TM_SHARED ? 1 : kP1Warps) * p.local_bytes;
 }
 
+template <int M, int WK, int NK>
+static void *p1_fast_nk(int nf) {
+  return nf <= 1 ? (void *)k_pane_agg<M, WK, 1, true, NK> : (void *)k_pane_agg<M, WK, 2, true, NK>;
+}
+// compile-time key count for FAST time-window plans with dense/global tables
 template <int M, int WK>
-static void *p1_nf(int nf, bool fast) {
-  if (fast) return nf <= 1 ? (void *)k_pane_agg<M, WK, 1, true> : (void *)k_pane_agg<M, WK, 2, true>;
+static void *p1_fast(const Plan &p) {
+  if (WK == WK_TIME && M != TM_HASHED && !std::getenv("SABER_NO_NK")) {
+    if (p.key_mode == KM_GLOBAL) return p1_fast_nk<M, WK, 0>(p.nf);
+    if (p.key_pack == KP_RADIX && p.key_mode != KM_HASH) {
+      if (p.nkeys == 1) return p1_fast_nk<M, WK, 1>(p.nf);
+      if (p.nkeys == 2) return p1_fast_nk<M, WK, 2>(p.nf);
+      if (p.nkeys == 3) return p1_fast_nk<M, WK, 3>(p.nf);
+    }
+  }
+  return p1_fast_nk<M, WK, -1>(p.nf);
+}
+template <int M, int WK>
+static void *p1_nf(const Plan &p, int nf, bool fast) {
+  if (fast) return p1_fast<M, WK>(p);
   switch (p1_nf_template(nf)) {
     case 1: return (void *)k_pane_agg<M, WK, 1, false>;
     case 2: return (void *)k_pane_agg<M, WK, 2, false>;
@@ -732,10 +751,10 @@ template <int WK>
 static void *p1_mode(const Plan &p) {
   const bool f = p.fast_keys;
   switch (p.local_mode) {
-    case TM_LANE: return p1_nf<TM_LANE, WK>(p.nf, f);
-    case TM_DIRECT: return p1_nf<TM_DIRECT, WK>(p.nf, f);
-    case TM_SHARED: return p1_nf<TM_SHARED, WK>(p.nf, f);
-    default: return p1_nf<TM_HASHED, WK>(p.nf, f);
+    case TM_LANE: return p1_nf<TM_LANE, WK>(p, p.nf, f);
+    case TM_DIRECT: return p1_nf<TM_DIRECT, WK>(p, p.nf, f);
+    case TM_SHARED: return p1_nf<TM_SHARED, WK>(p, p.nf, f);
+    default: return p1_nf<TM_HASHED, WK>(p, p.nf, f);
   }
 }
 static void *p1_generic(const Plan &p) {
