@@ -294,20 +294,82 @@ k_vh_build_cta(const Plan p, const State *__restrict__ st, const uint64_t *__res
 // directions over the whole pane range of the task).
 constexpr int kVhU = 8;
 
+// combine with the field kind fixed at compile time (OP >= 0) or per lane (OP < 0)
+template <int OP>
+__device__ __forceinline__ uint64_t vh_comb(int op, uint64_t a, uint64_t b) {
+  if (OP == FK_SUM_I) return a + b;
+  if (OP == FK_SUM_F) return (uint64_t)__double_as_longlong(__longlong_as_double((long long)a) + __longlong_as_double((long long)b));
+  if (OP == FK_MIN) return a < b ? a : b;
+  if (OP == FK_MAX) return a < b ? b : a;
+  return field_combine_sel(op, a, b);
+}
+
+// one (block, direction, 32-word group) item: walk `len` panes from `start`
+// (forward for prefixes, backward for suffixes) in tiles of 8 warps × kVhU panes
+template <int OP>
+__device__ __forceinline__ void vh_tile_walk(uint64_t (*s_tot)[32], const uint64_t *__restrict__ table,
+                                             uint64_t *__restrict__ dst, int64_t start, int64_t len, bool prefix,
+                                             int64_t Rm, int64_t words, int64_t w, bool live, int op,
+                                             uint64_t id, uint64_t carry) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  auto slot = [&](int64_t k) { return ((prefix ? start + k : start - k) & Rm) * words + w; };
+  uint64_t v[kVhU], vn[kVhU];
+  auto load = [&](int64_t k0, uint64_t (&x)[kVhU]) {
+#pragma unroll
+    for (int u = 0; u < kVhU; ++u) {
+      const int64_t k = k0 + warp * kVhU + u;
+      x[u] = (live && k < len) ? table[slot(k)] : id;
+    }
+  };
+  load(0, vn);
+  for (int64_t k0 = 0; k0 < len; k0 += 8 * kVhU) {
+#pragma unroll
+    for (int u = 0; u < kVhU; ++u) v[u] = vn[u];
+    if (k0 + 8 * kVhU < len) load(k0 + 8 * kVhU, vn);
+    uint64_t acc = id;
+#pragma unroll
+    for (int u = 0; u < kVhU; ++u) {
+      acc = vh_comb<OP>(op, acc, v[u]);
+      v[u] = acc;
+    }
+    s_tot[warp][lane] = acc;
+    __syncthreads();
+    uint64_t run = carry, all = carry;
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const uint64_t x = s_tot[c][lane];
+      if (c < warp) run = vh_comb<OP>(op, run, x);
+      all = vh_comb<OP>(op, all, x);
+    }
+    carry = all;
+    if (live) {
+#pragma unroll
+      for (int u = 0; u < kVhU; ++u) {
+        const int64_t k = k0 + warp * kVhU + u;
+        if (k < len) dst[slot(k)] = vh_comb<OP>(op, run, v[u]);
+      }
+    }
+    __syncthreads();
+  }
+}
+
 __global__ void __launch_bounds__(256, 3)
 k_vh_build_tile(const Plan p, const State *__restrict__ st, const uint64_t *__restrict__ table,
                 uint64_t *__restrict__ pre, uint64_t *__restrict__ suf) {
   __shared__ uint64_t s_tot[8][32];
   const int64_t J0 = st->J0, J1 = st->J1;
   if (J1 <= J0) return;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
   const int64_t K = p.K, Rm = p.R - 1, words = p.slot_words, groups = (words + 31) / 32;
-  const int64_t a0 = J0 * p.L, a1 = (J1 - 1) * p.L, e0 = a0 + K - 1, e1 = a1 + K - 1;
+  const int64_t a0 = J0 * p.L, a1 = (J1 - 1) * p.L, e1 = a1 + K - 1;
   const int64_t sb0 = a0 / K, nS = a1 / K - sb0 + 1;             // suffix blocks
   const int64_t pb0 = a0 / K + 1, nP = e1 / K >= pb0 ? e1 / K - pb0 + 1 : 0;   // prefix blocks (start > a0)
   const int64_t pdone = st->vh_pre_hi;
   const int64_t items = (nS + nP) * groups;
-  (void)e0;
+  auto op_of = [&](int64_t w) {                                   // count words add as integers
+    const int f = (int)(w / p.C) - 1;
+    return f < 0 ? (int)FK_SUM_I : p.field[f].kind;
+  };
   for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
     const int64_t grp = it % groups, seg = it / groups;
     const bool prefix = seg >= nS;
@@ -325,50 +387,21 @@ k_vh_build_tile(const Plan p, const State *__restrict__ st, const uint64_t *__re
     if (len <= 0) continue;                                       // uniform across the CTA
     const int64_t w = grp * 32 + lane;
     const bool live = w < words;
-    const int f = live ? (int)(w / p.C) - 1 : -1;
-    const int op = f < 0 ? FK_SUM_I : p.field[f].kind;             // count words add as integers
+    const int op = live ? op_of(w) : FK_SUM_I;
     const uint64_t id = field_identity(op);
     uint64_t carry = id;
     if (prefix && start > bs && live) carry = pre[((start - 1) & Rm) * words + w];
     uint64_t *dst = prefix ? pre : suf;
-    auto pane_of = [&](int64_t k) { return prefix ? start + k : start - k; };
-    uint64_t v[kVhU], vn[kVhU];
-    auto load = [&](int64_t k0, uint64_t (&x)[kVhU]) {
-#pragma unroll
-      for (int u = 0; u < kVhU; ++u) {
-        const int64_t k = k0 + warp * kVhU + u;
-        x[u] = (live && k < len) ? table[(pane_of(k) & Rm) * words + w] : id;
-      }
-    };
-    load(0, vn);
-    for (int64_t k0 = 0; k0 < len; k0 += 8 * kVhU) {
-#pragma unroll
-      for (int u = 0; u < kVhU; ++u) v[u] = vn[u];
-      if (k0 + 8 * kVhU < len) load(k0 + 8 * kVhU, vn);
-      uint64_t acc = id;
-#pragma unroll
-      for (int u = 0; u < kVhU; ++u) {
-        acc = field_combine_sel(op, acc, v[u]);
-        v[u] = acc;
-      }
-      s_tot[warp][lane] = acc;
-      __syncthreads();
-      uint64_t run = carry, all = carry;
-#pragma unroll
-      for (int c = 0; c < 8; ++c) {
-        const uint64_t x = s_tot[c][lane];
-        if (c < warp) run = field_combine_sel(op, run, x);
-        all = field_combine_sel(op, all, x);
-      }
-      carry = all;
-      if (live) {
-#pragma unroll
-        for (int u = 0; u < kVhU; ++u) {
-          const int64_t k = k0 + warp * kVhU + u;
-          if (k < len) dst[(pane_of(k) & Rm) * words + w] = field_combine_sel(op, run, v[u]);
-        }
-      }
-      __syncthreads();
+    // the group's 32 words usually lie in one section (count or one field): the
+    // combine is then fixed for the whole walk
+    const int64_t wl = grp * 32, wh = (wl + 31 < words ? wl + 31 : words - 1);
+    const int uop = op_of(wl) == op_of(wh) ? op_of(wl) : -1;
+    switch (uop) {
+      case FK_SUM_I: vh_tile_walk<FK_SUM_I>(s_tot, table, dst, start, len, prefix, Rm, words, w, live, op, id, carry); break;
+      case FK_SUM_F: vh_tile_walk<FK_SUM_F>(s_tot, table, dst, start, len, prefix, Rm, words, w, live, op, id, carry); break;
+      case FK_MIN: vh_tile_walk<FK_MIN>(s_tot, table, dst, start, len, prefix, Rm, words, w, live, op, id, carry); break;
+      case FK_MAX: vh_tile_walk<FK_MAX>(s_tot, table, dst, start, len, prefix, Rm, words, w, live, op, id, carry); break;
+      default: vh_tile_walk<-1>(s_tot, table, dst, start, len, prefix, Rm, words, w, live, op, id, carry);
     }
   }
 }
