@@ -115,18 +115,43 @@ class Clocks:
         self.index, self.path = index, path
         self.rows, self.timed, self._stop = [], False, False
         self.thread = None
+        self.error = None
 
     def _run(self):
         import pynvml
-        pynvml.nvmlInit()
-        h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
-        mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
-        while not self._stop:
-            sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
-            rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
-            self.rows.append((time.perf_counter(), self.timed, sm, mx, int(rs)))
-            time.sleep(0.002)
-        pynvml.nvmlShutdown()
+        for attempt in range(20):                   # NVML init can fail transiently right after another process
+            try:
+                pynvml.nvmlInit()
+                break
+            except Exception as e:                  # noqa: BLE001
+                self.error = f"nvmlInit: {e}"
+                time.sleep(0.05)
+        else:
+            return
+        try:
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            reasons = getattr(pynvml, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                pynvml.nvmlDeviceGetCurrentClocksThrottleReasons
+            while not self._stop:
+                sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                rs = reasons(h)
+                self.rows.append((time.perf_counter(), self.timed, sm, mx, int(rs)))
+                time.sleep(0.002)
+        except Exception as e:                      # noqa: BLE001
+            self.error = f"nvml: {e}"
+        finally:
+            pynvml.nvmlShutdown()
+
+    def smi_once(self):
+        """Fallback when NVML sampling produced nothing: one nvidia-smi reading."""
+        try:
+            out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,"
+                                  "clocks_event_reasons.active", "--format=csv,noheader,nounits"],
+                                 capture_output=True, text=True, timeout=20).stdout.strip().split(",")
+            return int(out[0]), int(out[1]), int(out[2].strip(), 16)
+        except Exception:                           # noqa: BLE001
+            return None
 
     def __enter__(self):
         try:
@@ -155,10 +180,15 @@ class Clocks:
         if not rows:
             rows, where = self.rows, "whole run (no sample fell inside a timed step)"
         if not rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+            one = self.smi_once()
+            if one is None:
+                return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0,
+                        "error": self.error}
+            rows, where = [(0.0, False, one[0], one[1], one[2])], "after the timed region (nvidia-smi, NVML failed)"
         reasons = sorted({n for r in rows for n, bit in self.REASONS.items() if r[4] & bit})
         return {"sm_mhz": statistics.median(r[2] for r in rows), "sm_max_mhz": max(r[3] for r in rows),
-                "reasons": reasons, "samples": len(rows), "sampled": where, "source": "NVML, ~2 ms poll"}
+                "reasons": reasons, "samples": len(rows), "sampled": where,
+                "source": "nvidia-smi" if where.startswith("after") else "NVML, ~2 ms poll"}
 
 
 def measured_peaks():
