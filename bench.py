@@ -473,24 +473,35 @@ def main():
                 chunks.append(halo_np)
             chunks.append(host_np)
             per = e2e_task * 7
+
+            def take():
+                """Next result slice through the C ABI: poll returns once the slice's
+                headers and rows are in the query's pinned host mirror (the D2H read
+                of the result); count its bytes and hand the slot back."""
+                st, r = q.poll_raw(-1)
+                if st != 0:
+                    raise saber.SaberError(st, q.last_error())
+                nb = r.nrows * sum(r.col_bytes[c] for c in range(r.ncols)) + r.ntuples * r.tuple_bytes + \
+                    (r.nwindows * 32 if r.hdr else 0)
+                q.release(r)
+                return nb
             for arr in chunks:
                 off = 0
                 while off < arr.size:
                     part_np = arr[off:off + per]
                     st = q.submit(part_np)
                     if st == saber.EAGAIN:
-                        s = q.poll()
-                        got_bytes += sum(k.nbytes for k in s.keys) + sum(v.nbytes for v in s.vals) + \
-                            len(s.tuples) + s.nwindows * 32
+                        got_bytes += take()
                         continue
                     if st != 0:
                         raise saber.SaberError(st, q.last_error())
                     off += part_np.size
             while (st := q.finish()) == saber.EAGAIN:
-                s = q.poll()
-                got_bytes += sum(k.nbytes for k in s.keys) + sum(v.nbytes for v in s.vals) + len(s.tuples) + s.nwindows * 32
-            while (s := q.poll()) is not None:
-                got_bytes += sum(k.nbytes for k in s.keys) + sum(v.nbytes for v in s.vals) + len(s.tuples) + s.nwindows * 32
+                got_bytes += take()
+            if st != 0:
+                raise saber.SaberError(st, q.last_error())
+            while q.stats()["tasks_pending"] > 0:
+                got_bytes += take()
             torch.cuda.synchronize()
             dt = time.perf_counter() - t0
             if it >= args.warmup:
