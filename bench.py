@@ -384,6 +384,9 @@ def main():
                     emit_on_finish=(rank == world - 1), task_bytes=task_bytes,
                     result_mode=saber.RESULTS_DEVICE, profile=True, result_slots=8, device=local)
     with Clocks(local, os.path.join(clk_dir, f"clocks_rank{rank}.csv")) as clk:
+        t_wait = time.perf_counter()                 # NVML initialised and sampling before timing
+        while clk.thread is not None and not clk.rows and time.perf_counter() - t_wait < 5.0:
+            time.sleep(0.01)
         for it in range(args.warmup + args.steps):
             q.reset(base_index, first_window)
             barrier()
