@@ -541,7 +541,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   static_assert(OC != 2 || NF == 1, "fixed layout: one value column");
   extern __shared__ __align__(128) unsigned char smem[];
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const int tb = p.tuple_bytes;
+  const int tb = OC == 2 ? 32 : p.tuple_bytes;                 // the fixed layout is the 32-B Syn tuple
   const int ST = kStageBytes / tb;
   unsigned char *stages = smem;
   uint64_t *full = (uint64_t *)(smem + kStages * kStageBytes);
@@ -776,7 +776,7 @@ static void *p1_cnt_nf2(const Plan &p, int kk) {
 }
 // τ in words 0-1, one value in word 2, the key (if any) in word 3 of one chunk
 static bool syn_layout(const Plan &p, int kk) {
-  return one_chunk(p) && (p.ts_word & 3) == 0 && p.nf == 1 && (p.field[0].word & 3) == 2 &&
+  return one_chunk(p) && p.tuple_bytes == 32 && (p.ts_word & 3) == 0 && p.nf == 1 && (p.field[0].word & 3) == 2 &&
          (kk == KK_GLOBAL || (p.key[0].word & 3) == 3) && !std::getenv("SABER_NO_FIXED_LAYOUT");
 }
 template <int M>
