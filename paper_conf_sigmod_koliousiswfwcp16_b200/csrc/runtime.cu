@@ -461,7 +461,8 @@ static saber_status size_plan(saber_query *q) {
     }
     // dense / global count-window plans overlap the window phase of a task with the
     // next task's scan (Plan::overlap): the ring then holds two tasks' panes
-    if (!p.bucket_mode && !p.slab_mode && p.key_mode != KM_HASH && p.win_kind == WK_COUNT && c.max_panes <= 0) {
+    if (!p.bucket_mode && !p.slab_mode && p.key_mode != KM_HASH && p.win_kind == WK_COUNT && c.max_panes <= 0 &&
+        getenv_flag("SABER_OVERLAP")) {
       const int64_t R2 = next_pow2(2 * ((T + p.g - 1) / p.g + 2) + p.K + p.L + 2);
       if (R2 > p.R && R2 * slot_bytes <= (1ll << 30)) p.R = R2;
     }
