@@ -153,6 +153,33 @@ __device__ __forceinline__ int64_t global_insert(const Plan &p, State *st, uint6
 }
 
 
+// Compensated fp64 accumulation for window states that slide by adding entering
+// and subtracting expiring values (bucket / hash / slab plans).  Plain fp64
+// add/subtract leaves an error proportional to everything the state ever held
+// (a key that once summed 1e12 and now sums 1e-3 would be off by ~1e-4); with
+// Knuth's error-free TwoSum the rounding error of every update is kept in a
+// second word, so the state's error is ~2^-106 of its history.
+// No multiplications: nothing for FMA contraction to change.
+__device__ __forceinline__ double two_sum(double a, double b, double &e) {
+  const double s = a + b;
+  const double bb = s - a;
+  e = (a - (s - bb)) + (b - bb);
+  return s;
+}
+// shared-memory version for concurrent updates: CAS on the sum word, the
+// (exact) rounding error of the successful update goes to the compensation word
+__device__ __forceinline__ void dd_atomic_add(double *hi, double *lo, double x) {
+  unsigned long long *a = (unsigned long long *)hi;
+  unsigned long long old = *(volatile unsigned long long *)a, assumed;
+  double s, e;
+  do {
+    assumed = old;
+    s = two_sum(__longlong_as_double((long long)assumed), x, e);
+    old = atomicCAS(a, assumed, (unsigned long long)__double_as_longlong(s));
+  } while (old != assumed);
+  if (e != 0.0) atomicAdd(lo, e);
+}
+
 // decoupled look-back status words: epoch (24 bits) | flag (2: 1 aggregate, 2 inclusive) | value (38 bits)
 __device__ __forceinline__ uint64_t lb_ld(const uint64_t *p) {
   uint64_t v;

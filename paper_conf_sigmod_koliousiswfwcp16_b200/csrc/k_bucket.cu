@@ -20,9 +20,10 @@
 //                    ranges and write the rows of present keys coalesced
 //                    (ballot/popc positions, per-warp-range counts tracked
 //                    incrementally, so no block-wide scan per window).
-// Float sums are added and subtracted in fp64 (reading A12: the tolerance is
-// relative to the sum of |x|, which bounds the cancellation error); a key whose
-// count returns to 0 has its sum reset to exactly 0.
+// Float sums are added and subtracted in compensated fp64 (sum + TwoSum error
+// word, common.cuh dd_atomic_add): the state's error does not grow with the
+// magnitude of values that already left the window; a key whose count returns to
+// 0 has both words reset to exactly 0.
 #include <cuda_runtime.h>
 #include <climits>
 #include <stdint.h>
@@ -361,7 +362,8 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
   __shared__ int wn[32];
   const int S = p.S, SB = 1 << p.bk_shift, W = p.bk_W, g = (int)p.g;
   double *sum = (double *)smem;                               // [NF][SB]
-  uint32_t *cnt = (uint32_t *)(smem + (size_t)8 * NF * SB);    // [SB]
+  double *cmp = sum + (size_t)NF * SB;                        // [NF][SB] TwoSum compensation
+  uint32_t *cnt = (uint32_t *)(smem + (size_t)16 * NF * SB);   // [SB]
   uint16_t *slist = (uint16_t *)(cnt + SB);                   // [SB]: per-warp lists of present slots
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
   if (nw <= 0) return;
@@ -385,7 +387,7 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
       if (atomicSub(&cnt[k], 1u) == 1u) atomicSub(&wn[k >> rs_shift], 1);
     }
 #pragma unroll
-    for (int f = 0; f < NF; ++f) atomicAdd(&sum[f * SB + k], add ? (double)v.v[f] : -(double)v.v[f]);
+    for (int f = 0; f < NF; ++f) dd_atomic_add(&sum[f * SB + k], &cmp[f * SB + k], add ? (double)v.v[f] : -(double)v.v[f]);
   };
   for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
     const int64_t chunk = item / S;
@@ -396,7 +398,7 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
     for (int i = tid; i < SB; i += nt) {
       cnt[i] = 0;
 #pragma unroll
-      for (int f = 0; f < NF; ++f) sum[f * SB + i] = 0.0;
+      for (int f = 0; f < NF; ++f) sum[f * SB + i] = cmp[f * SB + i] = 0.0;
     }
     if (tid < 32) wn[tid] = 0;
     __syncthreads();
@@ -415,7 +417,7 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
         const uint32_t k = __ldg(kp + e);
         if (cnt[k] == 0u)
 #pragma unroll
-          for (int f = 0; f < NF; ++f) sum[f * SB + k] = 0.0;
+          for (int f = 0; f < NF; ++f) sum[f * SB + k] = cmp[f * SB + k] = 0.0;
       }
     };
     auto pane_b = [&](int64_t q) { return (q & Rm) * S + s; };
@@ -488,7 +490,7 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
           kcol[i] = kb + sl;
           double sv[NF > 0 ? NF : 1];
 #pragma unroll
-          for (int f = 0; f < NF; ++f) sv[f] = sum[f * SB + wid * RS + sl];
+          for (int f = 0; f < NF; ++f) sv[f] = sum[f * SB + wid * RS + sl] + cmp[f * SB + wid * RS + sl];
           const double dc = (double)c;
 #pragma unroll
           for (int a = 0; a < NA; ++a) {
@@ -528,7 +530,7 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
           const int e = tid + u * nt;
           if (e < A.nl && cnt[A.kl[u]] == 0u)
 #pragma unroll
-            for (int f = 0; f < NF; ++f) sum[f * SB + A.kl[u]] = 0.0;
+            for (int f = 0; f < NF; ++f) sum[f * SB + A.kl[u]] = cmp[f * SB + A.kl[u]] = 0.0;
         }
         zero_fix(A.bl, kEmitPF * nt, A.nl);
         A = B;
@@ -542,7 +544,7 @@ k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long 
 // ---------------------------------------------------------------------------
 // host side
 int bk_scan_smem() { return kBkStages * kBkStageBytes + 2 * kBkStages * 8 + 2 * kBkHist * 4; }
-int bk_emit_smem(const Plan &p) { return (1 << p.bk_shift) * (6 + 8 * p.nf); }
+int bk_emit_smem(const Plan &p) { return (1 << p.bk_shift) * (6 + 16 * p.nf); }
 int bk_count_smem(const Plan &p) { return (1 << p.bk_shift) * 4; }
 
 static void *bk_scan_kernel(const Plan &p) {

@@ -38,9 +38,11 @@ __device__ __forceinline__ double sel_s_flt(const unsigned char *t, int word, in
 __global__ void __launch_bounds__(kSelThreads, 2)
 k_select(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ task,
          const unsigned char *__restrict__ carry0, const unsigned char *__restrict__ carry1,
-         unsigned char *__restrict__ stage_rows, int64_t *__restrict__ cta_cnt) {
+         unsigned char *__restrict__ stage_rows, int64_t *__restrict__ cta_cnt,
+         int64_t *__restrict__ ihdr, int64_t *__restrict__ win_ts, int64_t ts_mask) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_cnt[kSelMaxIter][kSelWarps];
+  __shared__ unsigned s_bal[kSelMaxIter][kSelWarps];
   __shared__ int s_off[kSelMaxIter][kSelWarps];
   __shared__ int s_total;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -52,6 +54,7 @@ k_select(const Plan p, State *__restrict__ st, const unsigned char *__restrict__
   uint64_t *empty = full + kSelStages;
   const int64_t cl = st->cover_lo, ch = st->cover_hi;
   const int64_t tpos = st->task_pos, cpos = st->carry_pos;
+  const int64_t J0 = st->J0, J1 = st->J1;
   const unsigned char *carry = st->carry_sel ? carry1 : carry0;
   // contiguous, stage-aligned range of this CTA within [cover_lo, cover_hi)
   const int64_t n = ch - cl;
@@ -117,8 +120,9 @@ k_select(const Plan p, State *__restrict__ st, const unsigned char *__restrict__
         }
       }
       bal[j] = __ballot_sync(kFull, s);
-      if (lane == 0) s_cnt[j][wid] = __popc(bal[j]);
+      if (lane == 0) { s_cnt[j][wid] = __popc(bal[j]); s_bal[j][wid] = bal[j]; }
     }
+    const int64_t prev_tau_stage = prev_tau;
     prev_tau = *(const int64_t *)(sb + (ns - 1) * tb + 4 * p.ts_word);
     __syncthreads();
     if (wid == 0) {                                      // scan of the (j, warp) counts in stream order
@@ -138,6 +142,47 @@ k_select(const Plan p, State *__restrict__ st, const unsigned char *__restrict__
       if (lane == 0) s_total = run;
     }
     __syncthreads();
+    // window headers (reading A9: window j's rows are the selected tuples of
+    // W_j \ W_{j-1}, a position segment): record, for every window whose segment
+    // starts in this stage, the CTA-relative rank of its first row
+    const int64_t a0 = lo + (int64_t)k * ST;
+    auto rank_at = [&](int x) -> int64_t {        // selected tuples of the CTA before local index x
+      const int jx = x / kSelThreads, tx = x - jx * kSelThreads;
+      return written + s_off[jx][tx >> 5] + __popc(s_bal[jx][tx >> 5] & ((1u << (tx & 31)) - 1u));
+    };
+    const int64_t pack_cta = (int64_t)blockIdx.x << 44;
+    if (p.win_kind == WK_COUNT) {
+      const int64_t sl = p.l, ss = p.s;
+      // τ at window starts j·l inside the stage (header ts, reading A7)
+      for (int64_t jj = (a0 + sl - 1) / sl + tid; jj * sl < a0 + ns; jj += kSelThreads)
+        win_ts[jj & ts_mask] = *(const int64_t *)(sb + (jj * sl - a0) * tb + 4 * p.ts_word);
+      // segment starts: position 0 (window 0) and (j-1)·l + s (window j >= 1)
+      int64_t jf = a0 <= ss ? 1 : (a0 - ss + sl - 1) / sl + 1;
+      if (a0 == 0 && tid == 0 && J0 == 0) ihdr[0] = pack_cta | rank_at(0);
+      for (int64_t jj = jf + tid; (jj - 1) * sl + ss < a0 + ns; jj += kSelThreads)
+        if (jj >= J0 && jj < J1) ihdr[jj - J0] = pack_cta | rank_at((int)((jj - 1) * sl + ss - a0));
+    } else {
+      const int64_t sl = p.l, B0 = p.T0 + p.s;
+      auto seg = [&](int64_t tau) -> int64_t { return tau < B0 ? 0 : (tau - B0) / sl + 1; };
+      for (int x = tid; x < ns; x += kSelThreads) {
+        const int64_t pos = a0 + x;
+        const int64_t tau = *(const int64_t *)(sb + x * tb + 4 * p.ts_word);
+        int64_t jfrom;
+        if (pos == cl) jfrom = J0;
+        else {
+          const int64_t up = x > 0 ? *(const int64_t *)(sb + (x - 1) * tb + 4 * p.ts_word) : prev_tau_stage;
+          if (up == tau) continue;
+          jfrom = seg(up) + 1;
+        }
+        int64_t jto = seg(tau);
+        if (jto > J1 - 1) jto = J1 - 1;
+        if (jfrom < J0) jfrom = J0;
+        if (jfrom <= jto) {
+          const int64_t v = pack_cta | rank_at(x);
+          for (int64_t jj = jfrom; jj <= jto; ++jj) ihdr[jj - J0] = v;
+        }
+      }
+    }
     // π: projected words of the selected tuples, compacted in stream order
 #pragma unroll
     for (int j = 0; j < kSelMaxIter; ++j) {
@@ -163,14 +208,24 @@ k_select(const Plan p, State *__restrict__ st, const unsigned char *__restrict__
       issue(k + kSelStages);
     }
   }
-  if (tid == 0) cta_cnt[blockIdx.x] = written;
+  if (tid == 0) {
+    cta_cnt[blockIdx.x] = written;
+    // time windows whose segments are empty at the end of the cover start at
+    // the cover's end: they begin after every row of the last CTA
+    if (p.win_kind == WK_TIME && lo < hi && hi == ch) {
+      const int64_t sl = p.l, B0 = p.T0 + p.s;
+      const int64_t jfrom = (prev_tau < B0 ? 0 : (prev_tau - B0) / sl + 1) + 1;
+      for (int64_t jj = jfrom > J0 ? jfrom : J0; jj < J1; ++jj) ihdr[jj - J0] = ((int64_t)blockIdx.x << 44) | written;
+    }
+  }
   if (err) atomicOr(&st->error, err);
 }
 
 // move every CTA's staged rows to its exclusive offset in the result slot
 __global__ void __launch_bounds__(256)
 k_select_fix(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ stage_rows,
-             const int64_t *__restrict__ cta_cnt, int ncta, unsigned char *__restrict__ rows) {
+             const int64_t *__restrict__ cta_cnt, int ncta, unsigned char *__restrict__ rows,
+             int64_t *__restrict__ cta_base) {
   __shared__ int64_t s_part[8];
   __shared__ int64_t s_base;
   const int b = blockIdx.x;
@@ -191,6 +246,7 @@ k_select_fix(const Plan p, State *__restrict__ st, const unsigned char *__restri
     int64_t s = 0;
     for (int w = 0; w < 8; ++w) s += s_part[w];
     s_base = s;
+    cta_base[b] = s;
     if (b == ncta - 1) {
       st->sel_rows = s + cta_cnt[b];
       if (s + cta_cnt[b] > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
@@ -212,6 +268,33 @@ k_select_fix(const Plan p, State *__restrict__ st, const unsigned char *__restri
   }
 }
 
+// window headers of the task: row_offset of window j = global rank of its first
+// new tuple; nrows = next window's offset - own (the last: the task's total)
+__global__ void __launch_bounds__(256)
+k_sel_hdr(const Plan p, const State *__restrict__ st, const int64_t *__restrict__ ihdr,
+          const int64_t *__restrict__ cta_base, const int64_t *__restrict__ win_ts, int64_t ts_mask,
+          WinHdr *__restrict__ hdr) {
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  const bool empty = st->cover_hi <= st->cover_lo;
+  const int64_t total = empty ? 0 : st->sel_rows;
+  auto off = [&](int64_t i) -> int64_t {
+    if (empty || i >= nw) return total;
+    const int64_t v = ihdr[i];
+    return cta_base[v >> 44] + (v & ((1ll << 44) - 1));
+  };
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nw; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j = J0 + i;
+    const int64_t o = off(i);
+    WinHdr h;
+    h.window_id = j;
+    h.ts = p.win_kind == WK_TIME ? p.T0 + j * p.l : win_ts[j & ts_mask];
+    h.row_offset = o;
+    h.nrows = (int32_t)(off(i + 1) - o);
+    h.flags = 0;
+    hdr[i] = h;
+  }
+}
+
 void *sel_kernel(const Plan &p) { return (void *)k_select; }
 
 int sel_smem_bytes() { return kSelStages * kSelStageBytes + 2 * kSelStages * 8; }
@@ -219,10 +302,13 @@ int sel_smem_bytes() { return kSelStages * kSelStageBytes + 2 * kSelStages * 8; 
 cudaError_t launch_select(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int grid,
                           cudaStream_t st) {
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&tuples, (void *)&q.carry[0], (void *)&q.carry[1],
-                  (void *)&q.sel_stage, (void *)&q.cta_cnt};
+                  (void *)&q.sel_stage, (void *)&q.cta_cnt, (void *)&q.ihdr_tmp, (void *)&q.win_ts,
+                  (void *)&q.ts_mask};
   cudaError_t e = cudaLaunchKernel(sel_kernel(p), dim3(grid), dim3(kSelThreads), args, (size_t)sel_smem_bytes(), st);
   if (e) return e;
-  k_select_fix<<<grid, 256, 0, st>>>(p, q.st, q.sel_stage, q.cta_cnt, grid, s.rows);
+  k_select_fix<<<grid, 256, 0, st>>>(p, q.st, q.sel_stage, q.cta_cnt, grid, s.rows, q.cta_base);
+  if ((e = cudaGetLastError())) return e;
+  k_sel_hdr<<<148, 256, 0, st>>>(p, q.st, q.ihdr_tmp, q.cta_base, q.win_ts, q.ts_mask, (WinHdr *)s.hdr);
   return cudaGetLastError();
 }
 

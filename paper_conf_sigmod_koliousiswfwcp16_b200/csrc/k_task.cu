@@ -9,7 +9,8 @@ namespace sb {
 
 __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, int64_t n, int final_,
                              int has_wm, int64_t wm, int emit_on_finish, SlotMeta *meta,
-                             const unsigned char *carry0, const unsigned char *carry1, int *tile_ctr) {
+                             const unsigned char *carry0, const unsigned char *carry1, int *tile_ctr,
+                             int64_t *win_ts, int64_t ts_mask) {
   const int lane = threadIdx.x;
   __shared__ int64_t sh[8];
   if (lane == 0) {
@@ -98,6 +99,14 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
     } else {
       cover_hi = cover_lo;
     }
+  }
+  // IStream count windows: header ts = τ at position j·l (reading A7); k_select
+  // records it for covered positions, the first task also for the positions of
+  // its first windows before its cover (a partition's halo, first_window > 0)
+  if (p.win_kind == WK_COUNT && st->first_task && n > 0) {
+    const int64_t cend = cover_lo < pos0 + n ? cover_lo : pos0 + n;
+    for (int64_t jj = (pos0 + p.l - 1) / p.l + lane; jj * p.l < cend; jj += 32)
+      win_ts[jj & ts_mask] = tau_at(p, tup, jj * p.l - pos0);
   }
   if (lane == 0) {
     if (cover_hi < cover_lo) cover_hi = cover_lo;
@@ -345,7 +354,7 @@ namespace sb {
 cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
                               int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st) {
   k_task_begin<<<1, 32, 0, st>>>(p, q.st, (const unsigned char *)tuples, n, final_, has_wm, wm, emit_on_finish,
-                                 s.meta, q.carry[0], q.carry[1], q.tile_ctr);
+                                 s.meta, q.carry[0], q.carry[1], q.tile_ctr, q.win_ts, q.ts_mask);
   return cudaGetLastError();
 }
 cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st) {

@@ -279,6 +279,9 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
         write_row(p, rows, base + s_roff[r * 8 + warp] + __popc(bal & lt), kv, c, fv);
       }
     }
+    // the van Herk pass wrote `raw` with generic stores; the next ticket's bulk
+    // copies (async proxy) overwrite it after the barrier
+    fence_proxy_async_smem();
     __syncthreads();
   }
 }

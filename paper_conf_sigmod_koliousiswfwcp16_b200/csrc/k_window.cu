@@ -795,6 +795,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
   uint64_t *skeys = (uint64_t *)smem;
   int64_t *scnt = (int64_t *)(skeys + ST);
   uint64_t *sf = (uint64_t *)(scnt + ST);
+  double *sc = (double *)(sf + (size_t)p.nf * ST);     // TwoSum compensation of FK_SUM_F fields
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
   if (nw <= 0) return;
   const int64_t maxprobe = (int64_t)st->max_probe;
@@ -811,7 +812,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
     for (int h = threadIdx.x; h < ST; h += blockDim.x) {
       skeys[h] = kEmpty;
       scnt[h] = 0;
-      FOR_F(f) sf[f * ST + h] = field_identity(p.field[f].kind);
+      FOR_F(f) { sf[f * ST + h] = field_identity(p.field[f].kind); sc[f * ST + h] = 0.0; }
     }
     __syncthreads();
     auto find = [&](uint64_t k) -> int {
@@ -846,7 +847,8 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
         FOR_F(f) {
           const int kind = p.field[f].kind;
           const uint64_t v = b[fld_off(p, f) + h];
-          if (!minmax && kind == FK_SUM_F) atomicAdd((double *)&sf[f * ST + s], sign * __longlong_as_double((long long)v));
+          if (!minmax && kind == FK_SUM_F)
+            dd_atomic_add((double *)&sf[f * ST + s], &sc[f * ST + s], sign * __longlong_as_double((long long)v));
           else if (!minmax && kind == FK_SUM_I) atomicAdd((unsigned long long *)&sf[f * ST + s], (unsigned long long)(sign * (int64_t)v));
           else if (minmax && kind == FK_MIN) atomicMin((unsigned long long *)&sf[f * ST + s], (unsigned long long)v);
           else if (minmax && kind == FK_MAX) atomicMax((unsigned long long *)&sf[f * ST + s], (unsigned long long)v);
@@ -863,7 +865,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
       for (int h = threadIdx.x; h < ST; h += blockDim.x)
         if (scnt[h] == 0)
           FOR_F(f)
-            if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) sf[f * ST + h] = 0;
+            if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) { sf[f * ST + h] = 0; sc[f * ST + h] = 0.0; }
       if (p.has_minmax) {
         for (int h = threadIdx.x; h < ST; h += blockDim.x)
           FOR_F(f)
@@ -876,7 +878,8 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
       uint64_t fv[kMaxField];
       for (int h = threadIdx.x; h < ST; h += blockDim.x) {
         if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
-        FOR_F(f) fv[f] = sf[f * ST + h];
+        FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
+            __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];
         if (having_ok(p, scnt[h], fv)) ++my;
       }
       int total;
@@ -888,7 +891,8 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
         int64_t r = counts[ci] + excl;
         for (int h = threadIdx.x; h < ST; h += blockDim.x) {
           if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
-          FOR_F(f) fv[f] = sf[f * ST + h];
+          FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
+            __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];
           if (!having_ok(p, scnt[h], fv)) continue;
           int64_t kv[kMaxKey];
           decode_key(p, skeys[h], kv);
@@ -1044,6 +1048,7 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
   const int S = p.S, SB = p.SB;
   int64_t *scnt = (int64_t *)smem;
   uint64_t *sf = (uint64_t *)(scnt + SB);
+  double *sc = (double *)(sf + (size_t)p.nf * SB);      // TwoSum compensation of FK_SUM_F fields
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
   if (nw <= 0) return;
   const int64_t cw = p.C * (1 + p.nf);
@@ -1058,7 +1063,7 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
     __syncthreads();
     for (int s = threadIdx.x; s < SB; s += blockDim.x) {
       scnt[s] = 0;
-      FOR_F(f) sf[f * SB + s] = field_identity(p.field[f].kind);
+      FOR_F(f) { sf[f * SB + s] = field_identity(p.field[f].kind); sc[f * SB + s] = 0.0; }
     }
     __syncthreads();
     // entries of one pane have distinct keys: plain read-modify-write, barrier per pane
@@ -1072,9 +1077,12 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
         FOR_F(f) {
           const int kind = p.field[f].kind;
           const uint64_t v = ck_fld(p, cl, f)[e];
-          if (!minmax && kind == FK_SUM_F)
-            sf[f * SB + s] = (uint64_t)__double_as_longlong(__longlong_as_double((long long)sf[f * SB + s]) +
-                                                           sign * __longlong_as_double((long long)v));
+          if (!minmax && kind == FK_SUM_F) {
+            double e;
+            sf[f * SB + s] = (uint64_t)__double_as_longlong(two_sum(__longlong_as_double((long long)sf[f * SB + s]),
+                                                                    sign * __longlong_as_double((long long)v), e));
+            sc[f * SB + s] += e;
+          }
           else if (!minmax && kind == FK_SUM_I) sf[f * SB + s] = (uint64_t)((int64_t)sf[f * SB + s] + sign * (int64_t)v);
           else if (minmax && (kind == FK_MIN || kind == FK_MAX)) sf[f * SB + s] = field_combine(kind, sf[f * SB + s], v);
         }
@@ -1090,7 +1098,7 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
       for (int s = threadIdx.x; s < SB; s += blockDim.x)
         if (scnt[s] == 0)
           FOR_F(f)
-            if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) sf[f * SB + s] = 0;
+            if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) { sf[f * SB + s] = 0; sc[f * SB + s] = 0.0; }
       if (p.has_minmax) {
         for (int s = threadIdx.x; s < SB; s += blockDim.x)
           FOR_F(f)
@@ -1104,7 +1112,8 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
       for (int s = threadIdx.x; s < SB; s += blockDim.x) {
         if (scnt[s] <= 0) continue;
         if (p.nhave) {
-          FOR_F(f) fv[f] = sf[f * SB + s];
+          FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
+              __longlong_as_double((long long)sf[f * SB + s]) + sc[f * SB + s]) : sf[f * SB + s];
           if (!having_ok(p, scnt[s], fv)) continue;
         }
         ++my;
@@ -1118,7 +1127,8 @@ k_win_slab(const Plan p, State *__restrict__ st, uint64_t *__restrict__ clist, c
         int64_t r = counts[ci] + excl;
         for (int s = threadIdx.x; s < SB; s += blockDim.x) {
           if (scnt[s] <= 0) continue;
-          FOR_F(f) fv[f] = sf[f * SB + s];
+          FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
+              __longlong_as_double((long long)sf[f * SB + s]) + sc[f * SB + s]) : sf[f * SB + s];
           if (p.nhave && !having_ok(p, scnt[s], fv)) continue;
           int64_t kv[kMaxKey];
           decode_key(p, (uint64_t)(kbase + (uint32_t)s), kv);

@@ -31,6 +31,13 @@ struct QueryDev {
   unsigned char *carry[2];  // IStream raw tail
   int64_t carry_cap;        // tuples
   int *tile_ctr;
+  // σ/π (IStream) window headers: per closed window the (CTA, CTA-relative row
+  // rank) of its first new tuple, each CTA's global row base, and τ at window
+  // starts j·l (count windows; ring of ts_mask+1 entries indexed by j)
+  int64_t *ihdr_tmp;
+  int64_t *cta_base;
+  int64_t *win_ts;
+  int64_t ts_mask;
   unsigned char *bkt;       // bucket mode: [R][S][g] u16 key offsets, then [R][S][nf][g] f32 values
 };
 

@@ -398,7 +398,7 @@ static saber_status size_plan(saber_query *q) {
       (void)gpb; (void)smem_budget;
     } else {
       p.GS = 256;
-      p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + p.nf)));
+      p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + 2 * p.nf)));   // keys, counts, fields, compensation
       const double A = (double)(p.K + q->win_chunk * p.L) / 2.0;
       const double B = p.key_pack == KP_RADIX ? (double)p.G / (double)p.C : 1e30;
       const double per_slot = std::max(1e-9, std::min(A, B));
@@ -406,18 +406,18 @@ static saber_status size_plan(saber_query *q) {
       if (sb > p.C) sb = p.C;
       p.SB = (int)sb;
       p.S = (int)(p.C / sb);
-      p.p2_smem = p.state_cap * 8 * (2 + p.nf);
+      p.p2_smem = p.state_cap * 8 * (2 + 2 * p.nf);
       // radix-packed keys with a declared domain: key-range slabs with a dense
       // shared-memory state (48 KiB) over compacted pane buckets
       if (p.key_pack == KP_RADIX && p.G < (1ll << 31)) {
-        const int64_t slab = floor_pow2((48 * 1024) / (8 * (1 + p.nf)));
+        const int64_t slab = floor_pow2((48 * 1024) / (8 * (1 + 2 * p.nf)));
         const int64_t S = (p.G + slab - 1) / slab;
         if (S <= 1024) {
           p.slab_mode = 1;
           q->win_chunk = 128;          // K-pane initialisation amortised over 128 windows
           p.SB = (int)slab;
           p.S = (int)S;
-          p.p2_smem = (int)(slab * 8 * (1 + p.nf));
+          p.p2_smem = (int)(slab * 8 * (1 + 2 * p.nf));
         }
       }
     }
@@ -434,7 +434,7 @@ static saber_status size_plan(saber_query *q) {
         p.g <= 65536 && !getenv_flag("SABER_NO_BUCKET")) {
       const char *sbe = std::getenv("SABER_BK_SB");      // tuning: max keys per slab
       int64_t sb = std::min<int64_t>(sbe ? std::max(256, std::atoi(sbe)) : 16384,
-                                     floor_pow2((224 * 1024) / (6 + 8 * p.nf)));
+                                     floor_pow2((224 * 1024) / (6 + 16 * p.nf)));   // + compensation words
       sb = std::min<int64_t>(sb, next_pow2(p.G));
       const int64_t S = (p.G + sb - 1) / sb;
       const int64_t st_max = 16384 / p.tuple_bytes;           // tuples per scan stage
@@ -534,6 +534,12 @@ static saber_status alloc_query(saber_query *q) {
     CK(cudaMalloc(&q->qd.carry[1], (size_t)p.carry_cap * p.tuple_bytes));
     CK(cudaMalloc(&q->qd.sel_stage, (size_t)p.rows_cap * p.out_row_words * 4 + 16));
     CK(cudaMalloc(&q->qd.cta_cnt, 8192 * sizeof(int64_t)));
+    CK(cudaMalloc(&q->qd.cta_base, 8192 * sizeof(int64_t)));
+    CK(cudaMalloc(&q->qd.ihdr_tmp, (size_t)(p.win_cap + 1) * sizeof(int64_t)));
+    // τ at window starts j·l: windows from J0 up to the cover's end (< win_cap + s/l + 2)
+    const int64_t nts = p.win_kind == WK_COUNT ? next_pow2(p.win_cap + p.s / p.l + 8) : 1;
+    q->qd.ts_mask = nts - 1;
+    CK(cudaMalloc(&q->qd.win_ts, (size_t)nts * sizeof(int64_t)));
   }
   const int nslots = q->cfg.result_slots > 0 ? q->cfg.result_slots : 8;
   q->slots.resize(nslots);
@@ -611,16 +617,31 @@ static saber_status check_sticky(saber_query *q) {
   return SABER_OK;
 }
 
-static int free_slots(saber_query *q) {
-  int n = 0;
-  for (auto &s : q->slots) n += s.state == SLOT_FREE;
-  return n;
+// the next n tasks take ring slots next_task .. next_task+n-1 (slot = task id mod
+// slots); slices may be released in any order, so every one of those slots must
+// be FREE before a submit consumes input (else EAGAIN without consuming)
+static bool ring_free(saber_query *q, int64_t n) {
+  const int64_t ns = (int64_t)q->slots.size();
+  if (n > ns) return false;
+  for (int64_t t = 0; t < n; ++t)
+    if (q->slots[(q->next_task + t) % ns].state != SLOT_FREE) return false;
+  return true;
 }
 
 // enqueue one task (device-resident tuples) on the compute stream
 static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuples, int final_, int has_wm, int64_t wm) {
   Slot &s = q->slots[q->next_task % (int64_t)q->slots.size()];
   if (s.state != SLOT_FREE) return fail(q, SABER_EAGAIN, "no free result slot");
+  // look-back status words carry 24 bits of the task epoch (common.cuh lb_pack):
+  // when the field wraps, stale words of an older task could match, so they are
+  // cleared first (flag 0 = unpublished), after every earlier window phase
+  if (q->plan.nagg > 0 && ((q->epoch_base + q->next_task + 1) & 0xffffff) == 0) {
+    if (q->next_task >= 1) {
+      Slot &o = q->slots[(q->next_task - 1) % (int64_t)q->slots.size()];
+      CK(cudaStreamWaitEvent(q->cs, o.done, 0));
+    }
+    CK(cudaMemsetAsync(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8, q->cs));
+  }
   const bool lane = q->plan.lane_alt && q->use_lane;
   const Plan &p = lane ? q->plan_lane : q->plan;
   cudaError_t e;
@@ -742,7 +763,7 @@ void saber_query_destroy(saber_query *q) {
   for (auto &r : q->registered)
     if (std::find(q->prereg.begin(), q->prereg.end(), r.first) == q->prereg.end()) cudaHostUnregister(r.first);
   cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.vh_pre); cudaFree(q->qd.vh_suf);
-  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.bkt); cudaFree(q->qd.sel_stage); cudaFree(q->qd.cta_cnt); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
+  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.bkt); cudaFree(q->qd.sel_stage); cudaFree(q->qd.cta_cnt); cudaFree(q->qd.cta_base); cudaFree(q->qd.ihdr_tmp); cudaFree(q->qd.win_ts); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
   cudaFree(q->qd.carry[0]); cudaFree(q->qd.carry[1]); cudaFree(q->qd.tile_ctr); cudaFree(q->d_tmp);
   if (q->cs) cudaStreamDestroy(q->cs);
   if (q->h2d) cudaStreamDestroy(q->h2d);
@@ -765,7 +786,7 @@ saber_status saber_task_submit_device(saber_query *q, const void *dev_tuples, si
   if (((uintptr_t)dev_tuples) & 15) return fail(q, SABER_EINVAL, "device tuples must be 16-byte aligned");
   const int64_t ntasks = (n + q->task_tuples - 1) / q->task_tuples;
   if (ntasks > (int64_t)q->slots.size()) return fail(q, SABER_EINVAL, "submit at most result_slots * task_bytes per call");
-  if (ntasks > free_slots(q)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
+  if (!ring_free(q, ntasks)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
   CK(cudaSetDevice(q->device));
   cudaStream_t us = (cudaStream_t)cuda_stream;
   cudaEvent_t ev;
@@ -840,7 +861,7 @@ saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t n
   const int64_t whole = ((int64_t)nbytes + q->stage_fill) / tbytes;
   if (whole > (int64_t)q->slots.size())
     return fail(q, SABER_EINVAL, "submit at most result_slots * task_bytes per call");
-  if (whole > free_slots(q)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
+  if (!ring_free(q, whole)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
   const bool reg = is_registered(q, host_tuples, nbytes);
   const bool copyin = !reg || q->stage_fill > 0 || (int64_t)nbytes % tbytes != 0;
   if (saber_status s = ensure_stages(q, copyin)) return s;
@@ -905,7 +926,7 @@ saber_status saber_query_finish(saber_query *q, int64_t watermark) {
   if (q->closed) return fail(q, SABER_ECLOSED, "finish called twice");
   CK(cudaSetDevice(q->device));
   const int need = 1 + (q->stage_fill > 0);
-  if (free_slots(q) < need) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
+  if (!ring_free(q, need)) return fail(q, SABER_EAGAIN, "result slots busy: poll and release first");
   const int has_wm = watermark != INT64_MIN;
   if (q->stage_fill > 0) {
     Stage &g = q->stages[q->cur_stage];
@@ -981,12 +1002,16 @@ saber_status saber_results_poll(saber_query *q, saber_results *out, int32_t time
     for (int c = 0; c < p.ncols; ++c) out->cols[c] = rows + p.col_off[c];
   } else {
     out->tuple_bytes = p.out_row_words * 4;
-    if (host && s.meta.ntuples) {
-      CK(cudaMemcpyAsync(s.h_rows, s.dev.rows, (size_t)s.meta.ntuples * out->tuple_bytes, cudaMemcpyDeviceToHost, q->d2h));
+    if (host && (s.meta.ntuples || s.meta.nwindows)) {
+      if (s.meta.ntuples)
+        CK(cudaMemcpyAsync(s.h_rows, s.dev.rows, (size_t)s.meta.ntuples * out->tuple_bytes, cudaMemcpyDeviceToHost, q->d2h));
+      if (s.meta.nwindows)
+        CK(cudaMemcpyAsync(s.h_hdr, s.dev.hdr, (size_t)s.meta.nwindows * sizeof(saber_win_hdr), cudaMemcpyDeviceToHost, q->d2h));
       CK(cudaStreamSynchronize(q->d2h));
     }
     out->tuples = host ? (const void *)s.h_rows : (const void *)s.dev.rows;
-    out->hdr = nullptr;
+    // per-window headers: row_offset / nrows count projected tuples (reading A9)
+    out->hdr = host ? s.h_hdr : (const saber_win_hdr *)s.dev.hdr;
   }
   q->stats.windows += s.meta.nwindows;
   q->stats.rows += s.meta.nrows;

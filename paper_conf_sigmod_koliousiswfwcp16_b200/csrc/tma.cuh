@@ -24,6 +24,12 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase) {
       "r"(phase)
       : "memory");
 }
+// order this thread's generic-proxy shared-memory writes before later
+// async-proxy (TMA) accesses of the same bytes (PTX memory model: a bulk copy
+// into shared memory that earlier generic stores wrote needs this fence)
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
 // 1-D TMA bulk copy global → shared, completion counted on `bar` (SASS: UBLKCP)
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(

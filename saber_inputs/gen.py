@@ -154,3 +154,26 @@ def column(data: bytes | np.ndarray, kind_or_schema, name: str) -> np.ndarray:
             w = np.dtype(dt).itemsize
             return np.ascontiguousarray(arr[:, off:off + w]).view(dt).reshape(-1)
     raise KeyError(name)
+
+
+def wide_f32(seed: int, i0: int, n: int, lo_exp: float = -6.0, hi_exp: float = 12.0) -> np.ndarray:
+    """Non-negative, non-dyadic f32 values spanning 10^lo_exp .. 10^hi_exp
+    (log-uniform, counter-based): the float-robustness stream of DESIGN.md §4.
+    fp64 sums of these are NOT exact, unlike u24 data."""
+    i = np.arange(i0, i0 + n, dtype=np.uint64)
+    u = u24_f64(r(seed, i, 13)) + u24_f64(r(seed, i, 14)) * 2.0 ** -24
+    return (10.0 ** (lo_exp + (hi_exp - lo_exp) * u)).astype(np.float32)
+
+
+def with_column(data: bytes, kind: str, name: str, values: np.ndarray) -> bytes:
+    """Return ``data`` with column ``name`` replaced by ``values`` (test inputs)."""
+    sch = SCHEMAS[kind]
+    tb = sch["tuple_bytes"]
+    arr = np.frombuffer(data, dtype=np.uint8).reshape(-1, tb).copy()
+    for cname, ctype, off in sch["cols"]:
+        if cname == name:
+            v = np.ascontiguousarray(values.astype({"f32": np.float32, "i32": np.int32, "i64": np.int64,
+                                                    "f64": np.float64}[ctype]))
+            arr[:, off:off + v.itemsize] = v.view(np.uint8).reshape(-1, v.itemsize)
+            return arr.tobytes()
+    raise KeyError(name)

@@ -25,13 +25,16 @@ def compare(spec, got, exp, rtol=RTOL):
     """Raise AssertionError with a precise message on the first mismatch."""
     assert np.array_equal(got["win_id"], exp["win_id"]), \
         f"window ids differ: got {got['win_id'][:8]}.. ({len(got['win_id'])}) exp {exp['win_id'][:8]}.. ({len(exp['win_id'])})"
+    # headers: σ/π (IStream) windows too -- nrows counts the projected tuples of
+    # W_j \ W_{j-1} (reading A9), ts is reading A7
+    assert np.array_equal(got["win_ts"], exp["win_ts"]), \
+        f"window timestamps differ at {np.nonzero(got['win_ts'] != exp['win_ts'])[0][:5]}"
+    assert np.array_equal(got["win_nrows"], exp["win_nrows"]), \
+        f"rows per window differ at {np.nonzero(got['win_nrows'] != exp['win_nrows'])[0][:5]}"
     if not spec.get("aggs"):
         assert got["tuples"] == exp["tuples"], \
             f"IStream bytes differ ({len(got['tuples'])} vs {len(exp['tuples'])} bytes)"
         return
-    assert np.array_equal(got["win_ts"], exp["win_ts"]), "window timestamps differ"
-    assert np.array_equal(got["win_nrows"], exp["win_nrows"]), \
-        f"rows per window differ at {np.nonzero(got['win_nrows'] != exp['win_nrows'])[0][:5]}"
     nk = len(spec.get("group_by", []))
     na = len(spec["aggs"])
     nrows = int(exp["win_nrows"].sum())

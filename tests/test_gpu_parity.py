@@ -437,3 +437,98 @@ def test_win_wide(saber, oracle_lib, case):
         data = gen.generate("syn", 1 << 17, 33, groups=2048)
         tb = 1 << 20
     check(saber, oracle_lib, spec, data, task_bytes=tb, result_slots=3)
+
+
+# ------------------------------------------------- registered host memory ---
+@pytest.mark.parametrize("mode", ["registered", "mixed"])
+def test_register_host_direct_dma(saber, oracle_lib, mode):
+    """The bench's end-to-end path: saber_register_host, then submits of whole
+    tasks straight from the registered range (no copyin stage) plus a ragged tail,
+    HOST result mode.  'mixed' interleaves unregistered (pageable, copyin) chunks
+    and chunks that start mid-task."""
+    import torch
+    spec, g = workloads.c3(groups=64)
+    spec["window"] = workloads.count_window(4096, 1024)
+    n = (1 << 18) + 777
+    data = gen.generate("syn", n, g["seed"], groups=64)
+    exp = oracle_lib.run(spec, data, nthreads=8)
+    pinned = torch.empty(len(data), dtype=torch.uint8).pin_memory() if mode == "mixed" else None
+    host = np.frombuffer(data, np.uint8).copy()
+    tb = 32 * 10000
+    q = saber.Query(spec, task_bytes=tb, result_mode=saber.RESULTS_HOST, result_slots=4)
+    if mode == "registered":
+        q.register_host(host)            # cudaHostRegister of the caller's pages
+        src = host
+    else:
+        pinned.numpy()[:] = host         # already page-locked (torch pinned memory)
+        src = pinned.numpy()
+        q.register_host(src)
+    slices = []
+    if mode == "registered":
+        cuts = [0, 3 * tb, 5 * tb, len(data)]
+    else:
+        cuts = [0, tb + 32 * 5, 2 * tb + 32 * 5, 4 * tb, 4 * tb + 32 * 3, len(data)]
+    unreg = np.frombuffer(data, np.uint8).copy()
+    for c, (a, b) in enumerate(zip(cuts[:-1], cuts[1:])):
+        chunk = src[a:b] if (mode == "registered" or c % 2 == 0) else unreg[a:b]
+        off = 0
+        while off < chunk.size:
+            part = chunk[off:off + 3 * tb]
+            st = q.submit(part)
+            if st == saber.EAGAIN:
+                slices.append(q.poll())
+                continue
+            assert st == 0, q.last_error()
+            off += part.size
+    while (st := q.finish()) == saber.EAGAIN:
+        slices.append(q.poll())
+    assert st == 0
+    while (s := q.poll()) is not None:
+        slices.append(s)
+    q.close()
+    compare(spec, saber.merge_slices(slices, q.m), exp)
+
+
+def test_release_out_of_order_no_partial_submit(saber, oracle_lib):
+    """Slices may be released in any order: a submit whose ring slots are not all
+    free returns EAGAIN *without consuming* input, so retrying after the
+    release continues the stream exactly (no tuple submitted twice or lost)."""
+    spec, g = workloads.c3(groups=64)
+    spec["window"] = workloads.count_window(2048, 512)
+    tb = 32 * 4096
+    n = 4096 * 9
+    data = np.frombuffer(gen.generate("syn", n, g["seed"], groups=64), np.uint8)
+    exp = oracle_lib.run(spec, data.tobytes(), nthreads=8)
+    q = saber.Query(spec, task_bytes=tb, result_slots=4)
+    for t in range(3):
+        assert q.submit(data[t * tb:(t + 1) * tb]) == 0
+    st0, r0 = q.poll_raw(-1)
+    st1, r1 = q.poll_raw(-1)
+    assert st0 == 0 and st1 == 0
+    skip = set(range(int(r1.first_window), int(r1.first_window + r1.nwindows)))
+    q.release(r1)                        # slot 1 free, slot 0 still held
+    # the next two tasks need ring slots 3 and 0: slot 0 is held -> EAGAIN, nothing consumed
+    assert q.submit(data[3 * tb:5 * tb]) == saber.EAGAIN
+    q.release(r0)                        # slice 0 and 1 are not read: their windows are skipped
+    skip |= set(range(int(r0.first_window), int(r0.first_window + r0.nwindows)))
+    slices, off = [], 3 * tb
+    while off < data.size:
+        st = q.submit(data[off:off + 2 * tb])
+        if st == saber.EAGAIN:
+            slices.append(q.poll())
+            continue
+        assert st == 0, q.last_error()
+        off += 2 * tb
+    while (st := q.finish()) == saber.EAGAIN:
+        slices.append(q.poll())
+    assert st == 0
+    while (sl := q.poll()) is not None:
+        slices.append(sl)
+    q.close()
+    got = saber.merge_slices(slices, q.m)
+    keep = ~np.isin(exp["win_id"], sorted(skip))
+    rowkeep = np.repeat(keep, exp["win_nrows"])
+    sub = {"win_id": exp["win_id"][keep], "win_ts": exp["win_ts"][keep], "win_nrows": exp["win_nrows"][keep],
+           "keys": exp["keys"][rowkeep], "vals": [v[rowkeep] for v in exp["vals"]], "tuples": b""}
+    assert len(sub["win_id"]) > 0
+    compare(spec, got, sub)

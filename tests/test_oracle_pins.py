@@ -343,3 +343,41 @@ def test_errors(oracle_lib):
     r = oracle_lib.run(spec({"kind": "count", "size": 4, "slide": 1}, aggs=[("count", None)]),
                        stream(v=[1, 2, 3]))
     assert len(r["win_id"]) == 0
+
+
+def test_int64_sum_overflow_detected(oracle_lib):
+    """SUM over an I64 column is checked (reading A14): a window whose exact sum
+    leaves [-2^63, 2^63) makes the oracle report OQ_EOVERFLOW (-75); sums that end
+    exactly on the representable boundary do not."""
+    def run(m):
+        a = np.zeros(len(m), dtype=[("ts", "<i8"), ("v", "<i4"), ("x", "<f4"), ("m", "<i8"),
+                                    ("k", "<i4"), ("o", "<i4")])
+        a["ts"] = np.arange(len(m))
+        a["m"] = m
+        return oracle_lib.run(spec({"kind": "count", "size": 2, "slide": 2}, aggs=[("sum", "m")]), a.tobytes())
+    big = 1 << 62
+    r = run([big, big - 1, -big, -big])                  # 2^63 - 1 and -2^63: both exact
+    assert list(r["vals"][0]) == [(1 << 63) - 1, -(1 << 63)]
+    for m in ([big, big], [-big, -big - 1], [1, 2, big, big]):
+        with pytest.raises(oracle_lib.OracleError) as e:
+            run(m)
+        assert e.value.code == -75, m
+
+
+def test_istream_rows_per_window(oracle_lib):
+    """IStream headers (reading A9): window j's row count is the number of selected
+    tuples in the position segment W_j \\ W_{j-1} = [(j-1)·l + s, j·l + s) (j >= 1;
+    W_0 whole), counted here with numpy; header ts = τ of position j·l (A7)."""
+    n = 3000
+    d = _syn(n)
+    a3 = gen.column(d, "syn", "a3")
+    ts = gen.column(d, "syn", "ts")
+    th = 1 << 30
+    for s, l in [(64, 8), (100, 100), (1, 1), (50, 49), (7, 3)]:
+        r = oracle_lib.run(_syn_spec({"kind": "count", "size": s, "slide": l},
+                                     where=[("a3", "<", th)], project=["a3"]), d)
+        W = (n - s) // l + 1
+        sel = (a3 < th).astype(np.int64)
+        exp = [int(sel[0:s].sum())] + [int(sel[(j - 1) * l + s:j * l + s].sum()) for j in range(1, W)]
+        assert list(r["win_nrows"]) == exp
+        assert list(r["win_ts"]) == [int(ts[j * l]) for j in range(W)]
