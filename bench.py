@@ -45,13 +45,16 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="saber", choices=["saber", "reference"])
-    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "C5a", "C5b", "SG1"])
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "C5a", "C5b", "SG1", "CM2"])
+    ap.add_argument("--npred", type=int, default=1,
+                    help="C2: SELECT_n -- n predicate terms (n-1 always-true terms, Fig. 10a)")
     ap.add_argument("--groups", type=int, default=64)
     ap.add_argument("--sel", type=float, default=0.5)
     ap.add_argument("--rate", type=int, default=0)
     ap.add_argument("--tuples-log2", type=int, default=0, help="tuples per GPU (default: the config's)")
-    ap.add_argument("--task-mb", type=int, default=4096,
-                    help="query task size φ in MiB (device-resident leg; B200 plateau: DESIGN.md §8 φ sweep)")
+    ap.add_argument("--task-mb", type=int, default=0,
+                    help="query task size φ in MiB (device-resident leg; default: the config's, "
+                         "saber_inputs.workloads.BENCH_TASK_MB -- B200 plateau: DESIGN.md §8 φ sweep)")
     ap.add_argument("--e2e-task-mb", type=int, default=256,
                     help="task size φ of the end-to-end leg (finer tasks pipeline H2D with compute)")
     ap.add_argument("--size", type=int, default=0, help="override the window size (slide sweeps, Fig. 11)")
@@ -67,7 +70,7 @@ def workload(args):
     if c == "C1":
         spec, g = workloads.c1()
     elif c == "C2":
-        spec, g = workloads.c2(sel=args.sel)
+        spec, g = workloads.c2(sel=args.sel, npred=args.npred)
     elif c == "C3":
         spec, g = workloads.c3(groups=args.groups)
     elif c == "C4":
@@ -76,6 +79,8 @@ def workload(args):
         spec, g = workloads.c5a(rate=args.rate or 4096)
     elif c == "C5b":
         spec, g = workloads.c5b(rate=args.rate or 8192)
+    elif c == "CM2":
+        spec, g = workloads.cm2(rate=args.rate or 64)
     else:
         spec, g = workloads.sg1(rate=args.rate or 4096)
     if args.tuples_log2:
@@ -93,7 +98,10 @@ def workload(args):
         "C5a": f"SG 32-B, AVG(value) GROUP BY plug,household,house, time w(3600,1), R={g['rate']}/s",
         "C5b": f"LRB 32-B, AVG(speed) GROUP BY highway,direction,position/5280 HAVING avg<40, time w(300,1), R={g['rate']}/s",
         "SG1": f"SG 32-B, AVG(value), time w(3600,1), R={g['rate']}/s",
+        "CM2": f"CM 64-B, AVG(cpu) WHERE eventType==1 GROUP BY jobId (int64, undeclared), time w(60,1), R={g['rate']}/s",
     }[c]
+    if c == "C2" and args.npred > 1:
+        desc += f" [SELECT_{args.npred}: {args.npred - 1} extra always-true terms]"
     if args.size or args.slide:
         desc += f" [window overridden: size {w['size']}, slide {w['slide']}]"
     name = f"{c}: {desc}, 2^{int(np.log2(g['n']))} tuples ({g['n'] * spec['schema']['tuple_bytes'] >> 20} MiB) per GPU"
@@ -325,7 +333,7 @@ def main():
     stream = torch.cuda.current_stream()
     gen_device(lib_gen, g["kind"], g["seed"], begin, n, g["rate"], g["groups"], part, stream.cuda_stream)
     torch.cuda.synchronize()
-    task_bytes = args.task_mb << 20
+    task_bytes = (args.task_mb or workloads.bench_task_mb(args.config, args.groups)) << 20
 
     def barrier():
         if world > 1:
@@ -438,8 +446,17 @@ def main():
         traffic = traffic["dram_bytes"] * (per_launch_bytes / cap_in) if cap_in else None
         if cap_in != int(per_launch_bytes):
             traffic_note = f"scaled from an ncu capture of a {cap_in >> 20} MiB launch"
+    # whole-step roofline: algorithmic bytes of the step (input sectors read + result
+    # rows, headers and projected tuples written) / step time
+    ctype = {c[0]: c[1] for c in spec["schema"]["cols"]}
+    row_bytes = sum(4 if ctype[c] == "i32" else 8 for c, _, _ in spec.get("group_by", [])) + 8 * len(spec.get("aggs", []))
+    proj_bytes = sum(4 if ctype[c] in ("i32", "f32") else 8 for c in spec.get("project", []))
+    step_bytes = n * tb + out_rows * row_bytes + out_windows * 32 + out_tuples * proj_bytes   # per GPU
+    step_gbs = step_bytes / (ms_step / 1e3) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": (achieved / peak) if achieved else None, "traffic": traffic, "traffic_note": traffic_note,
+                "frac": (achieved / peak) if achieved else None,
+                "step_achieved": step_gbs, "step_frac": step_gbs / peak, "step_bytes_per_gpu": step_bytes,
+                "traffic": traffic, "traffic_note": traffic_note,
                 "kernel": saber.SCAN_KERNELS[stats_acc[-1]["scan_kind"]] if stats_acc else None,
                 "window_kernels": saber.WINDOW_KERNELS[stats_acc[-1]["window_kind"]] if stats_acc else None,
                 "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,

@@ -16,6 +16,7 @@
 // look-back over earlier tickets and writes headers and rows (window-major,
 // key order inside a window).
 #include <cuda_runtime.h>
+#include <cstdlib>
 #include <stdint.h>
 
 #include "common.cuh"
@@ -26,13 +27,31 @@ namespace sb {
 
 constexpr int kWbThreads = 256;
 constexpr int kWbMaxWin = 512;          // windows per item (row counts in shared memory)
-constexpr int kWbMaxRounds = 256;       // (window, key) rounds of 256 per item
+constexpr int kWbMaxRounds = 64;        // (window, key) rounds of 256 per item
+constexpr int kWbMaxWords = 1024;       // table words per pane slot
 
+template <bool FAST>
 __device__ __forceinline__ uint64_t wb_combine(int kind, uint64_t a, uint64_t b) {
+  if (FAST)        // counts and sums only: integer or fp64 add
+    return kind == FK_SUM_F ? (uint64_t)__double_as_longlong(__longlong_as_double((long long)a) +
+                                                             __longlong_as_double((long long)b))
+                            : a + b;
   return kind < 0 ? a + b : field_combine(kind, a, b);
 }
 
-template <int NF>
+// fp64 x / c for a positive count c: reciprocal seed, one Newton step and a
+// residual correction of the quotient (within an ulp; AVG is compared at 1e-5, A12)
+__device__ __forceinline__ double wb_div(double x, double c) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(c));
+  r = fma(r, fma(-c, r, 1.0), r);
+  const double q = x * r;
+  return fma(r, fma(-c, q, x), q);
+}
+
+// FAST: dense / global keys (one int32 key or none), only COUNT / SUM / AVG over
+// sum fields, no HAVING: presence is count > 0 and rows are written directly
+template <int NF, bool FAST>
 __global__ void __launch_bounds__(kWbThreads)
 k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table,
             const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
@@ -43,6 +62,9 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
   __shared__ int64_t s_base;
   __shared__ int s_wcnt[kWbMaxWin];           // rows per window of the item
   __shared__ int s_roff[kWbMaxRounds * 8];    // rows per (round, warp) → exclusive offsets
+  __shared__ unsigned s_rbal[kWbMaxRounds * 8];  // presence ballots per (round, warp)
+  __shared__ int s_woff[kWbMaxWin];           // first row of each window inside the item
+  __shared__ signed char s_kind[kWbMaxWords];  // combine of each table word: -1 count, else the field kind
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t J0 = st->J0, J1 = st->J1;
   if (J1 <= J0) return;
@@ -59,6 +81,10 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
   uint64_t *V = NB == 1 ? raw : raw + (int64_t)NP * W;
   const unsigned lt = (1u << lane) - 1u;
   if (tid == 0) { mbar_init(&bar, 1); fence_mbar_init(); }
+  for (int w = tid; w < W; w += kWbThreads) {
+    const int f = (int)(w / C) - 1;
+    s_kind[w] = (signed char)(f < 0 ? -1 : p.field[f].kind);
+  }
   __syncthreads();
   uint32_t phase = 0;
   for (;;) {
@@ -106,6 +132,10 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
     phase ^= 1u;
     // ---- van Herk / Gil-Werman per table word (threads over consecutive words,
     // so shared-memory accesses are conflict-free)
+    // presence of a row depends only on the window count when there is no HAVING:
+    // the count words are assembled first and the item's row count is published
+    // to the look-back chain before the field words are, so successors rarely wait
+    const bool early = NB == 1 && !p.nhave;
     if (NB == 1) {
       // in place: (A) suffix of block b0 into its own rows and prefix of block
       // b0+1 into its own rows, one thread per (word, direction); (B) V[a] =
@@ -113,58 +143,76 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
       const int64_t bs = q0, be = (bs + K - 1) < qhi ? (bs + K - 1) : qhi;
       const int64_t lo = bs > qlo ? bs : qlo;
       const int64_t pe = (bs + 2 * K - 2) < qhi ? (bs + 2 * K - 2) : qhi;   // last prefix pane needed
-      // field of table word w (count words first): compares instead of a division
-      auto field_of = [&](int w) {
-        int f = -1;
-#pragma unroll
-        for (int k = 0; k < kMaxField; ++k)
-          if (k < p.nf && w >= (k + 1) * (int)C) f = k;
-        return f;
-      };
       const int Wi = (int)W;
-      for (int x = tid; x < 2 * Wi; x += kWbThreads) {
-        const bool suffix = x < Wi;
-        const int w = suffix ? x : x - Wi;
-        const int f = field_of(w);
-        const int kind = f < 0 ? -1 : p.field[f].kind;
-        uint64_t acc = kind < 0 ? 0ull : field_identity(kind);
-        // 4 loads in flight per step (the combine chain is the only dependency)
-        const int qa = suffix ? (int)(be - q0) : (int)(bs + K - q0);
-        const int qe = suffix ? (int)(lo - q0) : (int)(pe - q0);     // inclusive end of the walk
-        const int n = suffix ? qa - qe + 1 : qe - qa + 1;
-        const int dq = suffix ? -Wi : Wi;
-        uint64_t *r = raw + qa * Wi + w;
-        int k = 0;
-        for (; k + 4 <= n; k += 4) {
-          const uint64_t v0 = r[0], v1 = r[dq], v2 = r[2 * dq], v3 = r[3 * dq];
-          acc = wb_combine(kind, acc, v0); r[0] = acc;
-          acc = wb_combine(kind, acc, v1); r[dq] = acc;
-          acc = wb_combine(kind, acc, v2); r[2 * dq] = acc;
-          acc = wb_combine(kind, acc, v3); r[3 * dq] = acc;
-          r += 4 * dq;
+      auto vh_words = [&](int wa, int wb) {          // words [wa, wb) of every staged pane
+        const int Wr = wb - wa;
+        for (int x = tid; x < 2 * Wr; x += kWbThreads) {
+          const bool suffix = x < Wr;
+          const int w = wa + (suffix ? x : x - Wr);
+          const int kind = s_kind[w];
+          uint64_t acc = kind < 0 ? 0ull : field_identity(kind);
+          // 4 loads in flight per step (the combine chain is the only dependency)
+          const int qa = suffix ? (int)(be - q0) : (int)(bs + K - q0);
+          const int qe = suffix ? (int)(lo - q0) : (int)(pe - q0);     // inclusive end of the walk
+          const int n = suffix ? qa - qe + 1 : qe - qa + 1;
+          const int dq = suffix ? -Wi : Wi;
+          uint64_t *r = raw + qa * Wi + w;
+          int k = 0;
+          for (; k + 4 <= n; k += 4) {
+            const uint64_t v0 = r[0], v1 = r[dq], v2 = r[2 * dq], v3 = r[3 * dq];
+            acc = wb_combine<FAST>(kind, acc, v0); r[0] = acc;
+            acc = wb_combine<FAST>(kind, acc, v1); r[dq] = acc;
+            acc = wb_combine<FAST>(kind, acc, v2); r[2 * dq] = acc;
+            acc = wb_combine<FAST>(kind, acc, v3); r[3 * dq] = acc;
+            r += 4 * dq;
+          }
+          for (; k < n; ++k) {
+            acc = wb_combine<FAST>(kind, acc, r[0]);
+            r[0] = acc;
+            r += dq;
+          }
         }
-        for (; k < n; ++k) {
-          acc = wb_combine(kind, acc, r[0]);
-          r[0] = acc;
-          r += dq;
+        __syncthreads();
+        const int64_t a0 = lo > bs ? lo : bs + 1;                // windows starting at a0..be need a prefix
+        const int64_t a1 = (pe - K + 1) < be ? (pe - K + 1) : be;
+        const int nvals = a1 >= a0 ? (int)((a1 - a0 + 1) * Wr) : 0;
+        // (pane, word) pairs walked incrementally: no division per element
+        const int step_a = kWbThreads / Wr, step_w = kWbThreads % Wr;
+        int ao = tid / Wr, w = tid - (tid / Wr) * Wr;
+        const int base_a = (int)(a0 - q0), Kd = (int)(K - 1) * Wi;
+        for (int x = tid; x < nvals; x += kWbThreads) {
+          const int kind = s_kind[wa + w];
+          uint64_t *rr = raw + (base_a + ao) * Wi + wa + w;
+          *rr = wb_combine<FAST>(kind, *rr, rr[Kd]);
+          ao += step_a;
+          w += step_w;
+          if (w >= Wr) { w -= Wr; ++ao; }
         }
-      }
-      __syncthreads();
-      const int64_t a0 = lo > bs ? lo : bs + 1;                // windows starting at a0..be need a prefix
-      const int64_t a1 = (pe - K + 1) < be ? (pe - K + 1) : be;
-      const int nvals = a1 >= a0 ? (int)((a1 - a0 + 1) * W) : 0;
-      // (pane, word) pairs walked incrementally: no division per element
-      const int step_a = kWbThreads / Wi, step_w = kWbThreads % Wi;
-      int ao = tid / Wi, w = tid - (tid / Wi) * Wi;
-      const int base_a = (int)(a0 - q0), Kd = (int)(K - 1) * Wi;
-      for (int x = tid; x < nvals; x += kWbThreads) {
-        const int f = field_of(w);
-        const int kind = f < 0 ? -1 : p.field[f].kind;
-        uint64_t *rr = raw + (base_a + ao) * Wi + w;
-        *rr = wb_combine(kind, *rr, rr[Kd]);
-        ao += step_a;
-        w += step_w;
-        if (w >= Wi) { w -= Wi; ++ao; }
+      };
+      if (early) {
+        vh_words(0, (int)C);
+        __syncthreads();
+        // rows per window from the counts alone; the item total is published now
+        const int Ci = (int)C;
+        const int nit = nwin * Ci;
+        int mine = 0;
+        for (int it = tid; it < nit; it += kWbThreads) {
+          const int wi = it / Ci, key = it - wi * Ci;
+          const bool pres = (int64_t)(V + ((ja + wi) * L - q0) * W)[key] > 0;
+          mine += pres;
+          if (pres) atomicAdd(&s_wcnt[wi], 1);
+        }
+        mine = __reduce_add_sync(kFull, (unsigned)mine);
+        if (lane == 0) s_roff[warp] = mine;
+        __syncthreads();
+        if (tid == 0) {
+          int tot = 0;
+          for (int i = 0; i < kWbThreads / 32; ++i) tot += s_roff[i];
+          if (t > 0) lb_st(&status[t], lb_pack(epoch, 1, (uint64_t)tot));
+        }
+        vh_words((int)C, Wi);
+      } else {
+        vh_words(0, Wi);
       }
     } else {
       // separate V: one thread per (block, word): suffix into V, then the prefix
@@ -181,15 +229,15 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
         const int64_t be = (bs + K - 1) < qhi ? (bs + K - 1) : qhi;
         uint64_t acc = id;
         for (int64_t q = be; q >= lo; --q) {
-          acc = wb_combine(kind, acc, raw[(q - q0) * W + w]);
+          acc = wb_combine<FAST>(kind, acc, raw[(q - q0) * W + w]);
           V[(q - q0) * W + w] = acc;
         }
         acc = id;
         for (int64_t a = bs + 1; a <= be; ++a) {
           const int64_t e = a + K - 1;
           if (e > qhi) break;
-          acc = wb_combine(kind, acc, raw[(e - q0) * W + w]);
-          if (a >= lo) V[(a - q0) * W + w] = wb_combine(kind, V[(a - q0) * W + w], acc);
+          acc = wb_combine<FAST>(kind, acc, raw[(e - q0) * W + w]);
+          if (a >= lo) V[(a - q0) * W + w] = wb_combine<FAST>(kind, V[(a - q0) * W + w], acc);
         }
       }
     }
@@ -204,20 +252,21 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
       const int wi = win_of(it), key = it - wi * Ci;
       const uint64_t *v = V + ((ja + wi) * L - q0) * W;
       c = (int64_t)v[key];
-      if (c <= 0) return false;
+      if (FAST || c <= 0) return c > 0;
 #pragma unroll
       for (int f = 0; f < NF; ++f)
         if (f < p.nf) fv[f] = v[(1 + f) * C + key];
       return !p.nhave || having_ok(p, c, fv);
     };
+    // pass 1: presence per item (ballots kept for pass 2), rows per window
     for (int r = 0; r < nrounds; ++r) {
       const int it = r * kWbThreads + tid;
-      int64_t c;
+      int64_t c = 0;
       uint64_t fv[kMaxField];
       const bool pres = it < nitem && value(it, c, fv);
       const unsigned bal = __ballot_sync(kFull, pres);
-      if (lane == 0) s_roff[r * 8 + warp] = __popc(bal);
-      if (pres) atomicAdd(&s_wcnt[win_of(it)], 1);
+      if (lane == 0) { s_roff[r * 8 + warp] = __popc(bal); s_rbal[r * 8 + warp] = bal; }
+      if (pres && !early) atomicAdd(&s_wcnt[win_of(it)], 1);
     }
     __syncthreads();
     if (warp == 0) {                                          // exclusive scan of (round, warp) counts
@@ -243,41 +292,69 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
           if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
         }
       }
+    } else if (warp == 1) {                                   // window row offsets: scan of rows per window
+      int run = 0;
+      for (int b = 0; b < nwin; b += 32) {
+        const int v = b + lane < nwin ? s_wcnt[b + lane] : 0;
+        int y = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int z = __shfl_up_sync(kFull, y, o);
+          if (lane >= o) y += z;
+        }
+        if (b + lane < nwin) s_woff[b + lane] = run + y - v;
+        run += __shfl_sync(kFull, y, 31);
+      }
     }
     __syncthreads();
     const int64_t base = s_base;
-    // headers: a window's first row is the offset of its first (window, key) item
     for (int wi = tid; wi < nwin; wi += kWbThreads) {
-      const int it = wi * (int)C;
-      const int r = it / kWbThreads, ln = it % kWbThreads;
-      int before = 0;                                         // present items of round r before lane ln
-      for (int i = r * kWbThreads + (ln & ~31); i < it; ++i) {
-        int64_t c;
-        uint64_t fv[kMaxField];
-        before += value(i, c, fv);
-      }
       const int64_t j = ja + wi;
       WinHdr h;
       h.window_id = j;
       h.ts = (p.win_kind == WK_TIME) ? p.T0 + j * p.l : pane_ts[(j * L) & Rm];
-      h.row_offset = base + s_roff[r * 8 + (ln >> 5)] + before;
+      h.row_offset = base + s_woff[wi];
       h.nrows = s_wcnt[wi];
       h.flags = 0;
       hdr[j - J0] = h;
     }
     for (int r = 0; r < nrounds; ++r) {
       const int it = r * kWbThreads + tid;
+      const unsigned bal = s_rbal[r * 8 + warp];
+      if (!((bal >> lane) & 1u)) continue;
       int64_t c = 0;
       uint64_t fv[kMaxField];
 #pragma unroll
       for (int f = 0; f < kMaxField; ++f) fv[f] = 0;
-      const bool pres = it < nitem && value(it, c, fv);
-      const unsigned bal = __ballot_sync(kFull, pres);
-      if (pres) {
-        int64_t kv[kMaxKey];
-        decode_key(p, (uint64_t)(it - win_of(it) * Ci), kv);
-        write_row(p, rows, base + s_roff[r * 8 + warp] + __popc(bal & lt), kv, c, fv);
+      const int64_t row = base + s_roff[r * 8 + warp] + __popc(bal & lt);
+      if (FAST) {
+        if (row >= p.rows_cap) continue;
+        const int wi = win_of(it), key = it - wi * Ci;
+        const uint64_t *v = V + ((ja + wi) * L - q0) * W;
+        const int64_t cnt = (int64_t)v[key];
+        if (p.nkeys) ((int32_t *)(rows + p.col_off[0]))[row] = key;
+#pragma unroll
+        for (int a = 0; a < kMaxAgg; ++a) {
+          if (a >= p.nagg) break;
+          const AggOut &o = p.agg[a];
+          uint64_t x = 0;
+#pragma unroll
+          for (int f = 0; f < NF; ++f)
+            if (f == o.field) x = v[(1 + f) * C + key];
+          uint64_t bits = o.fn == AG_COUNT ? (uint64_t)cnt : x;
+          if (o.fn == AG_AVG) {
+            const double sum = p.field[o.field].kind == FK_SUM_F ? __longlong_as_double((long long)x)
+                                                                  : (double)(int64_t)x;
+            bits = (uint64_t)__double_as_longlong(wb_div(sum, (double)cnt));
+          }
+          ((uint64_t *)(rows + p.col_off[p.nkeys + a]))[row] = bits;
+        }
+        continue;
       }
+      value(it, c, fv);
+      int64_t kv[kMaxKey];
+      decode_key(p, (uint64_t)(it - win_of(it) * Ci), kv);
+      write_row(p, rows, row, kv, c, fv);
     }
     // the van Herk pass wrote `raw` with generic stores; the next ticket's bulk
     // copies (async proxy) overwrite it after the barrier
@@ -305,11 +382,21 @@ bool wb_usable(const Plan &p) {
   if ((nb == 1 ? 2 * p.slot_words : nb * p.slot_words) < 64) return false;
   const int64_t nwin = (nb * p.K + p.L - 1) / p.L + 1;
   if (nwin > kWbMaxWin || (nwin * p.C + kWbThreads - 1) / kWbThreads > kWbMaxRounds) return false;
+  if (p.slot_words > kWbMaxWords) return false;
   return wb_smem(p) <= 96 * 1024;
 }
+static bool wb_fast(const Plan &p) {
+  if (p.nhave || p.has_minmax || p.nf > 2 || p.key_mode == KM_HASH) return false;
+  if (p.nkeys > 1 || (p.nkeys == 1 && (p.key_pack != KP_RADIX || p.col_bytes[0] != 4))) return false;
+  if (p.C & (p.C - 1)) return false;
+  for (int a = 0; a < p.nagg; ++a)
+    if (p.agg[a].fn != AG_COUNT && p.agg[a].fn != AG_SUM && p.agg[a].fn != AG_AVG) return false;
+  return !std::getenv("SABER_NO_WBFAST");
+}
 static void *wb_kernel(const Plan &p) {
-  return p.nf <= 1 ? (void *)k_win_block<1> : p.nf <= 2 ? (void *)k_win_block<2>
-       : p.nf <= 4 ? (void *)k_win_block<4> : (void *)k_win_block<8>;
+  if (wb_fast(p)) return p.nf <= 1 ? (void *)k_win_block<1, true> : (void *)k_win_block<2, true>;
+  return p.nf <= 1 ? (void *)k_win_block<1, false> : p.nf <= 2 ? (void *)k_win_block<2, false>
+       : p.nf <= 4 ? (void *)k_win_block<4, false> : (void *)k_win_block<8, false>;
 }
 cudaError_t wb_set_attributes(const Plan &p) {
   return cudaFuncSetAttribute(wb_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, wb_smem(p));
