@@ -62,6 +62,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--launcher-check", action="store_true",
+                    help="CPU (gloo) check of the multi-rank launch: no GPU work")
     return ap.parse_args()
 
 
@@ -304,12 +306,48 @@ def run_reference(args, spec, g, name, rank, world):
 
 
 # --------------------------------------------------------------------------- product arm
+def launch_ranks(n):
+    """``--gpus N`` outside a torchrun environment: start N ranks, one process per
+    GPU, through torch.distributed.run on 127.0.0.1, and return its exit code
+    (rank 0 prints the JSON line).  Inside torchrun, WORLD_SIZE must equal N."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def launcher_check(args, rank, world):
+    """CPU check of the multi-rank plumbing (gloo): rendezvous, world size, the
+    max-over-ranks reduction of step times and rank-0-only output."""
+    import torch
+    import torch.distributed as dist
+    dist.init_process_group("gloo")
+    t = torch.tensor([float(rank + 1)], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    if rank == 0:
+        print(json.dumps({"launcher_check": True, "n_gpus": world, "ms_max": float(t.item()),
+                          "ranks": dist.get_world_size()}), flush=True)
+    dist.destroy_process_group()
+
+
 def main():
     args = parse()
     spec, g, name, w = workload(args)
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        sys.exit(launch_ranks(args.gpus))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        print(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}", file=sys.stderr)
+        sys.exit(2)
+    if args.launcher_check:
+        launcher_check(args, rank, world)
+        return
     import torch
     import torch.distributed as dist
     if world > 1:

@@ -556,8 +556,9 @@ __device__ __forceinline__ bool fx32(uint32_t xb, uint32_t &X) {
   X = m >> sh;
   return true;
 }
-__device__ __forceinline__ void red_add_s(uint32_t *p, uint32_t v) {
-  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(p)), "r"(v) : "memory");
+// shared-memory address (u32, from __cvta_generic_to_shared once per kernel)
+__device__ __forceinline__ void red_add_s(uint32_t saddr, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
 }
 
 // flush of FX tables: sum the copies' count and limbs of each entry, one set of
@@ -657,6 +658,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   for (int f = 0; f < NF; ++f) fw[f] = p.field[f].word & 3;
   const int64_t Rm = p.R - 1;
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(stages);
+  const uint32_t s_tcnt = (uint32_t)__cvta_generic_to_shared(tcnt), s_tf = (uint32_t)__cvta_generic_to_shared(tf);
   int err = 0;
   int prel = -1;                                             // CTA-uniform pane window [prel, prel+PL)
   int64_t prev_last = (lo > 0 && lo < hi) ? *(const int64_t *)(tup + (lo - 1) * tb + tsoff) : INT64_MIN;
@@ -751,11 +753,11 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
             const int e = po * C + (int)key;
             const uint32_t xb = OC == 2 ? sel4c<2>(v4) : ONECH ? sel4(v4, fw[0]) : lds_u32(t + foff[0]);
             uint32_t X;
-            red_add_s(&tcnt[e], 1u);
+            red_add_s(s_tcnt + 4u * (uint32_t)e, 1u);
             if (fx32(xb, X)) {
-              uint32_t *lm = (uint32_t *)tf + 2 * e;
+              const uint32_t lm = s_tf + 8u * (uint32_t)e;
               red_add_s(lm, X & 0xffffu);
-              red_add_s(lm + 1, X >> 16);
+              red_add_s(lm + 4u, X >> 16);
             } else {
               atomicAdd((double *)&table[((P0 + prel + po) & Rm) * p.slot_words + p.C + key], fv[0]);
             }

@@ -252,11 +252,15 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
       const int wi = win_of(it), key = it - wi * Ci;
       const uint64_t *v = V + ((ja + wi) * L - q0) * W;
       c = (int64_t)v[key];
-      if (FAST || c <= 0) return c > 0;
+      if constexpr (FAST) {
+        return c > 0;
+      } else {
+        if (c <= 0) return false;
 #pragma unroll
-      for (int f = 0; f < NF; ++f)
-        if (f < p.nf) fv[f] = v[(1 + f) * C + key];
-      return !p.nhave || having_ok(p, c, fv);
+        for (int f = 0; f < NF; ++f)
+          if (f < p.nf) fv[f] = v[(1 + f) * C + key];
+        return !p.nhave || having_ok(p, c, fv);
+      }
     };
     // pass 1: presence per item (ballots kept for pass 2), rows per window
     for (int r = 0; r < nrounds; ++r) {

@@ -17,8 +17,6 @@ bytes -- every window is computed by libsaber's kernels on the owning GPU.
 """
 from __future__ import annotations
 
-import numpy as np
-
 from .saber import partition_plan
 
 
@@ -30,37 +28,7 @@ def partition_bounds(n_total: int, world: int, rank: int) -> tuple[int, int]:
     return b, e
 
 
-def _lower_bound_ts(tuples_u8: np.ndarray, tuple_bytes: int, ts_off: int, key: int) -> int:
-    ts = np.ascontiguousarray(tuples_u8.reshape(-1, tuple_bytes)[:, ts_off:ts_off + 8]).view(np.int64).reshape(-1)
-    return int(np.searchsorted(ts, key, side="left"))
-
-
-def plan_host(spec, tuples_u8: np.ndarray, begin: int, n: int) -> tuple[int, int]:
-    """Host-side twin of saber_partition_plan for a partition held in host memory:
-    (windows closed by the partition's last tuple, first global position the
-    successor needs).  Count: closed form (L370-372); time: reading A1/A3."""
-    w = spec["window"]
-    s, l = w["size"], w["slide"]
-    if w["kind"] == "count":
-        total = begin + n
-        closed = (total - s) // l + 1 if total >= s else 0
-        return closed, closed * l
-    if n == 0:
-        return 0, begin
-    tb = spec["schema"]["tuple_bytes"]
-    ts_off = {c[0]: c[2] for c in spec["schema"]["cols"]}[spec["schema"]["ts"]]
-    tl = int(np.frombuffer(tuples_u8[(n - 1) * tb + ts_off:(n - 1) * tb + ts_off + 8].tobytes(), np.int64)[0])
-    T0 = w.get("origin", 0)
-    closed = (tl - T0 - s) // l + 1 if tl - T0 - s >= 0 else 0
-    B = T0 + closed * l
-    idx = _lower_bound_ts(tuples_u8[:n * tb], tb, ts_off, B)
-    t0 = int(np.frombuffer(tuples_u8[ts_off:ts_off + 8].tobytes(), np.int64)[0])
-    if idx == 0 and begin > 0 and t0 > B:
-        raise ValueError("partition is shorter than the window span")
-    return closed, begin + idx
-
-
-def exchange_halo(spec, part, begin: int, n: int, rank: int, world: int, device_ptr=None):
+def exchange_halo(spec, part, begin: int, n: int, rank: int, world: int, plan=None):
     """Send this partition's halo to rank+1 and receive the predecessor's.
 
     ``part`` is a torch uint8 tensor holding this rank's n tuples (CUDA tensor
@@ -68,6 +36,9 @@ def exchange_halo(spec, part, begin: int, n: int, rank: int, world: int, device_
     ``halo`` is a uint8 tensor of tuples to prepend (empty on rank 0),
     ``first_window`` the first window id this rank emits and ``base_index`` the
     global position of the first tuple it will submit (count windows).
+    ``plan(spec, part, begin, n) -> (closed, halo_first)`` defaults to
+    saber_partition_plan on the device (the window-closing rule lives in the
+    library; CPU tests pass their own, computed from the oracle).
     """
     import torch
     import torch.distributed as dist
@@ -76,10 +47,12 @@ def exchange_halo(spec, part, begin: int, n: int, rank: int, world: int, device_
     dev = part.device
     ops = []
     if rank < world - 1:
-        if part.is_cuda:
+        if plan is not None:
+            closed, halo_first = plan(spec, part, begin, n)
+        elif part.is_cuda:
             closed, halo_first = partition_plan(spec, part.data_ptr(), begin, n)
         else:
-            closed, halo_first = plan_host(spec, part.numpy(), begin, n)
+            raise ValueError("host partitions need an explicit plan (the library plans on the device)")
         meta_out = torch.tensor([closed, halo_first], dtype=torch.int64, device=dev)
         ops.append(dist.P2POp(dist.isend, meta_out, rank + 1))
     meta_in = torch.zeros(2, dtype=torch.int64, device=dev)

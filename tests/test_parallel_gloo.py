@@ -41,23 +41,42 @@ def _case(name):
     return spec, dict(g, n=3000)
 
 
+def oracle_plan(spec, part, begin, n):
+    """(windows closed by the partition's last tuple, first global position its
+    successor needs), from the oracle: the closed-window count of the stream
+    prefix and the first tuple of the next window (test-side twin of
+    saber_partition_plan; the partition holds every tuple from begin)."""
+    import oracle
+    w = spec["window"]
+    tb = spec["schema"]["tuple_bytes"]
+    data = part.numpy()
+    if w["kind"] == "count":
+        closed = (begin + n - w["size"]) // w["slide"] + 1 if begin + n >= w["size"] else 0
+        return closed, closed * w["slide"]
+    ts = np.ascontiguousarray(data.reshape(-1, tb)[:, :8]).view(np.int64).reshape(-1)
+    # windows closed by the last tuple: end <= τ_last (a tuple at or past the end arrived, reading A3)
+    closed = int(oracle.num_windows(spec, data.tobytes(), watermark=int(ts[-1])))
+    B = w.get("origin", 0) + closed * w["slide"]
+    return closed, begin + int(np.searchsorted(ts, B, side="left"))
+
+
 def _worker(rank, world, port, name, outq):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import oracle
-    from paper_conf_sigmod_koliousiswfwcp16_b200.parallel import exchange_halo, partition_bounds, plan_host
+    from paper_conf_sigmod_koliousiswfwcp16_b200.parallel import exchange_halo, partition_bounds
     spec, g = _case(name)
     N = g["n"]
     b, e = partition_bounds(N, world, rank)
     n = e - b
     data = gen.generate_array(g["kind"], n, g["seed"], i0=b, rate=g["rate"], groups=g["groups"]).reshape(-1)
     part = torch.from_numpy(data.copy())
-    halo, first_window, base_index = exchange_halo(spec, part, b, n, rank, world)
+    halo, first_window, base_index = exchange_halo(spec, part, b, n, rank, world, plan=oracle_plan)
     local = np.concatenate([halo.numpy(), data])
     tb = spec["schema"]["tuple_bytes"]
     # emulate the device pass on this rank with the oracle
     res = oracle.run(spec, local.tobytes())
-    closed = plan_host(spec, data, b, n)[0] if rank < world - 1 else None
+    closed = oracle_plan(spec, part, b, n)[0] if rank < world - 1 else None
     w = spec["window"]
     ids = res["win_id"] + (base_index // w["slide"] if w["kind"] == "count" else 0)
     keep = ids >= first_window
