@@ -39,7 +39,8 @@ typedef enum {
   SABER_EAGAIN = -11,     /* poll timed out / no result ready                        */
   SABER_EORDER = -1001,   /* timestamps not non-decreasing       */
   SABER_ECUDA = -1002,    /* CUDA runtime error or no device                         */
-  SABER_ENCCL = -1003,    /* reserved: collective failure (exchange runs in Python)  */
+  SABER_ENCCL = -1003,    /* reserved: the cross-GPU exchange runs in torch.distributed
+                             (NCCL) above this ABI                     */
   SABER_ECLOSED = -1004,  /* submit after finish                                     */
   SABER_ETS = -1005,      /* negative timestamp (time domain is {0,1,..}, L349-350)  */
   SABER_EKEY = -1006,     /* GROUP BY key outside its declared domain [0, domain)    */
@@ -147,11 +148,18 @@ saber_status saber_query_create(const saber_schema *schema, const saber_operator
                                 saber_query **out);
 
 /* Append nbytes (a multiple of tuple_bytes) of host tuples to the stream.
- * The bytes are borrowed only for the call (copied into the pinned ingest
- * ring, or DMA'd directly when the range was registered with
- * saber_register_host).  The dispatcher cuts φ-byte tasks (§4.1);
- * a partial task waits for more data or for finish().  Blocks while all
- * pipeline slots are busy. */
+ * Unregistered (pageable) bytes are borrowed only for the call: they are
+ * copied into the pinned ingest ring (the paper's copyin stage, §5.2
+ * L1220-1259).  Whole tasks inside a range registered with
+ * saber_register_host are DMA'd straight from it, asynchronously: submit
+ * returns once the copy is enqueued, and the caller must not modify those
+ * bytes until the result slice of the task holding them has been polled (or
+ * saber_query_sync returned) -- the movein of task i+1 overlaps the kernels of
+ * task i and the moveout of task i-1 (Fig. 6).  The dispatcher cuts φ-byte
+ * tasks (§4.1); a partial task waits for more data or for finish().
+ * Blocks only while a pinned staging buffer is still being copied (copyin
+ * path); returns SABER_EAGAIN, consuming nothing, when the result-ring slots
+ * the new tasks need are not all free. */
 saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t nbytes);
 
 /* Append tuples already resident in device memory.  No copy: the bytes must
@@ -209,7 +217,9 @@ typedef struct {
 
 /* Return the next result slice in task order (the paper's ordered output
  * stream, L1092-1099).  timeout_us < 0 waits forever, 0 polls.  Returns
- * SABER_EAGAIN if no slice is ready in time (or nothing is pending). */
+ * SABER_EAGAIN if no slice is ready in time (or nothing is pending).  In HOST
+ * mode the slice's D2H was issued by the query's moveout thread as soon as the
+ * task finished; poll only waits for that copy. */
 saber_status saber_results_poll(saber_query *q, saber_results *out, int32_t timeout_us);
 /* Hand a polled slice back; its slot is reused by a later task. */
 saber_status saber_results_release(saber_query *q, const saber_results *r);

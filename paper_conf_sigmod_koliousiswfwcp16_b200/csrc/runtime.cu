@@ -5,6 +5,10 @@
 //               monotone task ids (§4.1)
 //   ingest      pinned staging ring + H2D on a copy stream, event-chained to the
 //               compute stream (the paper's copyin/movein stages, §5.2)
+//   moveout     HOST result mode: a mover thread per query issues each finished
+//               task's D2H (exact sizes, from its slot metadata) on a second copy
+//               stream as soon as the task completes, so result copies overlap the
+//               next tasks' H2D and kernels (the moveout stage of Fig. 6)
 //   result ring result slot = task id mod slots; poll hands slices out in task
 //               order (the ordered output stream of §4.3)
 // Every step of a task executes in kernels.cu; nothing here touches tuple data.
@@ -15,6 +19,8 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <condition_variable>
+#include <deque>
 #include <mutex>
 #include <string>
 #include <thread>
@@ -38,6 +44,8 @@ struct Slot {
   saber_win_hdr *h_hdr = nullptr;
   SlotMeta *h_meta = nullptr;
   cudaEvent_t done = nullptr;
+  cudaEvent_t moved = nullptr;          // HOST mode: the slice's D2H on the moveout stream
+  int mstate = 0;                       // HOST mode: 0 not moved, 1 D2H issued, 2 task failed (mv_mu)
   cudaEvent_t scan_done = nullptr;      // overlap plans: the task's scan + epilogue on cs
   cudaEvent_t prof[3] = {nullptr, nullptr, nullptr};
   bool profiled = false, scanned = false;
@@ -49,7 +57,8 @@ struct Slot {
 struct Stage {
   unsigned char *h = nullptr;   // pinned
   unsigned char *d = nullptr;   // device
-  cudaEvent_t free_ev = nullptr;
+  cudaEvent_t free_ev = nullptr;     // the task reading d[] is done (device buffer reusable)
+  cudaEvent_t h2d_ev = nullptr;      // the H2D out of h[] is done (pinned staging reusable)
   bool used = false;
 };
 
@@ -94,6 +103,13 @@ struct saber_query {
   std::vector<std::pair<void *, size_t>> registered;
   std::vector<void *> prereg;   // registered by someone else: never unregistered here
   std::mutex mu;
+  // moveout (HOST result mode): task ids whose slices the mover thread copies out
+  std::thread mover;
+  std::mutex mv_mu;
+  std::condition_variable mv_cv;
+  std::deque<int64_t> mq;
+  int mv_busy = 0;
+  bool mv_stop = false;
   int64_t *d_tmp = nullptr;
   int64_t epoch_base = 0;       // look-back epoch offset across saber_query_reset
 };
@@ -500,6 +516,7 @@ static saber_status size_plan(saber_query *q) {
 }
 
 // ---------------------------------------------------------------------------
+static void mover_main(saber_query *q);
 static saber_status alloc_query(saber_query *q) {
   Plan &p = q->plan;
   CK(cudaSetDevice(q->device));
@@ -559,6 +576,7 @@ static saber_status alloc_query(saber_query *q) {
       CK(cudaMallocHost(&s.h_hdr, (size_t)p.win_cap * sizeof(saber_win_hdr)));
     }
     CK(cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&s.moved, cudaEventDisableTiming));
     if (q->cfg.profile)
       for (auto &e : s.prof) CK(cudaEventCreate(&e));
   }
@@ -609,7 +627,15 @@ static saber_status alloc_query(saber_query *q) {
   }
   CK(launch_init_state(p, q->qd, q->cfg.base_index, 0, q->cs));
   CK(cudaStreamSynchronize(q->cs));
+  if (q->cfg.result_mode == SABER_RESULTS_HOST) q->mover = std::thread(mover_main, q);
   return SABER_OK;
+}
+
+// wait until the mover has processed every task enqueued so far
+static void mover_drain(saber_query *q) {
+  if (!q->mover.joinable()) return;
+  std::unique_lock<std::mutex> lk(q->mv_mu);
+  q->mv_cv.wait(lk, [&] { return q->mq.empty() && !q->mv_busy; });
 }
 
 static saber_status check_sticky(saber_query *q) {
@@ -626,6 +652,48 @@ static bool ring_free(saber_query *q, int64_t n) {
   for (int64_t t = 0; t < n; ++t)
     if (q->slots[(q->next_task + t) % ns].state != SLOT_FREE) return false;
   return true;
+}
+
+// Moveout: for every enqueued task (task-id order), wait for it, read its slot
+// metadata and issue the D2H of exactly its headers and rows into the slot's
+// pinned mirror on the moveout stream; poll then only waits for that copy.
+static void mover_main(saber_query *q) {
+  cudaSetDevice(q->device);
+  const Plan &p = q->plan;
+  for (;;) {
+    int64_t t;
+    {
+      std::unique_lock<std::mutex> lk(q->mv_mu);
+      q->mv_cv.wait(lk, [&] { return q->mv_stop || !q->mq.empty(); });
+      if (q->mq.empty()) return;
+      t = q->mq.front();
+      q->mq.pop_front();
+      q->mv_busy = 1;
+    }
+    Slot &s = q->slots[t % (int64_t)q->slots.size()];
+    cudaError_t e = cudaEventSynchronize(s.done);
+    const SlotMeta m = *s.h_meta;
+    if (e == cudaSuccess && !m.error) {
+      if (m.nwindows)
+        e = cudaMemcpyAsync(s.h_hdr, s.dev.hdr, (size_t)m.nwindows * sizeof(saber_win_hdr), cudaMemcpyDeviceToHost,
+                            q->d2h);
+      if (p.nagg > 0) {
+        for (int c = 0; c < p.ncols && m.nrows && e == cudaSuccess; ++c)
+          e = cudaMemcpyAsync(s.h_rows + p.col_off[c], s.dev.rows + p.col_off[c], (size_t)m.nrows * p.col_bytes[c],
+                              cudaMemcpyDeviceToHost, q->d2h);
+      } else if (m.ntuples && e == cudaSuccess) {
+        e = cudaMemcpyAsync(s.h_rows, s.dev.rows, (size_t)m.ntuples * p.out_row_words * 4, cudaMemcpyDeviceToHost,
+                            q->d2h);
+      }
+      if (e == cudaSuccess) e = cudaEventRecord(s.moved, q->d2h);
+    }
+    {
+      std::lock_guard<std::mutex> lk(q->mv_mu);
+      s.mstate = (e == cudaSuccess && !m.error) ? 1 : 2;
+      q->mv_busy = 0;
+    }
+    q->mv_cv.notify_all();
+  }
 }
 
 // enqueue one task (device-resident tuples) on the compute stream
@@ -675,6 +743,14 @@ static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuple
   CK(cudaEventRecord(s.done, done_stream));
   s.state = SLOT_BUSY;
   s.task_id = q->next_task++;
+  if (q->mover.joinable()) {
+    {
+      std::lock_guard<std::mutex> lk(q->mv_mu);
+      s.mstate = 0;
+      q->mq.push_back(s.task_id);
+    }
+    q->mv_cv.notify_all();
+  }
   q->stats.tasks += 1;
   q->stats.tuples += ntuples;
   q->stats.bytes_in += ntuples * p.tuple_bytes;
@@ -744,6 +820,14 @@ saber_status saber_query_create(const saber_schema *schema, const saber_operator
 
 void saber_query_destroy(saber_query *q) {
   if (!q) return;
+  if (q->mover.joinable()) {
+    {
+      std::lock_guard<std::mutex> lk(q->mv_mu);
+      q->mv_stop = true;
+    }
+    q->mv_cv.notify_all();
+    q->mover.join();
+  }
   cudaSetDevice(q->device);
   if (q->cs) cudaStreamSynchronize(q->cs);
   if (q->h2d) cudaStreamSynchronize(q->h2d);
@@ -754,11 +838,13 @@ void saber_query_destroy(saber_query *q) {
     if (s.scan_done) cudaEventDestroy(s.scan_done);
     cudaFreeHost(s.h_meta); cudaFreeHost(s.h_rows); cudaFreeHost(s.h_hdr);
     if (s.done) cudaEventDestroy(s.done);
+    if (s.moved) cudaEventDestroy(s.moved);
     for (auto e : s.prof) if (e) cudaEventDestroy(e);
   }
   for (auto &g : q->stages) {
     cudaFreeHost(g.h); cudaFree(g.d);
     if (g.free_ev) cudaEventDestroy(g.free_ev);
+    if (g.h2d_ev) cudaEventDestroy(g.h2d_ev);
   }
   for (auto &r : q->registered)
     if (std::find(q->prereg.begin(), q->prereg.end(), r.first) == q->prereg.end()) cudaHostUnregister(r.first);
@@ -820,6 +906,7 @@ static saber_status ensure_stages(saber_query *q, bool need_host) {
     for (auto &g : q->stages) {
       CK(cudaMalloc(&g.d, tb));
       CK(cudaEventCreateWithFlags(&g.free_ev, cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&g.h2d_ev, cudaEventDisableTiming));
     }
   }
   if (need_host)
@@ -833,12 +920,10 @@ static saber_status dispatch_host_task(saber_query *q, Stage &g, const void *src
                                        int has_wm, int64_t wm) {
   const size_t bytes = (size_t)ntuples * q->plan.tuple_bytes;
   if (bytes) {
+    if (g.used) CK(cudaStreamWaitEvent(q->h2d, g.free_ev, 0));   // the previous task on g.d is done
     CK(cudaMemcpyAsync(g.d, src, bytes, cudaMemcpyHostToDevice, q->h2d));
-    cudaEvent_t ev;
-    CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-    CK(cudaEventRecord(ev, q->h2d));
-    CK(cudaStreamWaitEvent(q->cs, ev, 0));
-    CK(cudaEventDestroy(ev));
+    CK(cudaEventRecord(g.h2d_ev, q->h2d));
+    CK(cudaStreamWaitEvent(q->cs, g.h2d_ev, 0));
   }
   saber_status s = enqueue_task(q, g.d, ntuples, final_, has_wm, wm);
   if (s) return s;
@@ -867,21 +952,18 @@ saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t n
   if (saber_status s = ensure_stages(q, copyin)) return s;
   const unsigned char *src = (const unsigned char *)host_tuples;
   int64_t left = (int64_t)nbytes;
-  cudaEvent_t last_h2d = nullptr;
   while (left > 0) {
     Stage &g = q->stages[q->cur_stage];
-    if (q->stage_fill == 0 && g.used) CK(cudaEventSynchronize(g.free_ev));
     if (reg && q->stage_fill == 0 && left >= tbytes) {
-      // registered caller memory: DMA straight from it (no copyin stage)
-      CK(cudaStreamWaitEvent(q->h2d, g.free_ev, 0));
+      // registered caller memory: DMA straight from it (no copyin stage, no host wait)
       saber_status s = dispatch_host_task(q, g, src, q->task_tuples, 0, 0, 0);
       if (s) return s;
-      if (!last_h2d) CK(cudaEventCreateWithFlags(&last_h2d, cudaEventDisableTiming));
-      CK(cudaEventRecord(last_h2d, q->h2d));
       src += tbytes; left -= tbytes;
       q->cur_stage = (q->cur_stage + 1) % (int)q->stages.size();
       continue;
     }
+    // copyin: the pinned stage is rewritten only after its previous H2D completed
+    if (q->stage_fill == 0 && g.used) CK(cudaEventSynchronize(g.h2d_ev));
     const int64_t take = std::min(left, tbytes - q->stage_fill);
     std::memcpy(g.h + q->stage_fill, src, (size_t)take);   // copyin (pageable → pinned)
     q->stage_fill += take; src += take; left -= take;
@@ -891,10 +973,6 @@ saber_status saber_task_submit(saber_query *q, const void *host_tuples, size_t n
       q->stage_fill = 0;
       q->cur_stage = (q->cur_stage + 1) % (int)q->stages.size();
     }
-  }
-  if (last_h2d) {
-    CK(cudaEventSynchronize(last_h2d));   // the caller's registered bytes are free again
-    CK(cudaEventDestroy(last_h2d));
   }
   return SABER_OK;
 }
@@ -949,19 +1027,39 @@ saber_status saber_results_poll(saber_query *q, saber_results *out, int32_t time
   Slot &s = q->slots[q->next_poll % (int64_t)q->slots.size()];
   if (s.state != SLOT_BUSY || s.task_id != q->next_poll) return fail(q, SABER_EINVAL, "result ring out of order");
   CK(cudaSetDevice(q->device));
-  if (timeout_us < 0) {
-    CK(cudaEventSynchronize(s.done));
-  } else {
-    auto t0 = std::chrono::steady_clock::now();
+  const auto t0 = std::chrono::steady_clock::now();
+  auto left_us = [&]() -> int64_t {
+    return timeout_us - std::chrono::duration_cast<std::chrono::microseconds>(std::chrono::steady_clock::now() - t0).count();
+  };
+  auto wait_ev = [&](cudaEvent_t ev) -> saber_status {
+    if (timeout_us < 0) {
+      CK(cudaEventSynchronize(ev));
+      return SABER_OK;
+    }
     for (;;) {
-      cudaError_t e = cudaEventQuery(s.done);
-      if (e == cudaSuccess) break;
+      cudaError_t e = cudaEventQuery(ev);
+      if (e == cudaSuccess) return SABER_OK;
       if (e != cudaErrorNotReady) CK(e);
       cudaGetLastError();
-      auto us = std::chrono::duration_cast<std::chrono::microseconds>(std::chrono::steady_clock::now() - t0).count();
-      if (us >= timeout_us) return fail(q, SABER_EAGAIN, "poll timeout");
+      if (left_us() <= 0) return fail(q, SABER_EAGAIN, "poll timeout");
       std::this_thread::sleep_for(std::chrono::microseconds(20));
     }
+  };
+  if (saber_status w = wait_ev(s.done)) return w;
+  const bool host_mv = q->cfg.result_mode == SABER_RESULTS_HOST && q->mover.joinable();
+  if (host_mv) {
+    // the mover issued (or skipped, for a failed task) this slice's D2H
+    int ms;
+    {
+      std::unique_lock<std::mutex> lk(q->mv_mu);
+      auto ready = [&] { return s.mstate != 0; };
+      if (timeout_us < 0) q->mv_cv.wait(lk, ready);
+      else if (!q->mv_cv.wait_for(lk, std::chrono::microseconds(std::max<int64_t>(0, left_us())), ready))
+        return fail(q, SABER_EAGAIN, "poll timeout");
+      ms = s.mstate;
+    }
+    if (ms == 1)
+      if (saber_status w = wait_ev(s.moved)) return w;
   }
   s.meta = *s.h_meta;
   const Plan &p = q->plan;
@@ -989,26 +1087,11 @@ saber_status saber_results_poll(saber_query *q, saber_results *out, int32_t time
   if (p.nagg > 0) {
     out->ncols = p.ncols;
     for (int c = 0; c < p.ncols; ++c) out->col_bytes[c] = p.col_bytes[c];
-    if (host) {
-      if (s.meta.nwindows)
-        CK(cudaMemcpyAsync(s.h_hdr, s.dev.hdr, (size_t)s.meta.nwindows * sizeof(saber_win_hdr), cudaMemcpyDeviceToHost, q->d2h));
-      for (int c = 0; c < p.ncols && s.meta.nrows; ++c)
-        CK(cudaMemcpyAsync(s.h_rows + p.col_off[c], s.dev.rows + p.col_off[c], (size_t)s.meta.nrows * p.col_bytes[c],
-                           cudaMemcpyDeviceToHost, q->d2h));
-      CK(cudaStreamSynchronize(q->d2h));
-    }
     unsigned char *rows = host ? s.h_rows : s.dev.rows;
     out->hdr = host ? s.h_hdr : (const saber_win_hdr *)s.dev.hdr;
     for (int c = 0; c < p.ncols; ++c) out->cols[c] = rows + p.col_off[c];
   } else {
     out->tuple_bytes = p.out_row_words * 4;
-    if (host && (s.meta.ntuples || s.meta.nwindows)) {
-      if (s.meta.ntuples)
-        CK(cudaMemcpyAsync(s.h_rows, s.dev.rows, (size_t)s.meta.ntuples * out->tuple_bytes, cudaMemcpyDeviceToHost, q->d2h));
-      if (s.meta.nwindows)
-        CK(cudaMemcpyAsync(s.h_hdr, s.dev.hdr, (size_t)s.meta.nwindows * sizeof(saber_win_hdr), cudaMemcpyDeviceToHost, q->d2h));
-      CK(cudaStreamSynchronize(q->d2h));
-    }
     out->tuples = host ? (const void *)s.h_rows : (const void *)s.dev.rows;
     // per-window headers: row_offset / nrows count projected tuples (reading A9)
     out->hdr = host ? s.h_hdr : (const saber_win_hdr *)s.dev.hdr;
@@ -1050,10 +1133,12 @@ saber_status saber_query_reset(saber_query *q, int64_t base_index, int64_t first
   for (auto &s : q->slots)
     if (s.state == SLOT_POLLED) return fail(q, SABER_EAGAIN, "release every polled slice before reset");
   CK(cudaSetDevice(q->device));
+  mover_drain(q);
   CK(cudaStreamSynchronize(q->h2d));
   CK(cudaStreamSynchronize(q->cs));
   CK(cudaStreamSynchronize(q->ws));
-  for (auto &s : q->slots) { s.state = SLOT_FREE; s.task_id = -1; s.profiled = false; }
+  CK(cudaStreamSynchronize(q->d2h));
+  for (auto &s : q->slots) { s.state = SLOT_FREE; s.task_id = -1; s.profiled = false; s.mstate = 0; }
   for (auto &g : q->stages) g.used = false;
   q->cfg.base_index = base_index;
   q->cfg.first_window = first_window;
