@@ -245,6 +245,9 @@ typedef struct {
   int32_t scan_grid, window_grid;
   /* 1 if window assembly of a task overlaps the next task's scan (SABER_OVERLAP=1) */
   int32_t overlap, reserved;
+  /* effective task size φ in tuples: task_bytes / tuple_bytes, lowered for count
+   * windows when a task's worst-case rows would not fit one result slot */
+  int64_t task_tuples;
 } saber_stats;
 saber_status saber_query_stats(const saber_query *q, saber_stats *out);
 

@@ -492,6 +492,19 @@ static saber_status size_plan(saber_query *q) {
                            : p.bucket_mode ? std::min<int64_t>(p.s, p.G)
                            : (p.win_kind == WK_COUNT ? std::min<int64_t>(p.s, p.C * p.K) : p.C * p.K);
     int64_t rb = c.result_bytes;
+    if (p.win_kind == WK_COUNT) {
+      // a task must not close more rows than one result slot holds (else its
+      // emission would fail with SABER_ENOMEM): the dispatcher cuts smaller
+      // tasks when the worst case (rows_per_win rows in each of the T/l closed
+      // windows) exceeds the slot -- the effective φ is saber_stats.task_tuples
+      const int64_t cap = rb > 0 ? rb : (c.result_mode == SABER_RESULTS_DEVICE ? (4ll << 30) : (1ll << 30));
+      const int64_t cap_rows = cap / p.row_bytes;
+      const int64_t wmax = cap_rows / std::max<int64_t>(1, rows_per_win) - 4;
+      if (p.win_cap * rows_per_win > cap_rows && wmax >= 1) {
+        q->task_tuples = std::max<int64_t>(p.l, wmax * p.l);
+        p.win_cap = q->task_tuples / p.l + 4;
+      }
+    }
     if (rb <= 0) {
       long double bound = (long double)p.win_cap * rows_per_win * p.row_bytes;
       // device-resident results may use up to 4 GiB per slot; pinned host mirrors stay <= 1 GiB
@@ -1124,6 +1137,7 @@ saber_status saber_query_stats(const saber_query *q, saber_stats *out) {
   out->scan_grid = p.nagg == 0 ? q->sel_grid : (p.lane_alt && q->use_lane) ? q->p1_grid_lane : q->p1_grid;
   out->window_grid = p.win_block ? p.wb_grid : p.win_wide ? p.ww_grid : q->p2_grid;
   out->overlap = p.overlap;
+  out->task_tuples = q->task_tuples;
   return SABER_OK;
 }
 

@@ -91,7 +91,7 @@ class Stats(C.Structure):
                 ("last_pending", C.c_int64), ("kernel_launches", C.c_int64), ("scan_launches", C.c_int64),
                 ("scan_ms", C.c_double), ("assemble_ms", C.c_double), ("scan_kind", C.c_int32),
                 ("window_kind", C.c_int32), ("scan_grid", C.c_int32), ("window_grid", C.c_int32),
-                ("overlap", C.c_int32), ("reserved", C.c_int32)]
+                ("overlap", C.c_int32), ("reserved", C.c_int32), ("task_tuples", C.c_int64)]
 
 SCAN_KERNELS = ["k_select", "k_pane_agg", "k_pane_cnt", "k_pane_bucket"]
 WINDOW_KERNELS = ["none", "k_vh_build+k_win_packed/k_win_fused", "k_win_block", "k_bkt_count+k_win_scan+k_bkt_emit",

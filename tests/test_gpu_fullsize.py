@@ -265,6 +265,7 @@ def c6_sample(spec, g, task_bytes, nrand=1024):
 
     def ids(nwin, q):
         s, l = w["size"], w["slide"]
+        tt = q.stats()["task_tuples"]                  # effective φ (the dispatcher may cut smaller tasks)
         out = set()
         if w["kind"] == "count":
             out.update(range(0, max(0, ((1 << 22) - s) // l + 1)))
@@ -300,6 +301,9 @@ FULL = {
     "C3_G4096": (lambda: workloads.c3(groups=4096), "C3", 4096, False),
     "C3_G16384": (lambda: workloads.c3(groups=16384), "C3", 16384, False),
     "C3_G65536": (lambda: workloads.c3(groups=65536), "C3", 65536, False),
+    # φ = 4 GiB requested: one task would close 131K windows x up to 32,768 rows, more
+    # than a 4 GiB result slot; the dispatcher cuts smaller tasks instead of failing
+    "C3_G65536_phi4G": (lambda: workloads.c3(groups=65536), "C3", -4096, False),
     "C4_R64": (lambda: workloads.c4(rate=64), "C4", 64, False),
     "C4_R4096": (lambda: workloads.c4(rate=4096), "C4", 64, False),
     "C5a": (lambda: workloads.c5a(), "C5a", 64, False),
@@ -313,7 +317,8 @@ EVERY_WINDOW_WHEN_ALL = {"C3_G256", "C3_G1024", "C3_G4096", "C4_R64", "C4_R4096"
 def test_full_size(saber, oracle_lib, name):
     mk, cfg, groups, full = FULL[name]
     spec, g = mk()
-    task_bytes = workloads.bench_task_mb(cfg, groups) << 20
+    task_bytes = (workloads.bench_task_mb(cfg, groups) if groups > 0 else -groups) << 20
+    groups = abs(groups)
     full = full or (FULL_ALL and name in EVERY_WINDOW_WHEN_ALL)
     # C5a / SG1 windows span 3,600 s x 4,096 tuples/s = 14.7 M tuples each: the
     # default run draws 256 random windows (~2 min of oracle time), SABER_FULLSIZE=all 1,024
