@@ -200,13 +200,15 @@ __device__ __forceinline__ uint64_t lb_pack(uint64_t epoch, uint64_t flag, uint6
 // (to every lane) and publishes the inclusive one.  A one-thread walk costs one
 // dependent L2 round trip per predecessor: with hundreds of tiles in flight the
 // chain of a wave's last tile was tens of microseconds.
-__device__ __forceinline__ int64_t lookback_warp(uint64_t *status, int64_t t, uint64_t epoch, uint64_t total) {
+// base0: the prefix before tile 0 (rows earlier rounds of the task already wrote).
+__device__ __forceinline__ int64_t lookback_warp(uint64_t *status, int64_t t, uint64_t epoch, uint64_t total,
+                                                 int64_t base0 = 0) {
   const int lane = threadIdx.x & 31;
   const uint64_t ep = epoch & 0xffffffull;
   const uint64_t vmask = (1ull << 38) - 1;
   if (t == 0) {
-    if (lane == 0) lb_st(&status[0], lb_pack(epoch, 2, total));
-    return 0;
+    if (lane == 0) lb_st(&status[0], lb_pack(epoch, 2, (uint64_t)base0 + total));
+    return base0;
   }
   if (lane == 0) lb_st(&status[t], lb_pack(epoch, 1, total));
   int64_t excl = 0;

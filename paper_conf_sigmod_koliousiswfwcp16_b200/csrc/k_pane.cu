@@ -238,6 +238,11 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     for (int f = 0; f < NF; ++f) tf[f * TE * CW + e] = f < p.nf ? field_identity(p.field[f].kind) : 0;
   }
 
+  // rounds (Plan::rounds > 1): this launch scans the sub-range k_task_begin chose
+  if (p.rounds > 1) {
+    tup += st->round_off * tb;
+    n = st->round_n;
+  }
   // contiguous, stage-aligned range of this CTA
   const int64_t per = ((n + gridDim.x - 1) / gridDim.x + ST - 1) / ST * ST;
   const int64_t lo = (int64_t)blockIdx.x * per;

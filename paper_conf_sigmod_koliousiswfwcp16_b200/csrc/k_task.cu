@@ -10,15 +10,51 @@ namespace sb {
 __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, int64_t n, int final_,
                              int has_wm, int64_t wm, int emit_on_finish, SlotMeta *meta,
                              const unsigned char *carry0, const unsigned char *carry1, int *tile_ctr,
-                             int64_t *win_ts, int64_t ts_mask) {
+                             int64_t *win_ts, int64_t ts_mask, int round) {
   const int lane = threadIdx.x;
   __shared__ int64_t sh[8];
+  // ---- rounds (time-window aggregation, Plan::rounds > 1): this round takes the
+  // longest unconsumed prefix of the task whose panes fit the ring next to the
+  // panes of windows not yet emitted (J0·L ..).  If not even the next tuple fits
+  // (a time gap wider than the ring), the round consumes nothing and only closes
+  // the windows that tuple's arrival closes (their end <= its τ, reading A3):
+  // the gap's windows are emitted -- empty ones with a header (A6) -- and the
+  // ring moves past the gap for the next round
+  int64_t off = 0, nn = n, closeB = INT64_MIN;
+  bool short_rounds = false;
+  if (p.rounds > 1) {
+    if (lane == 0) {
+      sh[0] = round == 0 ? 0 : st->round_off + st->round_n;
+      sh[1] = st->J0;
+    }
+    __syncwarp();
+    off = sh[0];
+    const int64_t rem = n - off;
+    nn = 0;
+    if (rem > 0) {
+      const int64_t pmax = sh[1] * p.L + p.R - 1;                 // last pane the ring can hold
+      const int64_t tbeyond = p.T0 + (pmax + 1) * p.g;            // first τ past it
+      const unsigned char *tr = tup + off * p.tuple_bytes;
+      nn = warp_lower_bound(p, tr, rem, tr, 0, tbeyond);
+      if (nn < rem) closeB = tau_at(p, tr, nn);          // the next tuple of the task has arrived
+      short_rounds = round == p.rounds - 1 && nn < rem;
+    }
+    __syncwarp();
+    tup += off * p.tuple_bytes;
+    n = nn;
+  }
   if (lane == 0) {
-    int err = 0;
+    int err = short_rounds ? ERR_CAPACITY : 0;
     const int64_t pos0 = st->pos_next;
     st->task_pos = pos0;
     st->task_n = n;
+    st->round_off = off;
+    st->round_n = n;
     int64_t J0 = st->J0, J1 = J0;
+    // result slot bases: the first round opens the slot, later ones append
+    if (round == 0) { st->slot_J0 = J0; st->row_base = 0; }
+    else st->row_base = st->sel_rows;
+    st->hdr_base = J0 - st->slot_J0;
     int64_t plo = 0, phi = -1;
     if (n > 0) {
       int64_t tf = tau_at(p, tup, 0), tl = tau_at(p, tup, n - 1);
@@ -42,6 +78,7 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
       bool haveB = true;
       if (use_wm && has_wm) B = wm;
       else if (use_wm) { B = st->tau_last + 1; haveB = st->has_tau; }
+      else if (closeB != INT64_MIN) B = closeB;                 // rounds: close by the next tuple's arrival
       else { B = st->tau_last; haveB = st->has_tau; }
       if (haveB && B - p.T0 - p.s >= 0) J1 = (B - p.T0 - p.s) / p.l + 1;
     } else {
@@ -51,28 +88,50 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
     }
     if (J1 < J0) J1 = J0;
     st->pos_next = pos0 + n;
-    st->J1 = J1;
-    // pane ring: slots of panes [J0·L, phi] must coexist during this task (from
-    // the previous task's J0 when its window phase may still be running)
+    if (phi > st->pane_hi) st->pane_hi = phi;
+    // time windows that start after the last pane holding data (a time gap, or a
+    // watermark past the data) are empty: they get headers only (reading A6,
+    // k_gap_hdr) and no pane of theirs is read, so a gap never has to fit the ring
+    int64_t Jn = J1;
+    st->jgap_hi = 0;
+    if (p.win_kind == WK_TIME && p.nagg > 0) {
+      const int64_t Jd = st->pane_hi >= 0 ? st->pane_hi / p.L + 1 : 0;
+      if (J1 > Jd) {
+        Jn = Jd > J0 ? Jd : J0;
+        st->jgap_hi = J1;
+      }
+    }
+    st->J1 = Jn;
+    // pane ring: slots of panes [J0·L, phi] and of the windows closed now must
+    // coexist during this task (from the previous task's J0 when its window phase
+    // may still be running)
     int64_t live_lo = (p.overlap ? st->live_J0 : J0) * p.L;
     int64_t zlo = st->zeroed_hi > live_lo ? st->zeroed_hi : live_lo;
     int64_t zhi = zlo;
-    if (phi >= 0 && p.nagg > 0) {
-      if (phi - live_lo + 1 > p.R) err |= ERR_CAPACITY;
-      else if (phi + 1 > zlo) zhi = phi + 1;
+    int64_t need_hi = phi;
+    if (Jn > J0 && (Jn - 1) * p.L + p.K - 1 > need_hi) need_hi = (Jn - 1) * p.L + p.K - 1;
+    if (need_hi >= 0 && p.nagg > 0) {
+      if (need_hi - live_lo + 1 > p.R) err |= ERR_CAPACITY;
+      else if (need_hi + 1 > zlo) zhi = need_hi + 1;
     }
     st->zero_lo = zlo;
     st->zero_hi = zhi;
     if (zhi > st->zeroed_hi) st->zeroed_hi = zhi;
-    if (phi > st->pane_hi) st->pane_hi = phi;
     meta->in_tuples = n;
     meta->in_panes = (n > 0 && phi >= plo) ? phi - plo + 1 : 0;
-    if (J1 - J0 > p.win_cap) err |= ERR_RESULT;
-    meta->first_window = J0;
-    meta->nwindows = J1 - J0;
+    const int64_t Jend = st->jgap_hi > Jn ? st->jgap_hi : Jn;
+    if (Jend - st->slot_J0 > p.win_cap) {
+      // more windows than the slot's headers hold: a sticky error, and nothing is
+      // written past the slot
+      err |= ERR_RESULT;
+      st->J1 = J0;
+      st->jgap_hi = 0;
+    }
+    meta->first_window = st->slot_J0;
+    meta->nwindows = st->J1 - st->slot_J0;
     if (err) st->error |= err;
     st->tile_epoch += 1;
-    st->sel_rows = 0;
+    st->sel_rows = st->row_base;
     *tile_ctr = 0;
     sh[0] = J0; sh[1] = J1; sh[2] = pos0;
   }
@@ -173,6 +232,7 @@ constexpr int kScanThreads = 256, kScanPer = 4, kScanTW = kScanThreads * kScanPe
 __global__ void __launch_bounds__(kScanThreads)
 k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t *__restrict__ counts,
            WinHdr *__restrict__ hdr, SlotMeta *meta, uint64_t *__restrict__ status, int *__restrict__ ticket) {
+  hdr += st->hdr_base;                         // windows earlier rounds of the task wrote
   __shared__ int64_t wsum[kScanThreads / 32];
   __shared__ int64_t s_base;
   __shared__ int s_t;
@@ -182,7 +242,7 @@ k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int64_t ntiles = (nw + kScanTW - 1) / kScanTW;
   if (nw <= 0) {
-    if (blockIdx.x == 0 && tid == 0) { meta->nrows = 0; st->sel_rows = 0; }
+    if (blockIdx.x == 0 && tid == 0) { meta->nrows = st->row_base; st->sel_rows = st->row_base; }
     return;
   }
   for (;;) {
@@ -218,7 +278,7 @@ k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t
       }
       if (lane < kScanThreads / 32) wsum[lane] = y - w;
       const uint64_t total = (uint64_t)__shfl_sync(kFull, (unsigned long long)y, 31);   // the tile total
-      const int64_t excl = lookback_warp(status, t, epoch, total);
+      const int64_t excl = lookback_warp(status, t, epoch, total, st->row_base);
       if (lane == 31) {
         s_base = excl;
         if (t == ntiles - 1) {
@@ -254,8 +314,8 @@ k_win_scan(const Plan p, State *st, const int64_t *__restrict__ pane_ts, int64_t
 
 __global__ void k_task_end(const Plan p, State *st, SlotMeta *meta) {
   if (threadIdx.x) return;
-  meta->first_window = st->J0;
-  meta->nwindows = st->J1 - st->J0;
+  meta->first_window = st->slot_J0;
+  meta->nwindows = st->J1 - st->slot_J0;
   meta->error = st->error;
   meta->pos_end = st->pos_next;
   meta->tau_last = st->tau_last;
@@ -280,7 +340,26 @@ __global__ void k_task_end(const Plan p, State *st, SlotMeta *meta) {
     if (e > st->vh_pre_hi) st->vh_pre_hi = e;
   }
   st->live_J0 = st->J0;
-  st->J0 = st->J1;
+  st->J0 = st->jgap_hi > st->J1 ? st->jgap_hi : st->J1;
+  meta->nwindows = st->J0 - st->slot_J0;
+}
+
+// headers of the empty windows [J1, jgap_hi) of a time gap (k_task_begin):
+// nrows = 0, row_offset = the slot's row count so far (reading A6)
+__global__ void k_gap_hdr(const Plan p, const State *st, WinHdr *hdr, SlotMeta *meta) {
+  const int64_t a = st->J1, b = st->jgap_hi;
+  if (b <= a) return;
+  const int64_t rows = st->sel_rows;
+  for (int64_t j = a + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < b; j += (int64_t)gridDim.x * blockDim.x) {
+    WinHdr h;
+    h.window_id = j;
+    h.ts = p.T0 + j * p.l;
+    h.row_offset = rows;
+    h.nrows = 0;
+    h.flags = 0;
+    hdr[j - st->slot_J0] = h;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) meta->nrows = rows;
 }
 
 // overlap plans: close the window phase of a slot that ran on its State snapshot
@@ -352,9 +431,9 @@ __global__ void k_partition_plan(int ts_word, int tuple_bytes, int win_kind, int
 namespace sb {
 
 cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
-                              int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st) {
+                              int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st, int round) {
   k_task_begin<<<1, 32, 0, st>>>(p, q.st, (const unsigned char *)tuples, n, final_, has_wm, wm, emit_on_finish,
-                                 s.meta, q.carry[0], q.carry[1], q.tile_ctr, q.win_ts, q.ts_mask);
+                                 s.meta, q.carry[0], q.carry[1], q.tile_ctr, q.win_ts, q.ts_mask, round);
   return cudaGetLastError();
 }
 cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st) {
@@ -369,6 +448,11 @@ cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, 
   return cudaGetLastError();
 }
 cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st) {
+  if (p.win_kind == WK_TIME && p.nagg > 0) {
+    k_gap_hdr<<<148, 256, 0, st>>>(p, q.st, (WinHdr *)s.hdr, s.meta);
+    cudaError_t e = cudaGetLastError();
+    if (e) return e;
+  }
   k_task_end<<<1, 32, 0, st>>>(p, q.st, s.meta);
   return cudaGetLastError();
 }

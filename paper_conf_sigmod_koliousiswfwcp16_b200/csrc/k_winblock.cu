@@ -56,6 +56,7 @@ __global__ void __launch_bounds__(kWbThreads)
 k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table,
             const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
             uint64_t *__restrict__ status, int *__restrict__ ticket, int NB) {
+  hdr += st->hdr_base;                         // windows earlier rounds of the task wrote
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ uint64_t bar;
   __shared__ int s_t;
@@ -288,7 +289,7 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
         run += __shfl_sync(kFull, y, 31);
       }
       const uint64_t total = (uint64_t)run;
-      const int64_t excl = lookback_warp(status, t, epoch, total);
+      const int64_t excl = lookback_warp(status, t, epoch, total, st->row_base);
       if (lane == 0) {
         s_base = excl;
         if (t == nitems - 1) {

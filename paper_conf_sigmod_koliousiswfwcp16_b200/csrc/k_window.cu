@@ -418,6 +418,7 @@ __global__ void __launch_bounds__(256)
 k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre, const uint64_t *__restrict__ suf,
             const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
             uint64_t *__restrict__ status, int *__restrict__ ticket, int WC) {
+  hdr += st->hdr_base;                         // windows earlier rounds of the task wrote
   constexpr int gpb = 256 / GS;
   __shared__ int s_cnt[kFusedMaxItems];
   __shared__ int s_off[kFusedMaxItems];
@@ -503,7 +504,7 @@ k_win_fused(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ p
     __syncthreads();
     if (threadIdx.x < 32) {
       const uint64_t total = (uint64_t)s_total;
-      const int64_t excl = lookback_warp(status, t, epoch, total);
+      const int64_t excl = lookback_warp(status, t, epoch, total, st->row_base);
       if (threadIdx.x == 0) {
         s_base = excl;
         if (t == nchunks - 1) {
@@ -624,6 +625,7 @@ __global__ void __launch_bounds__(256)
 k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre, const uint64_t *__restrict__ suf,
              const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
              uint64_t *__restrict__ status, int *__restrict__ ticket, int cshift) {
+  hdr += st->hdr_base;                         // windows earlier rounds of the task wrote
   __shared__ int s_wcnt[8];
   __shared__ int64_t s_base;
   __shared__ int s_t;
@@ -676,7 +678,7 @@ k_win_packed(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ 
       const uint64_t total = (uint64_t)__shfl_sync(kFull, x, 7);
       __syncwarp();
       if (lane < 8) s_wcnt[lane] = x - v;
-      const int64_t excl = lookback_warp(status, t, epoch, total);
+      const int64_t excl = lookback_warp(status, t, epoch, total, st->row_base);
       if (lane == 0) {
         s_base = excl;
         if (t == nchunks - 1) {

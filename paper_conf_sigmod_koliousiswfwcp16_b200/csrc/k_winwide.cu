@@ -31,6 +31,7 @@ __global__ void __launch_bounds__(kWwThreads)
 k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre, const uint64_t *__restrict__ suf,
            const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
            uint64_t *__restrict__ status, int *__restrict__ ticket, int ktab, const int64_t *__restrict__ offs) {
+  hdr += st->hdr_base;                         // windows earlier rounds of the task wrote
   extern __shared__ __align__(16) int32_t s_keys[];           // ktab: decoded key columns [nkeys][C]
   __shared__ int s_cnt[RR * 8];                              // rows per (round, warp) -> exclusive offsets
   __shared__ int64_t s_base;
@@ -116,7 +117,7 @@ k_win_wide(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pr
       if (PRE) {                           // offsets from k_win_wide_count + k_win_scan (headers too)
         if (lane == 0) s_base = offs[t];
       } else {
-      const int64_t excl = lookback_warp(status, t, epoch, total);
+      const int64_t excl = lookback_warp(status, t, epoch, total, st->row_base);
       if (lane == 0) {
         s_base = excl;
         WinHdr h;

@@ -6,6 +6,10 @@
 
 namespace sb {
 
+cudaError_t launch_agg_round(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
+                             int final_, int has_wm, int64_t wm, int emit_on_finish, int p1_grid, int p2_grid,
+                             int win_chunk, cudaStream_t st, cudaEvent_t *evs, int *launches, int round);
+
 cudaError_t set_kernel_attributes(const Plan &p) {
   cudaError_t e = cudaSuccess;
   if (p.nagg == 0) return cudaFuncSetAttribute(sel_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem_bytes());
@@ -45,8 +49,31 @@ int sel_blocks_per_sm(const Plan &p) {
 cudaError_t launch_agg_task(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
                             int final_, int has_wm, int64_t wm, int emit_on_finish, int p1_grid, int p2_grid,
                             int win_chunk, cudaStream_t st, cudaEvent_t *evs, int *launches) {
+  // rounds (State::round_off): every round re-runs the kernel sequence on the next
+  // sub-range of the task that k_task_begin chose; the last round applies finish()
+  if (p.rounds > 1) {
+    int total = 0;
+    for (int r = 0; r < p.rounds; ++r) {
+      int l = 0;
+      const bool last = r == p.rounds - 1;
+      cudaError_t e = launch_agg_round(p, q, s, tuples, n, last ? final_ : 0, has_wm, wm, emit_on_finish, p1_grid,
+                                       p2_grid, win_chunk, st, r == 0 ? evs : nullptr, &l, r);
+      if (e) return e;
+      total += l;
+    }
+    if (evs) cudaEventRecord(evs[2], st);
+    *launches = total;
+    return cudaSuccess;
+  }
+  return launch_agg_round(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, p1_grid, p2_grid, win_chunk, st,
+                          evs, launches, 0);
+}
+
+cudaError_t launch_agg_round(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
+                             int final_, int has_wm, int64_t wm, int emit_on_finish, int p1_grid, int p2_grid,
+                             int win_chunk, cudaStream_t st, cudaEvent_t *evs, int *launches, int round) {
   cudaError_t e;
-  if ((e = launch_task_begin(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, st))) return e;
+  if ((e = launch_task_begin(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, st, round))) return e;
   if ((e = launch_zero_panes(p, q, st))) return e;
   *launches = 2;
   if (evs) cudaEventRecord(evs[0], st);

@@ -9,7 +9,7 @@
 namespace sb {
 // k_task.cu
 cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
-                              int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st);
+                              int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st, int round = 0);
 cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st);
 cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);
 cudaError_t launch_win_end(const QueryDev &q, const SlotDev &s, cudaStream_t st);

@@ -106,6 +106,7 @@ struct Plan {
   // State, and the pane ring keeps the previous task's windows live
   int32_t overlap, pad9;
   int32_t win_wide, ww_grid;       // many dense keys (256 < C <= 2048): k_win_wide (k_winwide.cu), its grid
+  int32_t rounds, pad11;           // kernel rounds per task (State::round_off): time-window aggregation 3, else 1
 };
 
 // Per-query device state, updated only by kernels on the query's stream.
@@ -131,6 +132,14 @@ struct State {
   int64_t compacted_hi;           // slab mode: panes < compacted_hi have bucketed lists
   int64_t live_J0;                // overlap: first window of the task whose window phase may still run
   int64_t vh_pre_hi;              // van Herk block-prefix values are valid for panes < vh_pre_hi (k_vh_build_tile)
+  // rounds (time-window aggregation): a task is processed as up to Plan::rounds
+  // consecutive sub-ranges so that the pane ring never has to hold a time gap
+  // (reading A6: the gap's windows still get headers); every round appends its
+  // windows and rows to the task's result slot
+  int64_t round_off, round_n;     // this round's tuples: [round_off, round_off + round_n) of the task
+  int64_t slot_J0;                // first window of the task's result slot
+  int64_t row_base, hdr_base;     // rows / windows the earlier rounds of the task wrote into the slot
+  int64_t jgap_hi;                // time windows [J1, jgap_hi) are empty (they start after the last data)
 };
 
 // Per result slot metadata, copied to the host after a task.

@@ -112,6 +112,7 @@ struct saber_query {
   bool mv_stop = false;
   int64_t *d_tmp = nullptr;
   int64_t epoch_base = 0;       // look-back epoch offset across saber_query_reset
+  int64_t nbegin = 0;           // k_task_begin launches since the last reset (one epoch each)
 };
 
 static saber_status fail(saber_query *q, saber_status s, const std::string &msg) {
@@ -330,7 +331,9 @@ static saber_status size_plan(saber_query *q) {
     p.slot_words = (p.key_mode == KM_HASH ? p.C : 0) + p.C * (1 + p.nf);
     const int64_t slot_bytes = p.slot_words * 8;
     const int64_t budget = 2ll << 30;
-    int64_t need = p.K + p.L + 2;
+    // time windows: the windows closed next to a time gap read up to K-1 panes past
+    // the data while the open ones hold K+L (k_task_begin), so twice that at least
+    int64_t need = p.win_kind == WK_TIME ? 2 * (p.K + p.L) + 2 : p.K + p.L + 2;
     int64_t R;
     if (c.max_panes > 0) R = next_pow2(c.max_panes + need);
     else if (p.win_kind == WK_COUNT) R = next_pow2(need + (T + p.g - 1) / p.g + 1);
@@ -488,6 +491,11 @@ static saber_status size_plan(saber_query *q) {
     for (int i = 0; i < p.nkeys; ++i) { p.col_bytes[i] = type_bytes(p.key[i].type); p.row_bytes += p.col_bytes[i]; }
     for (int a = 0; a < p.nagg; ++a) { p.col_bytes[p.nkeys + a] = 8; p.row_bytes += 8; }
     p.win_cap = p.win_kind == WK_COUNT ? T / p.l + 4 : p.R / p.L + 4;
+    // time windows: a time gap closes many empty windows at once (headers only,
+    // reading A6): room for 2^20 of them per slot, bounded by the per-(window,
+    // slab) count array (<= 256 MiB per slot)
+    if (p.win_kind == WK_TIME)
+      p.win_cap = std::max<int64_t>(p.win_cap, std::min<int64_t>(1 << 20, (256ll << 20) / (8 * std::max(1, p.S))));
     int64_t rows_per_win = p.key_mode == KM_GLOBAL ? 1 : p.key_mode == KM_DENSE ? p.G
                            : p.bucket_mode ? std::min<int64_t>(p.s, p.G)
                            : (p.win_kind == WK_COUNT ? std::min<int64_t>(p.s, p.C * p.K) : p.C * p.K);
@@ -605,8 +613,8 @@ static saber_status alloc_query(saber_query *q) {
   // than it hides -- C3 G=64 3.00 -> 2.84 ms, C4/C5/SG1 10-35% slower)
   if (p.nagg > 0 && !p.bucket_mode && !p.slab_mode && p.key_mode != KM_HASH && getenv_flag("SABER_OVERLAP")) {
     const int64_t T = q->task_tuples;
-    const bool fits = p.win_kind == WK_COUNT ? p.R >= 2 * ((T + p.g - 1) / p.g + 2) + p.K + p.L + 2
-                                             : q->cfg.max_panes <= 0;
+    // count windows only: time windows run in rounds (gap windows, k_gap_hdr)
+    const bool fits = p.win_kind == WK_COUNT && p.R >= 2 * ((T + p.g - 1) / p.g + 2) + p.K + p.L + 2;
     if (fits) p.overlap = 1;
   }
   if (p.overlap) {
@@ -626,6 +634,14 @@ static saber_status alloc_query(saber_query *q) {
     q->p2_grid = p2_blocks_per_sm(p) * q->nsm * 2;
   } else {
     q->sel_grid = sel_blocks_per_sm(p) * q->nsm;
+  }
+  // time windows: a task runs in up to 3 rounds (State::round_off, k_task_begin) so
+  // that a time gap wider than the pane ring never fails (reading A6)
+  if (p.nagg > 0 && p.win_kind == WK_TIME && !p.overlap) {
+    const char *re = std::getenv("SABER_ROUNDS");
+    p.rounds = re ? std::max(1, std::atoi(re)) : 3;
+  } else {
+    p.rounds = 1;
   }
   if (p.lane_alt) {
     Plan &pl = q->plan_lane;
@@ -716,7 +732,10 @@ static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuple
   // look-back status words carry 24 bits of the task epoch (common.cuh lb_pack):
   // when the field wraps, stale words of an older task could match, so they are
   // cleared first (flag 0 = unpublished), after every earlier window phase
-  if (q->plan.nagg > 0 && ((q->epoch_base + q->next_task + 1) & 0xffffff) == 0) {
+  bool wraps = false;
+  for (int r = 0; r < q->plan.rounds; ++r) wraps |= ((q->epoch_base + q->nbegin + r + 1) & 0xffffff) == 0;
+  q->nbegin += q->plan.rounds;
+  if (q->plan.nagg > 0 && wraps) {
     if (q->next_task >= 1) {
       Slot &o = q->slots[(q->next_task - 1) % (int64_t)q->slots.size()];
       CK(cudaStreamWaitEvent(q->cs, o.done, 0));
@@ -1164,7 +1183,8 @@ saber_status saber_query_reset(saber_query *q, int64_t base_index, int64_t first
   q->err.clear();
   q->stats = saber_stats{};
   // task ids restart at 0; look-back epochs continue past every task run so far
-  q->epoch_base += q->next_task + 1;
+  q->epoch_base += q->nbegin + 1;
+  q->nbegin = 0;
   q->next_task = q->next_poll = 0;
   CK(launch_init_state(q->plan, q->qd, base_index, q->epoch_base, q->cs));
   CK(cudaStreamSynchronize(q->cs));

@@ -532,3 +532,47 @@ def test_release_out_of_order_no_partial_submit(saber, oracle_lib):
            "keys": exp["keys"][rowkeep], "vals": [v[rowkeep] for v in exp["vals"]], "tuples": b""}
     assert len(sub["win_id"]) > 0
     compare(spec, got, sub)
+
+
+# ------------------------------------------------------------ time gaps ---
+def _cm_with_jump(n, seed, rate, at, jump, groups=4):
+    d = gen.generate("cm", n, seed, rate=rate, groups=groups)
+    ts = gen.column(d, "cm", "ts").copy()
+    ts[at:] += jump
+    return gen.with_column(d, "cm", "ts", ts)
+
+
+@pytest.mark.parametrize("case", ["jump1e5_small_ring", "jump1e7_tumbling60", "jump1e6_w3600_s60", "jump_at_task_start"])
+def test_time_gap_wider_than_ring(saber, oracle_lib, case):
+    """A valid stream may jump in time by more than the pane ring holds (PAPER.md
+    L345-352: any discrete, non-decreasing τ).  The task runs in rounds: data before
+    the gap, the gap's windows as headers with nrows = 0 (reading A6) without
+    touching the ring, then the data after it -- with the gap inside a task, at a
+    task start, and a watermark far past the data."""
+    spec, g = workloads.c4(rate=64)
+    n = 60000
+    kw = {}
+    if case == "jump1e5_small_ring":
+        data = _cm_with_jump(n, 51, 64, 31111, 100000)
+        kw = dict(max_panes=2000)                      # ring of 4096 panes << the 10^5 s gap
+        tbs = [64 * 7777, 64 * 30000, 64 * 100000]
+    elif case == "jump1e7_tumbling60":
+        spec["window"] = workloads.time_window(60, 60)
+        data = _cm_with_jump(n, 52, 64, 20000, 10 ** 7)
+        tbs = [64 * 9999, 64 * 100000]
+    elif case == "jump1e6_w3600_s60":
+        spec["window"] = workloads.time_window(3600, 60)
+        data = _cm_with_jump(n, 53, 16, 40001, 10 ** 6)
+        kw = dict(max_panes=600)
+        tbs = [64 * 12345, 64 * 100000]
+    else:
+        data = _cm_with_jump(n, 54, 64, 30000, 50000)
+        kw = dict(max_panes=1000)
+        tbs = [64 * 30000, 64 * 15000]                 # the jump falls exactly on a task start
+    ts = gen.column(data, "cm", "ts")
+    for wm in (None, int(ts[-1]) + 5000):
+        exp = oracle_lib.run(spec, data, watermark=wm, nthreads=8)
+        for tb in tbs:
+            got = run_product(saber, spec, data, task_bytes=tb, watermark=wm, result_slots=3, **kw)
+            compare(spec, got, exp)
+    assert (exp["win_nrows"] == 0).sum() > 1000          # the gap's empty windows are there
