@@ -117,8 +117,11 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
     st->zero_lo = zlo;
     st->zero_hi = zhi;
     if (zhi > st->zeroed_hi) st->zeroed_hi = zhi;
-    meta->in_tuples = n;
-    meta->in_panes = (n > 0 && phi >= plo) ? phi - plo + 1 : 0;
+    // the task's input tuples and the panes they span, over all its rounds (the
+    // host picks the next tasks' table layout from them)
+    const int64_t inp = (n > 0 && phi >= plo) ? phi - plo + 1 : 0;
+    if (round == 0) { meta->in_tuples = n; meta->in_panes = inp; }
+    else { meta->in_tuples += n; meta->in_panes += inp; }
     const int64_t Jend = st->jgap_hi > Jn ? st->jgap_hi : Jn;
     if (Jend - st->slot_J0 > p.win_cap) {
       // more windows than the slot's headers hold: a sticky error, and nothing is

@@ -106,7 +106,7 @@ struct Plan {
   // State, and the pane ring keeps the previous task's windows live
   int32_t overlap, pad9;
   int32_t win_wide, ww_grid;       // many dense keys (256 < C <= 2048): k_win_wide (k_winwide.cu), its grid
-  int32_t rounds, pad11;           // kernel rounds per task (State::round_off): time-window aggregation 3, else 1
+  int32_t rounds, pad11;           // kernel rounds per task (State::round_off): time-window aggregation 2, else 1
 };
 
 // Per-query device state, updated only by kernels on the query's stream.

@@ -635,11 +635,11 @@ static saber_status alloc_query(saber_query *q) {
   } else {
     q->sel_grid = sel_blocks_per_sm(p) * q->nsm;
   }
-  // time windows: a task runs in up to 3 rounds (State::round_off, k_task_begin) so
+  // time windows: a task runs in up to 2 rounds (State::round_off, k_task_begin) so
   // that a time gap wider than the pane ring never fails (reading A6)
   if (p.nagg > 0 && p.win_kind == WK_TIME && !p.overlap) {
     const char *re = std::getenv("SABER_ROUNDS");
-    p.rounds = re ? std::max(1, std::atoi(re)) : 3;
+    p.rounds = re ? std::max(1, std::atoi(re)) : 2;      // one time gap per task
   } else {
     p.rounds = 1;
   }
