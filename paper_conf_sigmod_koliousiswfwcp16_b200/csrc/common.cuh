@@ -201,16 +201,18 @@ __device__ __forceinline__ uint64_t lb_pack(uint64_t epoch, uint64_t flag, uint6
 // dependent L2 round trip per predecessor: with hundreds of tiles in flight the
 // chain of a wave's last tile was tens of microseconds.
 // base0: the prefix before tile 0 (rows earlier rounds of the task already wrote).
+// published = true: the caller already published tile t's aggregate (or, for
+// t == 0, its inclusive prefix) -- the look-back only resolves.
 __device__ __forceinline__ int64_t lookback_warp(uint64_t *status, int64_t t, uint64_t epoch, uint64_t total,
-                                                 int64_t base0 = 0) {
+                                                 int64_t base0 = 0, bool published = false) {
   const int lane = threadIdx.x & 31;
   const uint64_t ep = epoch & 0xffffffull;
   const uint64_t vmask = (1ull << 38) - 1;
   if (t == 0) {
-    if (lane == 0) lb_st(&status[0], lb_pack(epoch, 2, (uint64_t)base0 + total));
+    if (lane == 0 && !published) lb_st(&status[0], lb_pack(epoch, 2, (uint64_t)base0 + total));
     return base0;
   }
-  if (lane == 0) lb_st(&status[t], lb_pack(epoch, 1, total));
+  if (lane == 0 && !published) lb_st(&status[t], lb_pack(epoch, 1, total));
   int64_t excl = 0;
   for (int64_t i = t - 1;;) {
     const int64_t idx = i - lane;

@@ -53,6 +53,21 @@ __device__ __forceinline__ int64_t bk_lds_s64(uint32_t a) {
 __device__ __forceinline__ int bk_divg(const Plan &p, int x) {     // floor(x / g), 0 <= x < 2^30
   return (int)(((uint64_t)(uint32_t)x * p.g_magic) >> p.g_mshift);
 }
+// A bucket's fill word carries kBkDirty once it holds a value that is not a
+// multiple of 2^-24 below 32 in magnitude: windows whose buckets are all clean
+// slide their state in plain fp64 exactly (every partial sum of < 2^24 such
+// values is a multiple of 2^-24 below 2^53·2^-24); windows touching a dirty
+// bucket slide it in compensated fp64 (sum + TwoSum error word, common.cuh),
+// half a slab at a time so the state still fits shared memory.
+constexpr unsigned long long kBkDirty = 1ull << 62;
+__device__ __forceinline__ bool bk_exact(uint32_t b) {
+  if ((b & 0x7fffffffu) == 0u) return true;
+  const uint32_t ex = (b >> 23) & 0xffu;
+  if (ex == 0u || ex >= 132u) return false;                 // denormal, |x| >= 32, inf, NaN
+  if (ex >= 126u) return true;                                // |x| >= 0.5: lowest bit >= 2^-24
+  const uint32_t m = (b & 0x7fffffu) | 0x800000u;
+  return (int)(__ffs(m) - 1) >= (int)(126u - ex);
+}
 __device__ __forceinline__ uint16_t *bk_keys(const Plan &p, unsigned char *bkt) { return (uint16_t *)bkt; }
 __device__ __forceinline__ float *bk_vals(const Plan &p, unsigned char *bkt) { return (float *)(bkt + p.bk_vals); }
 
@@ -71,7 +86,8 @@ k_pane_bucket(const Plan p, State *__restrict__ st, const unsigned char *__restr
   uint64_t *empty = full + kBkStages;
   int *hist = (int *)(empty + kBkStages);
   int *base = hist + kBkHist;
-  for (int e = tid; e < kBkHist; e += kBkThreads) hist[e] = 0;
+  int *hdirty = base + kBkHist;                  // (pane, slab) received a value fp64 cannot slide exactly
+  for (int e = tid; e < kBkHist; e += kBkThreads) { hist[e] = 0; hdirty[e] = 0; }
   const int64_t per = ((n + gridDim.x - 1) / gridDim.x + ST - 1) / ST * ST;
   const int64_t lo = (int64_t)blockIdx.x * per;
   const int64_t hi = lo + per < n ? lo + per : n;
@@ -145,8 +161,13 @@ k_pane_bucket(const Plan p, State *__restrict__ st, const unsigned char *__restr
       e_[u] = e;
       q_[u] = q;
       ko_[u] = key & smask;
+      bool dirty = false;
 #pragma unroll
-      for (int f = 0; f < NF; ++f) v_[u][f] = bk_lds_u32(t + foff[f]);
+      for (int f = 0; f < NF; ++f) {
+        v_[u][f] = bk_lds_u32(t + foff[f]);
+        dirty |= !bk_exact(v_[u][f]);
+      }
+      if (dirty) hdirty[e] = 1;
       r_[u] = atomicAdd(&hist[e], 1);
     }
     prev_last = bk_lds_s64(sb + (uint32_t)((ntup - 1) * tb) + tsoff);
@@ -164,7 +185,9 @@ k_pane_bucket(const Plan p, State *__restrict__ st, const unsigned char *__restr
       const int c = hist[e];
       if (c) {
         const int q = pf + e / S;
-        base[e] = (int)atomicAdd(&bcnt[((P0 + q) & Rm) * S + (e % S)], (unsigned long long)c);
+        unsigned long long *w = &bcnt[((P0 + q) & Rm) * S + (e % S)];
+        base[e] = (int)atomicAdd(w, (unsigned long long)c);     // fill count: the low 32 bits
+        if (hdirty[e]) { atomicOr(w, kBkDirty); hdirty[e] = 0; }
         hist[e] = 0;
       }
     }
@@ -353,210 +376,264 @@ __device__ __forceinline__ double bk_div(double x, double c) {
   return fma(r, fma(-c, q, x), q);
 }
 
-// window assembly, pass 2: rows
-template <int NF, int NA>
-__global__ void __launch_bounds__(512, 1)
-k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long *__restrict__ bcnt,
-           const unsigned char *__restrict__ bkt, const int64_t *__restrict__ offs, unsigned char *__restrict__ rows) {
-  extern __shared__ __align__(128) unsigned char smem[];
-  __shared__ int wn[32];
-  const int S = p.S, SB = 1 << p.bk_shift, W = p.bk_W, g = (int)p.g;
-  double *sum = (double *)smem;                               // [NF][SB]
-  double *cmp = sum + (size_t)NF * SB;                        // [NF][SB] TwoSum compensation
-  uint32_t *cnt = (uint32_t *)(smem + (size_t)16 * NF * SB);   // [SB]
-  uint16_t *slist = (uint16_t *)(cnt + SB);                   // [SB]: per-warp lists of present slots
-  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
-  if (nw <= 0) return;
-  const int64_t nitems = ((nw + W - 1) / W) * S;
+// window assembly, pass 2: rows of one (slab, window chunk) item for the keys
+// [half·SBe, (half+1)·SBe) of the slab.  COMP = false: the whole slab (SBe = SB)
+// in plain fp64 (clean buckets: exact); COMP = true: half a slab in compensated
+// fp64 (the item touches a dirty bucket).  n0[]: rows of half 0 per window, so
+// half 1 continues after them.
+template <int NF, int NA, bool COMP>
+__device__ __forceinline__ void bk_emit_item(const Plan &p, const State *__restrict__ st,
+                                             const unsigned long long *__restrict__ bcnt,
+                                             const unsigned char *__restrict__ bkt, const int64_t *__restrict__ offs,
+                                             unsigned char *__restrict__ rows, unsigned char *smem, int *wn, int *n0,
+                                             int s, int64_t ja, int64_t jb, int SBe, int half) {
+  const int S = p.S, g = (int)p.g;
+  double *sum = (double *)smem;                               // [NF][SBe]
+  double *cmp = sum + (size_t)NF * SBe;                       // [NF][SBe] TwoSum compensation (COMP)
+  uint32_t *cnt = (uint32_t *)(smem + (size_t)(COMP ? 16 : 8) * NF * SBe);   // [SBe]
+  uint16_t *slist = (uint16_t *)(cnt + SBe);                  // [SBe]: per-warp lists of present slots
+  const int64_t J0 = st->J0;
   const int64_t Rm = p.R - 1;
   const uint16_t *keys = (const uint16_t *)bkt;
   const float *vals = (const float *)(bkt + p.bk_vals);
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, nt = blockDim.x, nwarp = nt >> 5;
-  const int RS = SB / nwarp;                                  // slots per warp range (multiple of 32)
+  const int RS = SBe / nwarp;                                 // slots per warp range (multiple of 32)
   int rs_shift = 0;
   while ((1 << rs_shift) < RS) ++rs_shift;
   const unsigned lt = (1u << lane) - 1u;
   const bool pipe = p.L == 1;
+  const uint32_t klo = (uint32_t)(half * SBe);
   int akind[NA], afld[NA];
 #pragma unroll
   for (int a = 0; a < NA; ++a) { akind[a] = p.agg[a].fn; afld[a] = p.agg[a].field; }
-  auto upd = [&](uint32_t k, bool add, BkVals<NF> v) {
+  // key k of the slab -> state slot, or -1 for the other half
+  auto slot_of = [&](uint32_t k) -> int { return COMP ? ((k - klo) < (uint32_t)SBe ? (int)(k - klo) : -1) : (int)k; };
+  auto upd = [&](uint32_t k0, bool add, BkVals<NF> v) {
+    const int k = slot_of(k0);
+    if (k < 0) return;
     if (add) {
       if (atomicAdd(&cnt[k], 1u) == 0u) atomicAdd(&wn[k >> rs_shift], 1);
     } else {
       if (atomicSub(&cnt[k], 1u) == 1u) atomicSub(&wn[k >> rs_shift], 1);
     }
 #pragma unroll
-    for (int f = 0; f < NF; ++f) dd_atomic_add(&sum[f * SB + k], &cmp[f * SB + k], add ? (double)v.v[f] : -(double)v.v[f]);
+    for (int f = 0; f < NF; ++f) {
+      const double x = add ? (double)v.v[f] : -(double)v.v[f];
+      if (COMP) dd_atomic_add(&sum[f * SBe + k], &cmp[f * SBe + k], x);
+      else atomicAdd(&sum[f * SBe + k], x);
+    }
   };
+  __syncthreads();
+  for (int i = tid; i < SBe; i += nt) {
+    cnt[i] = 0;
+#pragma unroll
+    for (int f = 0; f < NF; ++f) {
+      sum[f * SBe + i] = 0.0;
+      if (COMP) cmp[f * SBe + i] = 0.0;
+    }
+  }
+  if (tid < 32) wn[tid] = 0;
+  __syncthreads();
+  auto visit = [&](int64_t b, int from, int ne, bool add) {
+    const uint16_t *kp = keys + b * g;
+    for (int e = from + tid; e < ne; e += nt) {
+      BkVals<NF> v;
+#pragma unroll
+      for (int f = 0; f < NF; ++f) v.v[f] = __ldg(vals + (b * NF + f) * g + e);
+      upd(__ldg(kp + e), add, v);
+    }
+  };
+  auto zero_key = [&](uint32_t k0) {                    // a key that left the window entirely: exact 0 sums
+    const int k = slot_of(k0);
+    if (k >= 0 && cnt[k] == 0u)
+#pragma unroll
+      for (int f = 0; f < NF; ++f) {
+        sum[f * SBe + k] = 0.0;
+        if (COMP) cmp[f * SBe + k] = 0.0;
+      }
+  };
+  auto zero_fix = [&](int64_t b, int from, int ne) {
+    const uint16_t *kp = keys + b * g;
+    for (int e = from + tid; e < ne; e += nt) zero_key(__ldg(kp + e));
+  };
+  auto pane_b = [&](int64_t q) { return (q & Rm) * S + s; };
+  for (int64_t q = ja * p.L; q < ja * p.L + p.K; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), true);
+  BkStep<NF, kEmitPF> A, B;
+  int cnl = 0, cne = 0;                 // bucket counts of the step after the prefetched one
+  if (pipe && ja + 1 < jb) {
+    int nl, ne;
+    bk_counts(p, bcnt, ja, s, nl, ne);
+    bk_prefetch<NF, true>(p, keys, vals, ja, s, nl, ne, A);
+    if (ja + 2 < jb) bk_counts(p, bcnt, ja + 1, s, cnl, cne);
+  }
+  int64_t r0n = offs[(ja - J0) * S + s];
+  __syncthreads();
+  for (int64_t j = ja; j < jb; ++j) {
+    const int64_t r0 = r0n + (COMP && half ? n0[j - ja] : 0);
+    if (j + 1 < jb) r0n = offs[(j + 1 - J0) * S + s];                                  // next window's offset
+    if (pipe && j + 2 < jb) {                                                          // in flight during the emission
+      bk_prefetch<NF, true>(p, keys, vals, j + 1, s, cnl, cne, B);
+      if (j + 3 < jb) bk_counts(p, bcnt, j + 2, s, cnl, cne);
+    }
+    // ---- emit window j, slab s: warp w owns slots [w·RS, (w+1)·RS)
+    const int wc = lane < nwarp ? wn[lane] : 0;
+    int x = wc;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(kFull, x, o);
+      if (lane >= o) x += y;
+    }
+    const int woff = __shfl_sync(kFull, x - wc, wid);
+    // column pointers at this warp's first row; rows of a window past the slot
+    // capacity are not written (k_win_scan flags SABER_ENOMEM)
+    const int tot = __shfl_sync(kFull, x, nwarp - 1);
+    if (COMP && half == 0 && tid == 0) n0[j - ja] = tot;
+    if (r0 + tot <= p.rows_cap) {
+      int32_t *kcol = (int32_t *)(rows + p.col_off[0]) + r0 + woff;
+      uint64_t *acol[NA];
+#pragma unroll
+      for (int a = 0; a < NA; ++a) acol[a] = (uint64_t *)(rows + p.col_off[1 + a]) + r0 + woff;
+      // pass 1: compact this warp's present slots into its slot list (ballot/popc;
+      // lane l reads slots 4l..4l+3 of each 128-slot block, list order is free)
+      uint16_t *sl_w = slist + wid * RS;
+      const uint4 *cw = (const uint4 *)(cnt + wid * RS) + lane;
+      int n = 0;
+      if (RS & 127) {                                       // small slabs: 32 slots per round
+        for (int o = 0; o < RS; o += 32) {
+          const uint32_t c = cnt[wid * RS + o + lane];
+          const unsigned bal = __ballot_sync(kFull, c != 0u);
+          if (c) sl_w[n + __popc(bal & lt)] = (uint16_t)(o + lane);
+          n += __popc(bal);
+        }
+      } else
+#pragma unroll 2
+      for (int o = 0; o < RS; o += 128) {
+        const uint4 c4 = cw[o >> 2];
+        const uint32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const unsigned bal = __ballot_sync(kFull, cc[u] != 0u);
+          if (cc[u]) sl_w[n + __popc(bal & lt)] = (uint16_t)(o + 4 * lane + u);
+          n += __popc(bal);
+        }
+      }
+      __syncwarp();
+      // pass 2: one row per lane, consecutive rows across the warp (coalesced stores)
+      const int32_t kb = (s << p.bk_shift) + (int32_t)klo + wid * RS;
+#pragma unroll 4
+      for (int i = lane; i < n; i += 32) {
+        const int sl = sl_w[i];
+        const uint32_t c = cnt[wid * RS + sl];
+        kcol[i] = kb + sl;
+        double sv[NF > 0 ? NF : 1];
+#pragma unroll
+        for (int f = 0; f < NF; ++f)
+          sv[f] = COMP ? sum[f * SBe + wid * RS + sl] + cmp[f * SBe + wid * RS + sl] : sum[f * SBe + wid * RS + sl];
+        const double dc = (double)c;
+#pragma unroll
+        for (int a = 0; a < NA; ++a) {
+          double xv = 0.0;
+#pragma unroll
+          for (int f = 0; f < NF; ++f) xv = afld[a] == f ? sv[f] : xv;
+          const uint64_t bits = akind[a] == AG_COUNT ? (uint64_t)c
+                                : akind[a] == AG_SUM ? (uint64_t)__double_as_longlong(xv)
+                                                     : (uint64_t)__double_as_longlong(bk_div(xv, dc));
+          acol[a][i] = bits;
+        }
+      }
+      __syncwarp();
+    }
+    if (j + 1 >= jb) break;
+    __syncthreads();
+    // ---- slide to window j+1
+    if (pipe) {
+#pragma unroll
+      for (int u = 0; u < kEmitPF; ++u) {
+        const int e = tid + u * nt;
+        if (e < A.nl) upd(A.kl[u], false, A.vl[u]);
+        if (e < A.ne) upd(A.ke[u], true, A.ve[u]);
+      }
+      visit(A.bl, kEmitPF * nt, A.nl, false);
+      visit(A.be, kEmitPF * nt, A.ne, true);
+    } else {
+      for (int64_t q = j * p.L; q < (j + 1) * p.L; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), false);
+      for (int64_t q = j * p.L + p.K; q < (j + 1) * p.L + p.K; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), true);
+    }
+    __syncthreads();
+    // zero-fix writes sums of keys with count 0 only; the next emission reads keys
+    // with count > 0 only, so no barrier separates them
+    if (pipe) {
+#pragma unroll
+      for (int u = 0; u < kEmitPF; ++u) {
+        const int e = tid + u * nt;
+        if (e < A.nl) zero_key(A.kl[u]);
+      }
+      zero_fix(A.bl, kEmitPF * nt, A.nl);
+      A = B;
+    } else {
+      for (int64_t q = j * p.L; q < (j + 1) * p.L; ++q) zero_fix(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)));
+    }
+  }
+}
+
+// COMP = false emits the clean items, COMP = true the dirty ones (two launches,
+// each skipping the other kind: one register allocation per path)
+template <int NF, int NA, bool COMP>
+__global__ void __launch_bounds__(512, 1)
+k_bkt_emit(const Plan p, const State *__restrict__ st, const unsigned long long *__restrict__ bcnt,
+           const unsigned char *__restrict__ bkt, const int64_t *__restrict__ offs, unsigned char *__restrict__ rows) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ int wn[32];
+  const int S = p.S, SB = 1 << p.bk_shift, W = p.bk_W;
+  // dirty items: rows of half 0 per window, after the half-slab state
+  int *n0 = (int *)(smem + (size_t)(SB / 2) * (6 + 16 * NF));
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  if (nw <= 0) return;
+  const int64_t nitems = ((nw + W - 1) / W) * S;
+  const int64_t Rm = p.R - 1;
+  const bool always = p.s >= (1ll << 24);       // exactness bound of clean buckets: < 2^24 values per key
   for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
     const int64_t chunk = item / S;
     const int s = (int)(item % S);
     const int64_t ja = J0 + chunk * W;
     const int64_t jb = ja + W < J1 ? ja + W : J1;
-    __syncthreads();
-    for (int i = tid; i < SB; i += nt) {
-      cnt[i] = 0;
-#pragma unroll
-      for (int f = 0; f < NF; ++f) sum[f * SB + i] = cmp[f * SB + i] = 0.0;
-    }
-    if (tid < 32) wn[tid] = 0;
-    __syncthreads();
-    auto visit = [&](int64_t b, int from, int ne, bool add) {
-      const uint16_t *kp = keys + b * g;
-      for (int e = from + tid; e < ne; e += nt) {
-        BkVals<NF> v;
-#pragma unroll
-        for (int f = 0; f < NF; ++f) v.v[f] = __ldg(vals + (b * NF + f) * g + e);
-        upd(__ldg(kp + e), add, v);
-      }
-    };
-    auto zero_fix = [&](int64_t b, int from, int ne) {   // keys that left the window entirely: exact 0 sums
-      const uint16_t *kp = keys + b * g;
-      for (int e = from + tid; e < ne; e += nt) {
-        const uint32_t k = __ldg(kp + e);
-        if (cnt[k] == 0u)
-#pragma unroll
-          for (int f = 0; f < NF; ++f) sum[f * SB + k] = cmp[f * SB + k] = 0.0;
-      }
-    };
-    auto pane_b = [&](int64_t q) { return (q & Rm) * S + s; };
-    for (int64_t q = ja * p.L; q < ja * p.L + p.K; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), true);
-    BkStep<NF, kEmitPF> A, B;
-    int cnl = 0, cne = 0;                 // bucket counts of the step after the prefetched one
-    if (pipe && ja + 1 < jb) {
-      int nl, ne;
-      bk_counts(p, bcnt, ja, s, nl, ne);
-      bk_prefetch<NF, true>(p, keys, vals, ja, s, nl, ne, A);
-      if (ja + 2 < jb) bk_counts(p, bcnt, ja + 1, s, cnl, cne);
-    }
-    int64_t r0n = offs[(ja - J0) * S + s];
-    __syncthreads();
-    for (int64_t j = ja; j < jb; ++j) {
-      const int64_t r0 = r0n;
-      if (j + 1 < jb) r0n = offs[(j + 1 - J0) * S + s];                                  // next window's offset
-      if (pipe && j + 2 < jb) {                                                          // in flight during the emission
-        bk_prefetch<NF, true>(p, keys, vals, j + 1, s, cnl, cne, B);
-        if (j + 3 < jb) bk_counts(p, bcnt, j + 2, s, cnl, cne);
-      }
-      // ---- emit window j, slab s: warp w owns slots [w·RS, (w+1)·RS)
-      const int wc = lane < nwarp ? wn[lane] : 0;
-      int x = wc;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(kFull, x, o);
-        if (lane >= o) x += y;
-      }
-      const int woff = __shfl_sync(kFull, x - wc, wid);
-      // column pointers at this warp's first row; rows of a window past the slot
-      // capacity are not written (k_win_scan flags SABER_ENOMEM)
-      const int tot = __shfl_sync(kFull, x, nwarp - 1);
-      if (r0 + tot <= p.rows_cap) {
-        int32_t *kcol = (int32_t *)(rows + p.col_off[0]) + r0 + woff;
-        uint64_t *acol[NA];
-#pragma unroll
-        for (int a = 0; a < NA; ++a) acol[a] = (uint64_t *)(rows + p.col_off[1 + a]) + r0 + woff;
-        // pass 1: compact this warp's present slots into its slot list (ballot/popc;
-        // lane l reads slots 4l..4l+3 of each 128-slot block, list order is free)
-        uint16_t *sl_w = slist + wid * RS;
-        const uint4 *cw = (const uint4 *)(cnt + wid * RS) + lane;
-        int n = 0;
-        if (RS & 127) {                                       // small slabs: 32 slots per round
-          for (int o = 0; o < RS; o += 32) {
-            const uint32_t c = cnt[wid * RS + o + lane];
-            const unsigned bal = __ballot_sync(kFull, c != 0u);
-            if (c) sl_w[n + __popc(bal & lt)] = (uint16_t)(o + lane);
-            n += __popc(bal);
-          }
-        } else
-#pragma unroll 2
-        for (int o = 0; o < RS; o += 128) {
-          const uint4 c4 = cw[o >> 2];
-          const uint32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
-#pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            const unsigned bal = __ballot_sync(kFull, cc[u] != 0u);
-            if (cc[u]) sl_w[n + __popc(bal & lt)] = (uint16_t)(o + 4 * lane + u);
-            n += __popc(bal);
-          }
-        }
-        __syncwarp();
-        // pass 2: one row per lane, consecutive rows across the warp (coalesced stores)
-        const int32_t kb = (s << p.bk_shift) + wid * RS;
-#pragma unroll 4
-        for (int i = lane; i < n; i += 32) {
-          const int sl = sl_w[i];
-          const uint32_t c = cnt[wid * RS + sl];
-          kcol[i] = kb + sl;
-          double sv[NF > 0 ? NF : 1];
-#pragma unroll
-          for (int f = 0; f < NF; ++f) sv[f] = sum[f * SB + wid * RS + sl] + cmp[f * SB + wid * RS + sl];
-          const double dc = (double)c;
-#pragma unroll
-          for (int a = 0; a < NA; ++a) {
-            double xv = 0.0;
-#pragma unroll
-            for (int f = 0; f < NF; ++f) xv = afld[a] == f ? sv[f] : xv;
-            const uint64_t bits = akind[a] == AG_COUNT ? (uint64_t)c
-                                  : akind[a] == AG_SUM ? (uint64_t)__double_as_longlong(xv)
-                                                       : (uint64_t)__double_as_longlong(bk_div(xv, dc));
-            acol[a][i] = bits;
-          }
-        }
-        __syncwarp();
-      }
-      if (j + 1 >= jb) break;
-      __syncthreads();
-      // ---- slide to window j+1
-      if (pipe) {
-#pragma unroll
-        for (int u = 0; u < kEmitPF; ++u) {
-          const int e = tid + u * nt;
-          if (e < A.nl) upd(A.kl[u], false, A.vl[u]);
-          if (e < A.ne) upd(A.ke[u], true, A.ve[u]);
-        }
-        visit(A.bl, kEmitPF * nt, A.nl, false);
-        visit(A.be, kEmitPF * nt, A.ne, true);
-      } else {
-        for (int64_t q = j * p.L; q < (j + 1) * p.L; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), false);
-        for (int64_t q = j * p.L + p.K; q < (j + 1) * p.L + p.K; ++q) visit(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)), true);
-      }
-      __syncthreads();
-      // zero-fix writes sums of keys with count 0 only; the next emission reads keys
-      // with count > 0 only, so no barrier separates them
-      if (pipe) {
-#pragma unroll
-        for (int u = 0; u < kEmitPF; ++u) {
-          const int e = tid + u * nt;
-          if (e < A.nl && cnt[A.kl[u]] == 0u)
-#pragma unroll
-            for (int f = 0; f < NF; ++f) sum[f * SB + A.kl[u]] = cmp[f * SB + A.kl[u]] = 0.0;
-        }
-        zero_fix(A.bl, kEmitPF * nt, A.nl);
-        A = B;
-      } else {
-        for (int64_t q = j * p.L; q < (j + 1) * p.L; ++q) zero_fix(pane_b(q), 0, (int)__ldg(bcnt + pane_b(q)));
-      }
+    // does any bucket of the item's panes hold a value plain fp64 cannot slide exactly?
+    bool dirty = always;
+    for (int64_t q = ja * p.L + threadIdx.x; q < (jb - 1) * p.L + p.K; q += blockDim.x)
+      dirty |= (__ldg(bcnt + (q & Rm) * S + s) & kBkDirty) != 0;
+    dirty = __syncthreads_or(dirty);
+    if (dirty != COMP) continue;
+    if (!COMP) {
+      bk_emit_item<NF, NA, false>(p, st, bcnt, bkt, offs, rows, smem, wn, n0, s, ja, jb, SB, 0);
+    } else {
+      for (int h = 0; h < 2; ++h)
+        bk_emit_item<NF, NA, true>(p, st, bcnt, bkt, offs, rows, smem, wn, n0, s, ja, jb, SB / 2, h);
     }
   }
 }
 
 // ---------------------------------------------------------------------------
 // host side
-int bk_scan_smem() { return kBkStages * kBkStageBytes + 2 * kBkStages * 8 + 2 * kBkHist * 4; }
-int bk_emit_smem(const Plan &p) { return (1 << p.bk_shift) * (6 + 16 * p.nf); }
+int bk_scan_smem() { return kBkStages * kBkStageBytes + 2 * kBkStages * 8 + 3 * kBkHist * 4; }
+// clean items: SB·(count + slot list + nf sums); dirty items: SB/2·(count + list + nf sums + nf compensations)
+int bk_emit_smem(const Plan &p) {
+  const int SB = 1 << p.bk_shift;
+  const int clean = SB * (6 + 8 * p.nf), dirty = (SB / 2) * (6 + 16 * p.nf) + 4 * 1024;
+  return clean > dirty ? clean : dirty;
+}
 int bk_count_smem(const Plan &p) { return (1 << p.bk_shift) * 4; }
 
 static void *bk_scan_kernel(const Plan &p) {
   return p.nf == 0 ? (void *)k_pane_bucket<0> : p.nf == 1 ? (void *)k_pane_bucket<1> : (void *)k_pane_bucket<2>;
 }
-template <int NF>
+template <int NF, bool C>
 static void *bk_emit_nf(int na) {
-  return na == 1 ? (void *)k_bkt_emit<NF, 1> : na == 2 ? (void *)k_bkt_emit<NF, 2> : na == 3 ? (void *)k_bkt_emit<NF, 3>
-                                                                                         : (void *)k_bkt_emit<NF, 4>;
+  return na == 1 ? (void *)k_bkt_emit<NF, 1, C> : na == 2 ? (void *)k_bkt_emit<NF, 2, C>
+       : na == 3 ? (void *)k_bkt_emit<NF, 3, C> : (void *)k_bkt_emit<NF, 4, C>;
 }
+template <bool C>
 static void *bk_emit_kernel(const Plan &p) {
-  return p.nf == 0 ? bk_emit_nf<0>(p.nagg) : p.nf == 1 ? bk_emit_nf<1>(p.nagg) : bk_emit_nf<2>(p.nagg);
+  return p.nf == 0 ? bk_emit_nf<0, C>(p.nagg) : p.nf == 1 ? bk_emit_nf<1, C>(p.nagg) : bk_emit_nf<2, C>(p.nagg);
 }
 
 cudaError_t bk_set_attributes(const Plan &p) {
@@ -564,7 +641,9 @@ cudaError_t bk_set_attributes(const Plan &p) {
   if (e) return e;
   e = cudaFuncSetAttribute((void *)k_bkt_count, cudaFuncAttributeMaxDynamicSharedMemorySize, bk_count_smem(p));
   if (e) return e;
-  return cudaFuncSetAttribute(bk_emit_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, bk_emit_smem(p));
+  e = cudaFuncSetAttribute(bk_emit_kernel<false>(p), cudaFuncAttributeMaxDynamicSharedMemorySize, bk_emit_smem(p));
+  if (e) return e;
+  return cudaFuncSetAttribute(bk_emit_kernel<true>(p), cudaFuncAttributeMaxDynamicSharedMemorySize, bk_emit_smem(p));
 }
 
 int bk_scan_blocks_per_sm(const Plan &p) {
@@ -590,7 +669,11 @@ cudaError_t launch_bucket_windows(const Plan &p, const QueryDev &q, const SlotDe
   cudaError_t e = launch_win_scan(p, q, s, st);
   if (e) return e;
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&bc, (void *)&q.bkt, (void *)&s.counts, (void *)&s.rows};
-  return cudaLaunchKernel(bk_emit_kernel(p), dim3(nsm * p.bk_ctas), dim3(p.bk_threads), args, (size_t)bk_emit_smem(p), st);
+  e = cudaLaunchKernel(bk_emit_kernel<false>(p), dim3(nsm * p.bk_ctas), dim3(p.bk_threads), args,
+                       (size_t)bk_emit_smem(p), st);
+  if (e) return e;
+  return cudaLaunchKernel(bk_emit_kernel<true>(p), dim3(nsm * p.bk_ctas), dim3(p.bk_threads), args,
+                          (size_t)bk_emit_smem(p), st);
 }
 
 }  // namespace sb

@@ -86,7 +86,7 @@ cudaError_t launch_agg_round(const Plan &p, const QueryDev &q, const SlotDev &s,
   if (evs) cudaEventRecord(evs[1], st);
   if (p.bucket_mode) {
     if ((e = launch_bucket_windows(p, q, s, p2_grid, st))) return e;
-    *launches += 3;
+    *launches += 4;     // k_bkt_count, k_win_scan, k_bkt_emit (clean items), k_bkt_emit (dirty items)
   } else if (p.slab_mode) {
     if ((e = launch_windows_slab(p, q, s, false, p2_grid, win_chunk, st))) return e;
     if ((e = launch_win_scan(p, q, s, st))) return e;
@@ -155,7 +155,7 @@ cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &
   if (evs) cudaEventRecord(evs[1], st);
   if ((e = launch_carry(p, q, tuples, st))) return e;
   if ((e = launch_task_end(p, q, s, st))) return e;
-  *launches = 6;     // k_task_begin, k_select, k_select_fix, k_sel_hdr, k_carry, k_task_end
+  *launches = 5;     // k_task_begin, k_select, k_sel_hdr, k_carry, k_task_end
   if (evs) cudaEventRecord(evs[2], st);
   return cudaGetLastError();
 }
