@@ -23,16 +23,19 @@ struct QueryDev {
   uint64_t *vh_suf;         // van Herk block-suffix arrays
   uint64_t *clist;          // slab mode: per pane slot, entries bucketed by key range
   int32_t *coff;            // slab mode: per pane slot, S+1 bucket offsets
+  unsigned char *sel_stage; // σ/π: per-CTA compacted rows before the final placement
+  int64_t *cta_cnt;         // σ/π: rows per CTA
   int64_t *pane_ts;         // R
   uint64_t *tile_status;    // IStream look-back
   int64_t tile_status_cap;
   unsigned char *carry[2];  // IStream raw tail
   int64_t carry_cap;        // tuples
   int *tile_ctr;
-  // σ/π (IStream) window headers: per closed window the global row rank of its
-  // first new tuple, and τ at window starts j·l (count windows; ring of
-  // ts_mask+1 entries indexed by j)
+  // σ/π (IStream) window headers: per closed window the (CTA, CTA-relative row
+  // rank) of its first new tuple, each CTA's global row base, and τ at window
+  // starts j·l (count windows; ring of ts_mask+1 entries indexed by j)
   int64_t *ihdr_tmp;
+  int64_t *cta_base;
   int64_t *win_ts;
   int64_t ts_mask;
   unsigned char *bkt;       // bucket mode: [R][S][g] u16 key offsets, then [R][S][nf][g] f32 values
@@ -62,7 +65,6 @@ int p1_smem_bytes(const Plan &p);
 int p1_blocks_per_sm(const Plan &p);
 int p2_blocks_per_sm(const Plan &p);
 int sel_blocks_per_sm(const Plan &p);
-int64_t sel_tiles(const Plan &p, int64_t cover);   // compaction tiles of a cover of `cover` tuples
 int bk_scan_blocks_per_sm(const Plan &p);
 bool wb_usable(const Plan &p);
 bool ww_usable(const Plan &p);

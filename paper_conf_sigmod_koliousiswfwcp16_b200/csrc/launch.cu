@@ -155,7 +155,7 @@ cudaError_t launch_select_task(const Plan &p, const QueryDev &q, const SlotDev &
   if (evs) cudaEventRecord(evs[1], st);
   if ((e = launch_carry(p, q, tuples, st))) return e;
   if ((e = launch_task_end(p, q, s, st))) return e;
-  *launches = 5;     // k_task_begin, k_select, k_sel_hdr, k_carry, k_task_end
+  *launches = 6;     // k_task_begin, k_select, k_select_fix, k_sel_hdr, k_carry, k_task_end
   if (evs) cudaEventRecord(evs[2], st);
   return cudaGetLastError();
 }

@@ -48,7 +48,6 @@ cudaError_t launch_windows_wide(const Plan &p, const QueryDev &q, const SlotDev 
 // k_select.cu
 void *sel_kernel(const Plan &p);
 int sel_smem_bytes();
-int64_t sel_tiles(const Plan &p, int64_t cover);
 cudaError_t launch_select(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int grid,
                           cudaStream_t st);
 }  // namespace sb

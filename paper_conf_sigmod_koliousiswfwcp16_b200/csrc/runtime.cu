@@ -570,10 +570,9 @@ static saber_status alloc_query(saber_query *q) {
     q->qd.carry_cap = p.carry_cap;
     CK(cudaMalloc(&q->qd.carry[0], (size_t)p.carry_cap * p.tuple_bytes));
     CK(cudaMalloc(&q->qd.carry[1], (size_t)p.carry_cap * p.tuple_bytes));
-    // look-back status of the single-pass compaction: one entry per tile of a cover
-    q->qd.tile_status_cap = sel_tiles(p, q->task_tuples + p.carry_cap) + 16;
-    CK(cudaMalloc(&q->qd.tile_status, (size_t)q->qd.tile_status_cap * 8));
-    CK(cudaMemset(q->qd.tile_status, 0, (size_t)q->qd.tile_status_cap * 8));
+    CK(cudaMalloc(&q->qd.sel_stage, (size_t)p.rows_cap * p.out_row_words * 4 + 16));
+    CK(cudaMalloc(&q->qd.cta_cnt, 8192 * sizeof(int64_t)));
+    CK(cudaMalloc(&q->qd.cta_base, 8192 * sizeof(int64_t)));
     CK(cudaMalloc(&q->qd.ihdr_tmp, (size_t)(p.win_cap + 1) * sizeof(int64_t)));
     // τ at window starts j·l: windows from J0 up to the cover's end (< win_cap + s/l + 2)
     const int64_t nts = p.win_kind == WK_COUNT ? next_pow2(p.win_cap + p.s / p.l + 8) : 1;
@@ -736,7 +735,7 @@ static saber_status enqueue_task(saber_query *q, const void *dev, int64_t ntuple
   bool wraps = false;
   for (int r = 0; r < q->plan.rounds; ++r) wraps |= ((q->epoch_base + q->nbegin + r + 1) & 0xffffff) == 0;
   q->nbegin += q->plan.rounds;
-  if (wraps) {
+  if (q->plan.nagg > 0 && wraps) {
     if (q->next_task >= 1) {
       Slot &o = q->slots[(q->next_task - 1) % (int64_t)q->slots.size()];
       CK(cudaStreamWaitEvent(q->cs, o.done, 0));
@@ -882,7 +881,7 @@ void saber_query_destroy(saber_query *q) {
   for (auto &r : q->registered)
     if (std::find(q->prereg.begin(), q->prereg.end(), r.first) == q->prereg.end()) cudaHostUnregister(r.first);
   cudaFree(q->qd.st); cudaFree(q->qd.table); cudaFree(q->qd.vh_pre); cudaFree(q->qd.vh_suf);
-  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.bkt); cudaFree(q->qd.ihdr_tmp); cudaFree(q->qd.win_ts); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
+  cudaFree(q->qd.clist); cudaFree(q->qd.coff); cudaFree(q->qd.bkt); cudaFree(q->qd.sel_stage); cudaFree(q->qd.cta_cnt); cudaFree(q->qd.cta_base); cudaFree(q->qd.ihdr_tmp); cudaFree(q->qd.win_ts); cudaFree(q->qd.pane_ts); cudaFree(q->qd.tile_status);
   cudaFree(q->qd.carry[0]); cudaFree(q->qd.carry[1]); cudaFree(q->qd.tile_ctr); cudaFree(q->d_tmp);
   if (q->cs) cudaStreamDestroy(q->cs);
   if (q->h2d) cudaStreamDestroy(q->h2d);
