@@ -71,7 +71,7 @@ typedef struct {
 } saber_window;
 
 typedef enum { SABER_LT = 0, SABER_LE, SABER_GT, SABER_GE, SABER_EQ, SABER_NE } saber_cmp;
-/* σ term `col op const` (conjunction of all terms, L1320-1322).  The constant
+/* σ term `col op const` (conjunction of up to 64 terms, L1320-1322; SELECT_n).  The constant
  * is ival for integer columns and fval for float columns.  In HAVING, col is
  * the index of an aggregate and the constant is ival for integer results
  * (COUNT, SUM/MIN/MAX of int columns) and fval otherwise. */

@@ -56,7 +56,7 @@ class _Query(C.Structure):
     _fields_ = [("tuple_bytes", C.c_int32), ("ts_off", C.c_int32),
                 ("win_kind", C.c_int32), ("pad", C.c_int32),
                 ("size", C.c_int64), ("slide", C.c_int64), ("origin", C.c_int64),
-                ("npred", C.c_int32), ("pred", _Pred * 16),
+                ("npred", C.c_int32), ("pred", _Pred * 64),
                 ("nproj", C.c_int32), ("proj", _Col * 16),
                 ("nagg", C.c_int32), ("agg", _Agg * 8),
                 ("nkeys", C.c_int32), ("key", _Key * 4),

@@ -188,7 +188,7 @@ int64_t closed_windows(const oq_query *q, const std::vector<int64_t> &tau, int64
 
 int validate(const oq_query *q, const uint8_t *tuples, int64_t n, std::vector<int64_t> &tau) {
   if (q->size < 1 || q->slide < 1 || q->tuple_bytes < 8) return OQ_EINVAL;
-  if (q->nagg > 8 || q->nkeys > 4 || q->npred > 16 || q->nproj > 16 || q->nhave > 8) return OQ_EINVAL;
+  if (q->nagg > 8 || q->nkeys > 4 || q->npred > 64 || q->nproj > 16 || q->nhave > 8) return OQ_EINVAL;
   for (int k = 0; k < q->nkeys; ++k) if (q->key[k].div == 0) return OQ_EINVAL;
   tau.resize(n);
   for (int64_t i = 0; i < n; ++i) {

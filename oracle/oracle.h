@@ -40,7 +40,7 @@ typedef struct {
   int32_t tuple_bytes, ts_off;
   int32_t win_kind; int32_t pad;
   int64_t size, slide, origin;
-  int32_t npred;  oq_pred pred[16];
+  int32_t npred;  oq_pred pred[64];
   int32_t nproj;  oq_col  proj[16];
   int32_t nagg;   oq_agg  agg[8];
   int32_t nkeys;  oq_key  key[4];

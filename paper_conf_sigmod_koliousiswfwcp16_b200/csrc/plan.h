@@ -15,7 +15,7 @@
 
 namespace sb {
 
-constexpr int kMaxPred = 16, kMaxProj = 16, kMaxAgg = 8, kMaxKey = 4, kMaxField = 8, kMaxHave = 8;
+constexpr int kMaxPred = 64, kMaxProj = 16, kMaxAgg = 8, kMaxKey = 4, kMaxField = 8, kMaxHave = 8;
 constexpr int kMaxCols = 12;
 constexpr int kMaxTupleWords = 64;      // tuples up to 256 bytes
 

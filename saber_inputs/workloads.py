@@ -54,8 +54,8 @@ def c2(sel=0.5, npred=1, n=1 << 25):
     theta = int(round(sel * 2 ** 31))
     where = [("a3", "<", theta)]
     extra = ["a4", "a5", "a6", "a2"]
-    for k in range(npred - 1):          # always-true terms: same selectivity, more ALU
-        where.append((extra[k % len(extra)], ">=", 0))
+    for k in range(npred - 1):          # always-true terms: same selectivity, more ALU (SELECT_n, Fig. 10a)
+        where.append((extra[k % len(extra)], ">=", -k))
     return (_spec("syn", count_window(1024, 64), where=where, project=["ts", "a1", "a2"]),
             {"kind": "syn", "n": n, "seed": 2, "rate": 1, "groups": 64})
 

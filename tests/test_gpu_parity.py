@@ -576,3 +576,11 @@ def test_time_gap_wider_than_ring(saber, oracle_lib, case):
             got = run_product(saber, spec, data, task_bytes=tb, watermark=wm, result_slots=3, **kw)
             compare(spec, got, exp)
     assert (exp["win_nrows"] == 0).sum() > 1000          # the gap's empty windows are there
+
+
+@pytest.mark.parametrize("npred", [16, 64])
+def test_select_n_predicates(saber, oracle_lib, npred):
+    """SELECT_n (Fig. 10a): n-1 extra always-true terms, same selectivity."""
+    spec, g = workloads.c2(sel=0.3, npred=npred)
+    data = gen.generate("syn", 1 << 18, g["seed"], rate=1)
+    check(saber, oracle_lib, spec, data, task_bytes=(1 << 20) + 32 * 13)
