@@ -98,6 +98,9 @@ def lib():
         _lib.oq_num_windows.restype = C.c_int64
         _lib.oq_num_windows.argtypes = [C.POINTER(_Query), C.c_void_p, C.c_int64, C.c_int64, C.c_int32]
         _lib.oq_free.argtypes = [C.POINTER(_Result)]
+        _lib.oq_join_run.restype = C.c_int32
+        _lib.oq_join_run.argtypes = [C.POINTER(_Join), C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_int32,
+                                     C.POINTER(_Result)]
     return _lib
 
 
@@ -144,6 +147,19 @@ def _marshal(spec) -> _Query:
         q.have[i].fval = float(const)
         q.have[i].ival = int(const) if float(const) == int(const) else 0
     return q
+
+
+class _JPred(C.Structure):
+    _fields_ = [("off1", C.c_int32), ("type1", C.c_int32), ("op", C.c_int32), ("off2", C.c_int32),
+                ("type2", C.c_int32), ("pad", C.c_int32)]
+
+
+class _Join(C.Structure):
+    _fields_ = [("tuple_bytes1", C.c_int32), ("tuple_bytes2", C.c_int32), ("ts_off1", C.c_int32),
+                ("pad", C.c_int32), ("size", C.c_int64), ("slide", C.c_int64),
+                ("npred", C.c_int32), ("pred", _JPred * 64),
+                ("nproj1", C.c_int32), ("proj1", _Col * 16),
+                ("nproj2", C.c_int32), ("proj2", _Col * 16)]
 
 
 class OracleError(RuntimeError):
@@ -206,3 +222,44 @@ def num_windows(spec, data, watermark=None):
     n = buf.size // q.tuple_bytes
     return L.oq_num_windows(C.byref(q), buf.ctypes.data if buf.size else None, n,
                             0 if watermark is None else int(watermark), 0 if watermark is None else 1)
+
+
+def join_run(jspec, data1, data2, nthreads=1):
+    """Windowed θ-join of two streams (oracle.h oq_join_run).  ``jspec``:
+    schema1, schema2, window (count), theta [(col1, op, col2)], project1, project2.
+    Returns win_id, win_ts, win_nrows, win_rowoff and ``tuples`` (pair rows)."""
+    L = lib()
+    q = _Join()
+    s1, s2 = jspec["schema1"], jspec["schema2"]
+    q.tuple_bytes1, q.tuple_bytes2 = s1["tuple_bytes"], s2["tuple_bytes"]
+    q.ts_off1 = _colinfo({"schema": s1}, s1["ts"])[0]
+    w = jspec["window"]
+    q.size, q.slide = w["size"], w["slide"]
+    q.npred = len(jspec.get("theta", []))
+    for i, (c1, op, c2) in enumerate(jspec.get("theta", [])):
+        q.pred[i].off1, q.pred[i].type1 = _colinfo({"schema": s1}, c1)
+        q.pred[i].off2, q.pred[i].type2 = _colinfo({"schema": s2}, c2)
+        q.pred[i].op = OPS[op]
+    q.nproj1 = len(jspec["project1"])
+    for i, c in enumerate(jspec["project1"]):
+        q.proj1[i].off, q.proj1[i].type = _colinfo({"schema": s1}, c)
+    q.nproj2 = len(jspec["project2"])
+    for i, c in enumerate(jspec["project2"]):
+        q.proj2[i].off, q.proj2[i].type = _colinfo({"schema": s2}, c)
+    b1 = np.ascontiguousarray(np.frombuffer(data1, np.uint8) if isinstance(data1, (bytes, bytearray)) else data1)
+    b2 = np.ascontiguousarray(np.frombuffer(data2, np.uint8) if isinstance(data2, (bytes, bytearray)) else data2)
+    res = _Result()
+    err = L.oq_join_run(C.byref(q), b1.ctypes.data if b1.size else None, b1.size // q.tuple_bytes1,
+                        b2.ctypes.data if b2.size else None, b2.size // q.tuple_bytes2, int(nthreads), C.byref(res))
+    try:
+        if err != 0:
+            raise OracleError(err)
+        nw = res.nwin
+
+        def arr(p, cnt):
+            return np.ctypeslib.as_array(p, shape=(cnt,)).astype(np.int64).copy() if cnt else np.zeros(0, np.int64)
+        return {"win_id": arr(res.win_id, nw), "win_ts": arr(res.win_ts, nw), "win_nrows": arr(res.win_nrows, nw),
+                "win_rowoff": arr(res.win_rowoff, nw), "row_bytes": res.row_bytes,
+                "tuples": bytes(np.ctypeslib.as_array(res.out, shape=(res.out_bytes,))) if res.out_bytes else b""}
+    finally:
+        L.oq_free(C.byref(res))

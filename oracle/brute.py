@@ -107,3 +107,39 @@ def brute(spec, data, watermark=None):
                 rows.append((key, vals))
         result.append((j, ts, rows))
     return result
+
+
+def brute_join(jspec, d1, d2):
+    """Windowed θ-join, written independently of oracle.cpp: 1-based windows
+    <t_k..t_m> on both streams (L370-372), a Python set of matching position
+    pairs per window, rows sorted by (a, b) only at the end."""
+    s1, s2 = jspec["schema1"], jspec["schema2"]
+    n1, n2 = len(d1) // s1["tuple_bytes"], len(d2) // s2["tuple_bytes"]
+    t1 = [bytes(d1[i * s1["tuple_bytes"]:(i + 1) * s1["tuple_bytes"]]) for i in range(n1)]
+    t2 = [bytes(d2[i * s2["tuple_bytes"]:(i + 1) * s2["tuple_bytes"]]) for i in range(n2)]
+    sp1, sp2 = {"schema": s1}, {"schema": s2}
+    w = jspec["window"]
+    s, l = w["size"], w["slide"]
+    out = []
+    k, j = 1, 0
+    while k + s - 1 <= min(n1, n2):
+        pos = range(k - 1, k + s - 1)
+        pairs = set()
+        for a in pos:
+            for b in pos:
+                ok = True
+                for c1, op, c2 in jspec.get("theta", []):
+                    x, y = _get(sp1, t1[a], c1), _get(sp2, t2[b], c2)
+                    if not _OPS[op](x, y):
+                        ok = False
+                        break
+                if ok:
+                    pairs.add((a, b))
+        rows = []
+        for a, b in sorted(pairs):
+            r = b"".join(t1[a][_col(sp1, c)[1]:_col(sp1, c)[1] + _W[_col(sp1, c)[0]]] for c in jspec["project1"])
+            r += b"".join(t2[b][_col(sp2, c)[1]:_col(sp2, c)[1] + _W[_col(sp2, c)[0]]] for c in jspec["project2"])
+            rows.append(r)
+        out.append((j, _get(sp1, t1[k - 1], s1["ts"]), rows))
+        k, j = k + l, j + 1
+    return out

@@ -287,3 +287,91 @@ extern "C" void oq_free(oq_result *r) {
   std::free(r->keys); std::free(r->vals); std::free(r->out);
   std::memset(r, 0, sizeof(*r));
 }
+
+// ---------------------------------------------------------------------------
+// Windowed θ-join (oracle.h): window j = W1_j ⋈θ W2_j, both count windows
+// [j·l, j·l+s); every pair tested literally, in (a, b) order.
+namespace {
+bool jpred_ok(const oq_join *q, const uint8_t *a, const uint8_t *b) {
+  for (int p = 0; p < q->npred; ++p) {
+    const oq_jpred &pr = q->pred[p];
+    bool ok;
+    if (is_float(pr.type1) || is_float(pr.type2)) {
+      const double x = is_float(pr.type1) ? read_float(a, pr.off1, pr.type1) : (double)read_int(a, pr.off1, pr.type1);
+      const double y = is_float(pr.type2) ? read_float(b, pr.off2, pr.type2) : (double)read_int(b, pr.off2, pr.type2);
+      ok = cmp(x, pr.op, y);
+    } else {
+      ok = cmp(read_int(a, pr.off1, pr.type1), pr.op, read_int(b, pr.off2, pr.type2));
+    }
+    if (!ok) return false;
+  }
+  return true;
+}
+int col_width(int32_t type) { return (type == OQ_I32 || type == OQ_F32) ? 4 : 8; }
+}  // namespace
+
+extern "C" int32_t oq_join_run(const oq_join *q, const uint8_t *t1, int64_t n1, const uint8_t *t2, int64_t n2,
+                               int32_t nthreads, oq_result *out) {
+  std::memset(out, 0, sizeof(*out));
+  if (q->size < 1 || q->slide < 1 || q->npred < 0 || q->npred > 64 || q->nproj1 > 16 || q->nproj2 > 16) {
+    out->error = OQ_EINVAL;
+    return OQ_EINVAL;
+  }
+  const int64_t n = n1 < n2 ? n1 : n2;
+  const int64_t nw = n >= q->size ? (n - q->size) / q->slide + 1 : 0;
+  int64_t rb = 0;
+  for (int c = 0; c < q->nproj1; ++c) rb += col_width(q->proj1[c].type);
+  for (int c = 0; c < q->nproj2; ++c) rb += col_width(q->proj2[c].type);
+  std::vector<std::vector<uint8_t>> wins((size_t)nw);
+  std::atomic<int64_t> next{0};
+  auto worker = [&]() {
+    for (;;) {
+      const int64_t j = next.fetch_add(1);
+      if (j >= nw) break;
+      std::vector<uint8_t> &o = wins[(size_t)j];
+      for (int64_t a = j * q->slide; a < j * q->slide + q->size; ++a) {
+        const uint8_t *ta = t1 + a * q->tuple_bytes1;
+        for (int64_t b = j * q->slide; b < j * q->slide + q->size; ++b) {
+          const uint8_t *tb = t2 + b * q->tuple_bytes2;
+          if (!jpred_ok(q, ta, tb)) continue;
+          for (int c = 0; c < q->nproj1; ++c)
+            o.insert(o.end(), ta + q->proj1[c].off, ta + q->proj1[c].off + col_width(q->proj1[c].type));
+          for (int c = 0; c < q->nproj2; ++c)
+            o.insert(o.end(), tb + q->proj2[c].off, tb + q->proj2[c].off + col_width(q->proj2[c].type));
+        }
+      }
+    }
+  };
+  if (nthreads < 1) nthreads = 1;
+  if (nthreads == 1) worker();
+  else {
+    std::vector<std::thread> th;
+    for (int t = 0; t < nthreads; ++t) th.emplace_back(worker);
+    for (auto &t : th) t.join();
+  }
+  int64_t nbytes = 0;
+  for (auto &w : wins) nbytes += (int64_t)w.size();
+  out->nwin = nw;
+  out->win_id = (int64_t *)std::malloc(sizeof(int64_t) * (nw + 1));
+  out->win_ts = (int64_t *)std::malloc(sizeof(int64_t) * (nw + 1));
+  out->win_nrows = (int64_t *)std::malloc(sizeof(int64_t) * (nw + 1));
+  out->win_rowoff = (int64_t *)std::malloc(sizeof(int64_t) * (nw + 1));
+  out->keys = (int64_t *)std::malloc(8);
+  out->vals = (uint64_t *)std::malloc(8);
+  out->out_bytes = nbytes;
+  out->out = (uint8_t *)std::malloc(nbytes + 1);
+  out->row_bytes = rb;
+  int64_t off = 0;
+  for (int64_t j = 0; j < nw; ++j) {
+    int64_t ts;
+    std::memcpy(&ts, t1 + j * q->slide * q->tuple_bytes1 + q->ts_off1, 8);   // reading A7
+    out->win_id[j] = j;
+    out->win_ts[j] = ts;
+    out->win_nrows[j] = rb ? (int64_t)wins[(size_t)j].size() / rb : 0;
+    out->win_rowoff[j] = rb ? off / rb : 0;
+    if (!wins[(size_t)j].empty()) std::memcpy(out->out + off, wins[(size_t)j].data(), wins[(size_t)j].size());
+    off += (int64_t)wins[(size_t)j].size();
+  }
+  out->nrows = rb ? nbytes / rb : 0;
+  return OQ_OK;
+}

@@ -73,6 +73,27 @@ int64_t oq_num_windows(const oq_query *q, const uint8_t *tuples, int64_t n,
                        int64_t watermark, int32_t has_wm);
 void oq_free(oq_result *r);
 
+/* Windowed θ-join of two streams (§2.4 L377-383 θ-join per window,
+ * RStream L401-405; n-ary query tasks §3; JOIN_r, Table 1).
+ * Reading A26: both streams use the same count window ω(s,l);
+ * window j of the join is W1_j ⋈θ W2_j with W_j = [j·l, j·l+s) on each stream,
+ * for j·l+s <= min(n1, n2); θ is a conjunction of `S1.col1 op S2.col2`
+ * (compared as int64 when both columns are integers, else as double); every
+ * matching pair (a, b) emits π1(t1[a]) ++ π2(t2[b]), pairs in (a, b) order;
+ * the window header ts is τ of t1[j·l] (reading A7). */
+typedef struct { int32_t off1, type1, op, off2, type2, pad; } oq_jpred;
+typedef struct {
+  int32_t tuple_bytes1, tuple_bytes2, ts_off1, pad;
+  int64_t size, slide;
+  int32_t npred;  oq_jpred pred[64];
+  int32_t nproj1; oq_col proj1[16];
+  int32_t nproj2; oq_col proj2[16];
+} oq_join;
+/* out: win_id/win_ts/win_nrows/win_rowoff per window, out/out_bytes the
+ * concatenated pair rows, row_bytes their width (nrows = pairs). */
+int32_t oq_join_run(const oq_join *q, const uint8_t *t1, int64_t n1, const uint8_t *t2, int64_t n2,
+                    int32_t nthreads, oq_result *out);
+
 #ifdef __cplusplus
 }
 #endif

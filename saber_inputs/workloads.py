@@ -121,3 +121,17 @@ def bench_task_mb(config, groups=64):
     if config == "C3" and groups != 64:
         return BENCH_TASK_MB.get(f"C3_G{groups}", 1024 if groups <= 4096 else 256)
     return BENCH_TASK_MB[config]
+
+
+# --- f3: JOIN_r, windowed θ-join of two Syn streams (Table 1, §6.2) ---
+def join_r(r=1, size=1024, slide=1024, n=1 << 20):
+    """SELECT S1.ts, S1.a1, S2.a1, S2.a2 FROM Syn1 [ROWS size SLIDE slide] AS S1,
+    Syn2 [ROWS size SLIDE slide] AS S2 WHERE S1.a3 < S2.a3 AND S1.a4 < S2.a4 ...
+    (r terms over a3..a6, cycling): the r-predicate θ-join JOIN_r; the attributes
+    are uniform and independent, so 2^-min(r, 4) of the pairs match."""
+    cols = ["a3", "a4", "a5", "a6"]
+    theta = [(cols[k % 4], "<", cols[k % 4]) for k in range(r)]
+    spec = {"schema1": copy.deepcopy(SCHEMAS["syn"]), "schema2": copy.deepcopy(SCHEMAS["syn"]),
+            "window": count_window(size, slide), "theta": theta,
+            "project1": ["ts", "a1"], "project2": ["a1", "a2"]}
+    return spec, {"kind": "syn", "n": n, "seed1": 7, "seed2": 8, "rate": 1, "groups": 64}

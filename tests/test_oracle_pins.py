@@ -381,3 +381,50 @@ def test_istream_rows_per_window(oracle_lib):
         exp = [int(sel[0:s].sum())] + [int(sel[(j - 1) * l + s:j * l + s].sum()) for j in range(1, W)]
         assert list(r["win_nrows"]) == exp
         assert list(r["win_ts"]) == [int(ts[j * l]) for j in range(W)]
+
+
+# ------------------------------------------------------------------ θ-join ---
+def _jspec(w, theta, p1=("ts", "a1"), p2=("a1", "a2")):
+    sch = gen.SCHEMAS["syn"]
+    return {"schema1": sch, "schema2": sch, "window": w, "theta": list(theta),
+            "project1": list(p1), "project2": list(p2)}
+
+
+def test_join_matches_brute_force(oracle_lib):
+    """The oracle's windowed θ-join equals an independent Python formulation
+    (oracle/brute.py: 1-based windows, sets of matching pairs) byte for byte."""
+    from oracle.brute import brute_join
+    rng = np.random.default_rng(5)
+    for _ in range(40):
+        n1, n2 = int(rng.integers(0, 40)), int(rng.integers(0, 40))
+        s = int(rng.integers(1, 9))
+        l = int(rng.integers(1, s + 1))
+        d1 = bytearray(gen.generate("syn", n1, int(rng.integers(1, 99)), groups=3))
+        d2 = bytearray(gen.generate("syn", n2, int(rng.integers(1, 99)), groups=3))
+        ops = ["<", "<=", ">", ">=", "==", "!="]
+        theta = [(str(rng.choice(["a2", "a3", "a1"])), str(rng.choice(ops)), str(rng.choice(["a2", "a4", "a1"])))
+                 for _ in range(int(rng.integers(0, 3)))]
+        js = _jspec({"kind": "count", "size": s, "slide": l}, theta)
+        got = oracle_lib.join_run(js, bytes(d1), bytes(d2))
+        exp = brute_join(js, bytes(d1), bytes(d2))
+        assert list(got["win_id"]) == [j for j, _, _ in exp]
+        assert list(got["win_ts"]) == [ts for _, ts, _ in exp]
+        assert list(got["win_nrows"]) == [len(r) for _, _, r in exp]
+        assert got["tuples"] == b"".join(b"".join(r) for _, _, r in exp)
+
+
+def test_join_cross_product_and_equijoin_counts(oracle_lib):
+    """Closed forms: with no θ term every window emits s^2 pairs (the window cross
+    product); an equi-join on a key emits sum_k c1(k)·c2(k) pairs per window
+    (numpy bincount of each side's window)."""
+    n, s, l = 3000, 64, 48
+    d1 = gen.generate("syn", n, 21, groups=7)
+    d2 = gen.generate("syn", n, 22, groups=7)
+    r = oracle_lib.join_run(_jspec({"kind": "count", "size": s, "slide": l}, []), d1, d2)
+    W = (n - s) // l + 1
+    assert list(r["win_nrows"]) == [s * s] * W
+    r = oracle_lib.join_run(_jspec({"kind": "count", "size": s, "slide": l}, [("a2", "==", "a2")]), d1, d2)
+    k1, k2 = gen.column(d1, "syn", "a2"), gen.column(d2, "syn", "a2")
+    exp = [int((np.bincount(k1[j * l:j * l + s], minlength=7) * np.bincount(k2[j * l:j * l + s], minlength=7)).sum())
+           for j in range(W)]
+    assert list(r["win_nrows"]) == exp
