@@ -62,6 +62,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--hash-capacity", type=int, default=0,
+                    help="pane hash-table slots (power of two; 0: the planner's guess).  CM2 defaults to "
+                         "2x the expected distinct jobIds per pane (the paper's static hash-table pool, L1293-1295)")
     ap.add_argument("--launcher-check", action="store_true",
                     help="CPU (gloo) check of the multi-rank launch: no GPU work")
     return ap.parse_args()
@@ -426,9 +429,14 @@ def main():
     out_rows = out_tuples = out_windows = 0
     clk_dir = os.path.join(ROOT, "gpurun_out") if os.path.isdir(os.path.join(ROOT, "gpurun_out")) else "/tmp"
     # one long-lived query; every step replays the stream after saber_query_reset
+    hcap = args.hash_capacity
+    if not hcap and args.config == "CM2":
+        # eventType == 1 keeps 1/9 of R tuples per 1-s pane; their jobIds are ~all distinct
+        hcap = 1 << max(6, int(np.ceil(np.log2(2 * max(1, g["rate"] // 9)))))
     q = saber.Query(spec, base_index=base_index, first_window=first_window,
                     emit_on_finish=(rank == world - 1), task_bytes=task_bytes,
-                    result_mode=saber.RESULTS_DEVICE, profile=True, result_slots=8, device=local)
+                    result_mode=saber.RESULTS_DEVICE, profile=True, result_slots=8, device=local,
+                    hash_capacity=hcap)
     with Clocks(local, os.path.join(clk_dir, f"clocks_rank{rank}.csv")) as clk:
         t_wait = time.perf_counter()                 # NVML initialised and sampling before timing
         while clk.thread is not None and not clk.rows and time.perf_counter() - t_wait < 5.0:
@@ -514,7 +522,8 @@ def main():
         d2h_bytes = 0
         e2e_task = args.e2e_task_mb << 20
         q = saber.Query(spec, task_bytes=e2e_task, result_mode=saber.RESULTS_HOST, device=local,
-                        base_index=base_index, first_window=first_window, emit_on_finish=(rank == world - 1))
+                        base_index=base_index, first_window=first_window, emit_on_finish=(rank == world - 1),
+                        hash_capacity=hcap)
         q.register_host(host_np)
         for it in range(args.warmup + min(args.steps, 3)):
             q.reset(base_index, first_window)

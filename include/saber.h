@@ -278,6 +278,47 @@ saber_status saber_partition_plan(const saber_schema *schema, const saber_window
                                   const void *dev_tuples, int64_t begin, int64_t n,
                                   int64_t *closed_windows, int64_t *halo_first);
 
+/* ---- windowed θ-join of two streams ----------------------
+ * The n-ary query task v = (f^q, <b1, b2>) of PAPER.md §3 L415-422 with the
+ * θ-join operator (§2.4; JOIN_r, Table 1), RStream (L401-405).
+ * Both streams use the same COUNT window ω(size, slide) (reading A26): window j
+ * of the join is W1_j ⋈θ W2_j, W_j = [j·slide, j·slide+size) on each stream,
+ * closed once both streams hold j·slide+size tuples.  θ is a conjunction of
+ * `S1.col1 op S2.col2` (both integer columns: int64 compare, else double).
+ * Every matching pair (a, b) emits one row π1(t1[a]) ++ π2(t2[b]) (projected
+ * columns packed in projection order); rows of a window are in (a, b) order;
+ * headers as for aggregation (ts = τ of S1's first tuple of the window, A7).
+ * Executed as in §5.4: count the matches per (window, row of S1),
+ * scan, then write the pairs at their offsets (no quadratic buffers). */
+typedef struct { int32_t col1; saber_cmp op; int32_t col2; } saber_join_pred;
+typedef struct {
+  int32_t npred;  const saber_join_pred *theta;    /* <= 64 terms                    */
+  int32_t nproj1; const int32_t *proj1;            /* S1 columns of an output row    */
+  int32_t nproj2; const int32_t *proj2;            /* S2 columns (nproj1+nproj2 >= 1) */
+} saber_join_op;
+typedef struct saber_join saber_join;
+
+/* Create a θ-join.  cfg: device, task_bytes (batch capacity per stream, bytes of
+ * S1 tuples) [32 MiB], result_mode, result_bytes (rows per slot) [256 MiB],
+ * result_slots [4]; other fields ignored.  Errors: SABER_EINVAL (time windows,
+ * bad columns/terms), SABER_ECUDA, SABER_ENOMEM. */
+saber_status saber_join_create(const saber_schema *s1, const saber_schema *s2, const saber_join_op *op,
+                               const saber_window *window, const saber_config *cfg, saber_join **out);
+/* One query task: ntuples tuples of each stream (device pointers, 16-B aligned),
+ * ordered after `cuda_stream`'s prior work, which then waits for the task's
+ * reads.  SABER_EAGAIN (nothing consumed) when the task's result slot is busy. */
+saber_status saber_join_submit_device(saber_join *j, const void *dev1, const void *dev2, size_t ntuples,
+                                      void *cuda_stream);
+/* The same from host memory (copied before return). */
+saber_status saber_join_submit(saber_join *j, const void *host1, const void *host2, size_t ntuples);
+/* Next task's slice in task order: nwindows headers, ntuples pair rows of
+ * tuple_bytes each in `tuples` (host or device pointers, valid until release).
+ * SABER_ENOMEM if the task's pairs exceed result_bytes. */
+saber_status saber_join_poll(saber_join *j, saber_results *out, int32_t timeout_us);
+saber_status saber_join_release(saber_join *j, const saber_results *r);
+void saber_join_destroy(saber_join *j);
+const char *saber_join_last_error(const saber_join *j);
+
 /* Library version string. */
 const char *saber_version(void);
 

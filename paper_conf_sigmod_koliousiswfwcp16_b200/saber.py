@@ -117,7 +117,24 @@ SIGNATURES = {
     "saber_partition_plan": (C.c_int, [C.POINTER(Schema), C.POINTER(Window), C.c_void_p, C.c_int64, C.c_int64,
                                        C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
     "saber_version": (C.c_char_p, []),
+    "saber_join_create": (C.c_int, [C.POINTER(Schema), C.POINTER(Schema), C.c_void_p, C.POINTER(Window),
+                                    C.POINTER(Config), C.POINTER(C.c_void_p)]),
+    "saber_join_submit_device": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p]),
+    "saber_join_submit": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_size_t]),
+    "saber_join_poll": (C.c_int, [C.c_void_p, C.POINTER(Results), C.c_int32]),
+    "saber_join_release": (C.c_int, [C.c_void_p, C.POINTER(Results)]),
+    "saber_join_destroy": (None, [C.c_void_p]),
+    "saber_join_last_error": (C.c_char_p, [C.c_void_p]),
 }
+
+
+class JoinPred(C.Structure):
+    _fields_ = [("col1", C.c_int32), ("op", C.c_int32), ("col2", C.c_int32)]
+
+
+class JoinOp(C.Structure):
+    _fields_ = [("npred", C.c_int32), ("theta", C.POINTER(JoinPred)), ("nproj1", C.c_int32),
+                ("proj1", C.POINTER(C.c_int32)), ("nproj2", C.c_int32), ("proj2", C.POINTER(C.c_int32))]
 
 _lib = None
 
@@ -396,3 +413,113 @@ def partition_plan(spec, dev_ptr, begin, n):
                                     int(n), C.byref(c), C.byref(h))
     _check(st)
     return c.value, h.value
+
+
+class Join:
+    """Windowed θ-join of two streams (wraps saber_join; include/saber.h).
+    ``jspec``: schema1, schema2, window (count), theta [(col1, op, col2)],
+    project1, project2 -- the dicts of saber_inputs.workloads.join_r."""
+
+    def __init__(self, jspec, device=None, task_bytes=32 << 20, result_mode=RESULTS_HOST, result_bytes=0,
+                 result_slots=4):
+        self.L = lib()
+        self.spec = jspec
+        self.m1 = _Marshalled({"schema": jspec["schema1"], "window": jspec["window"]})
+        self.m2 = _Marshalled({"schema": jspec["schema2"], "window": jspec["window"]})
+        n1, n2 = self.m1.names, self.m2.names
+        th = jspec.get("theta", [])
+        self.theta = (JoinPred * max(1, len(th)))(*[JoinPred(n1.index(a), OPS[op], n2.index(b)) for a, op, b in th])
+        self.p1 = (C.c_int32 * max(1, len(jspec["project1"])))(*[n1.index(c) for c in jspec["project1"]])
+        self.p2 = (C.c_int32 * max(1, len(jspec["project2"])))(*[n2.index(c) for c in jspec["project2"]])
+        self.op = JoinOp(len(th), self.theta, len(jspec["project1"]), self.p1, len(jspec["project2"]), self.p2)
+        cfg = Config()
+        cfg.device = -1 if device is None else int(device)
+        cfg.task_bytes = int(task_bytes)
+        cfg.result_mode = int(result_mode)
+        cfg.result_bytes = int(result_bytes)
+        cfg.result_slots = int(result_slots)
+        self.cfg = cfg
+        self.tb1, self.tb2 = jspec["schema1"]["tuple_bytes"], jspec["schema2"]["tuple_bytes"]
+        h = C.c_void_p()
+        st = self.L.saber_join_create(C.byref(self.m1.schema), C.byref(self.m2.schema), C.byref(self.op),
+                                      C.byref(self.m1.window), C.byref(cfg), C.byref(h))
+        if st != OK:
+            raise SaberError(st, (self.L.saber_join_last_error(None) or b"").decode())
+        self.h = h
+
+    def last_error(self):
+        m = self.L.saber_join_last_error(self.h)
+        return m.decode() if m else ""
+
+    def submit(self, d1, d2):
+        b1 = np.ascontiguousarray(np.frombuffer(d1, np.uint8) if isinstance(d1, (bytes, bytearray)) else d1)
+        b2 = np.ascontiguousarray(np.frombuffer(d2, np.uint8) if isinstance(d2, (bytes, bytearray)) else d2)
+        n = b1.size // self.tb1
+        assert b2.size // self.tb2 == n, "both batches of a task hold the same number of tuples"
+        return self.L.saber_join_submit(self.h, C.c_void_p(b1.ctypes.data), C.c_void_p(b2.ctypes.data), n)
+
+    def submit_device(self, ptr1, ptr2, ntuples, stream=0):
+        return self.L.saber_join_submit_device(self.h, C.c_void_p(ptr1), C.c_void_p(ptr2), int(ntuples),
+                                               C.c_void_p(stream))
+
+    def poll_raw(self, timeout_us=-1):
+        r = Results()
+        return self.L.saber_join_poll(self.h, C.byref(r), int(timeout_us)), r
+
+    def release(self, r):
+        st = self.L.saber_join_release(self.h, C.byref(r))
+        if st != OK:
+            raise SaberError(st, self.last_error())
+
+    def poll(self, timeout_us=-1):
+        """Next slice copied into numpy (host mode): (headers, pair-row bytes), or None."""
+        st, r = self.poll_raw(timeout_us)
+        if st == EAGAIN:
+            return None
+        if st != OK:
+            raise SaberError(st, self.last_error())
+        try:
+            hdr = np.zeros(r.nwindows, dtype=[("window_id", "<i8"), ("ts", "<i8"), ("row_offset", "<i8"),
+                                              ("nrows", "<i4"), ("flags", "<i4")])
+            if r.nwindows:
+                C.memmove(hdr.ctypes.data, r.hdr, r.nwindows * 32)
+            rows = C.string_at(r.tuples, r.ntuples * r.tuple_bytes) if r.ntuples else b""
+            return hdr, rows
+        finally:
+            self.release(r)
+
+    def run(self, d1, d2, batch_tuples):
+        """Submit both streams in tasks of batch_tuples tuples; concatenated results."""
+        n = min(len(d1) // self.tb1, len(d2) // self.tb2)
+        hdrs, rows = [], []
+        off = 0
+        while off < n:
+            k = min(batch_tuples, n - off)
+            st = self.submit(d1[off * self.tb1:(off + k) * self.tb1], d2[off * self.tb2:(off + k) * self.tb2])
+            if st == EAGAIN:
+                h, r = self.poll()
+                hdrs.append(h)
+                rows.append(r)
+                continue
+            if st != OK:
+                raise SaberError(st, self.last_error())
+            off += k
+        while (x := self.poll()) is not None:
+            hdrs.append(x[0])
+            rows.append(x[1])
+        h = np.concatenate(hdrs) if hdrs else np.zeros(0, dtype=[("window_id", "<i8"), ("ts", "<i8"),
+                                                                 ("row_offset", "<i8"), ("nrows", "<i4"),
+                                                                 ("flags", "<i4")])
+        return {"win_id": h["window_id"].astype(np.int64), "win_ts": h["ts"].astype(np.int64),
+                "win_nrows": h["nrows"].astype(np.int64), "tuples": b"".join(rows)}
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.L.saber_join_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
