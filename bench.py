@@ -45,7 +45,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="saber", choices=["saber", "reference"])
-    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "C5a", "C5b", "SG1", "CM2"])
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "C5a", "C5b", "SG1", "CM2", "JOIN"])
+    ap.add_argument("--join-r", type=int, default=4, help="JOIN: predicates r of JOIN_r (Table 1, L1385)")
     ap.add_argument("--npred", type=int, default=1,
                     help="C2: SELECT_n -- n predicate terms (n-1 always-true terms, Fig. 10a)")
     ap.add_argument("--groups", type=int, default=64)
@@ -337,8 +338,92 @@ def launcher_check(args, rank, world):
     dist.destroy_process_group()
 
 
+def run_join(args, rank, world):
+    """f3: JOIN_r over two Syn streams of 2^tuples_log2 tuples each (default 2^20),
+    ω(size, slide) (default the paper's ω32KB,32KB = 1024 tuples), device-resident
+    batches of φ tuples, DEVICE results.  Value: input tuples (both streams) / s.
+    The join is ALU-bound: s^2 pair tests per window; roofline.bound = "alu" with
+    the pair-test rate against a peak derived in DESIGN.md §6."""
+    import torch
+    from paper_conf_sigmod_koliousiswfwcp16_b200 import saber
+    size = args.size or 1024
+    slide = args.slide or size
+    n = 1 << (args.tuples_log2 or 20)
+    js, g = workloads.join_r(r=args.join_r, size=size, slide=slide, n=n)
+    name = (f"JOIN_{args.join_r}: Syn x Syn, theta = {args.join_r} terms S1.a_k < S2.a_k, count w({size},{slide}), "
+            f"2^{int(np.log2(n))} tuples per stream")
+    dev = torch.device("cuda", 0)
+    lib_gen = C.CDLL(os.path.join(ROOT, "saber_inputs", "libsaber_gen.so"))
+    st = torch.cuda.current_stream()
+    bufs = []
+    for seed in (g["seed1"], g["seed2"]):
+        b = torch.empty(n * 32, dtype=torch.uint8, device=dev)
+        gen_device(lib_gen, "syn", seed, 0, n, 1, 64, b, st.cuda_stream)
+        bufs.append(b)
+    torch.cuda.synchronize()
+    batch = max(size, ((args.task_mb or 32) << 20) // 32)
+    batch = min(batch, n)
+    nt = (n + batch - 1) // batch
+    j = saber.Join(js, task_bytes=batch * 32, result_mode=saber.RESULTS_DEVICE, result_slots=nt + 1,
+                   result_bytes=1 << 30)
+    times, pairs = [], 0
+    with Clocks(0, os.path.join(ROOT, "gpurun_out", "clocks_join.csv") if os.path.isdir(os.path.join(ROOT, "gpurun_out"))
+                else "/tmp/clocks_join.csv") as clk:
+        for it in range(args.warmup + args.steps):
+            j.close()
+            j = saber.Join(js, task_bytes=batch * 32, result_mode=saber.RESULTS_DEVICE, result_slots=nt + 1,
+                           result_bytes=1 << 30)
+            torch.cuda.synchronize()
+            clk.timed = it >= args.warmup
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(st)
+            for t in range(nt):
+                k = min(batch, n - t * batch)
+                rc = j.submit_device(bufs[0].data_ptr() + t * batch * 32, bufs[1].data_ptr() + t * batch * 32, k,
+                                     st.cuda_stream)
+                assert rc == 0, j.last_error()
+            e1.record(st)
+            torch.cuda.synchronize()
+            clk.timed = False
+            tot = 0
+            while True:
+                rc, r = j.poll_raw(-1)
+                if rc != 0:
+                    break
+                tot += r.ntuples
+                j.release(r)
+            if it >= args.warmup:
+                times.append(e0.elapsed_time(e1))
+                pairs = tot
+    j.close()
+    ms = statistics.median(times)
+    nwin = (n - size) // slide + 1
+    tests = nwin * size * size
+    tests_per_s = tests / (ms / 1e3)
+    # ALU roofline (DESIGN.md §6): a pair test needs at least a compare and a select per
+    # θ term on one INT32 lane; B200: 148 SMs x 128 INT32 lanes per clock
+    clk_ghz = MEASURED_SM_GHZ
+    peak = 148 * 128 * clk_ghz * 1e9 / (2 * args.join_r)
+    line = {"metric": METRIC, "value": 2 * n / (ms / 1e3), "unit": "tuples/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "i32", "data": "synthetic",
+            "config": {"workload": name, "task_tuples": batch, "windows_per_step": nwin, "pairs_out_per_step": pairs},
+            "roofline": {"bound": "alu", "achieved": tests_per_s, "peak": peak, "unit": "pair tests/s",
+                         "frac": tests_per_s / peak, "peak_source": "derived: 148 SMs x 128 INT32 lanes x SM clock / "
+                                                                    "(2 instructions x r terms per pair test)"},
+            "clocks": clk.summary(), "gpu_launches": 5 * nt}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+MEASURED_SM_GHZ = 1.965
+
+
 def main():
     args = parse()
+    if args.config == "JOIN":
+        run_join(args, int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")))
+        return
     spec, g, name, w = workload(args)
     if "WORLD_SIZE" not in os.environ and args.gpus > 1:
         sys.exit(launch_ranks(args.gpus))

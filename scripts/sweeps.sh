@@ -10,6 +10,10 @@ run() { out=$1; shift; echo "== $*" >&2; timeout 500 python bench.py --no-cpu "$
 o=gpurun_out/sweeps/f1_cm2.jsonl; : > $o
 run $o --config CM2 --steps 5 --warmup 3
 run $o --config CM2 --rate 4096 --steps 5 --warmup 3
+o=gpurun_out/sweeps/f3_join.jsonl; : > $o
+run $o --config JOIN --join-r 1 --steps 5 --warmup 3
+run $o --config JOIN --join-r 4 --steps 5 --warmup 3
+run $o --config JOIN --join-r 16 --steps 5 --warmup 3
 o=gpurun_out/sweeps/f1_select_n.jsonl; : > $o
 for n in 1 4 16 64; do run $o --config C2 --sel 0.5 --npred $n --steps 5 --warmup 3 --no-e2e; done
 o=gpurun_out/sweeps/f2_task_size.jsonl; : > $o
