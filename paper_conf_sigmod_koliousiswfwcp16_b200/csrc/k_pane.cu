@@ -209,6 +209,66 @@ __device__ __forceinline__ void flush_tables(const Plan &p, State *st, uint64_t 
   __syncthreads();
 }
 
+// FX3 tables of k_pane_agg (Plan::fx_agg): a sum field is three u32 limbs taking
+// the 16-bit chunks of X = x·2^32 for x in [0, 2^16) and a multiple of 2^-32
+// (SG's 1000·u24, LRB speeds, u24 values), with fire-and-forget shared REDs; a
+// limb takes <= 65,535 chunks of <= 0xffff between flushes (the CTA flushes every
+// 2^16 - stage tuples), so it cannot wrap.  Other values go as fp64 straight to
+// the pane ring (RED.ADD.F64).  Layout per warp (or CTA): [NF][3][TE] limbs, [TE] counts.
+__device__ __forceinline__ bool fx48(uint32_t xb, uint64_t &X) {
+  const uint32_t ex = (xb >> 23) & 0xffu;
+  const uint32_t m = (xb & 0x7fffffu) | 0x800000u;
+  X = 0;
+  if (xb == 0u) return true;
+  if ((xb >> 31) || ex >= 143u || ex == 0u) return false;
+  if (ex >= 118u) { X = (uint64_t)m << (ex - 118u); return true; }
+  const uint32_t sh = 118u - ex;
+  if (sh > 23u || (m & ((1u << sh) - 1u))) return false;
+  X = m >> sh;
+  return true;
+}
+__device__ __forceinline__ void red_add_u32(uint32_t *p, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(p)), "r"(v) : "memory");
+}
+template <int MODE, int NF>
+__device__ __forceinline__ void flush_fx3(const Plan &p, State *st, uint64_t *table, unsigned char *tabs,
+                                          int64_t pbase, int &err) {
+  const int tid = threadIdx.x;
+  const int TE = p.local_entries;
+  constexpr int NCOPY = MODE == TM_SHARED ? 1 : kP1Warps;
+  const int C = (int)p.C;
+  __syncthreads();
+  for (int e = tid; e < TE; e += kP1Threads) {
+    uint32_t c = 0;
+    double sum[NF];
+#pragma unroll
+    for (int f = 0; f < NF; ++f) sum[f] = 0.0;
+    for (int w = 0; w < NCOPY; ++w) {
+      uint32_t *lm = (uint32_t *)(tabs + (size_t)w * p.local_bytes);
+      uint32_t *oc = lm + 3 * NF * TE;
+      const uint32_t cw = oc[e];
+      if (!cw) continue;
+      c += cw;
+      oc[e] = 0;
+#pragma unroll
+      for (int f = 0; f < NF; ++f) {
+        uint32_t *l = lm + 3 * f * TE;
+        sum[f] += (double)l[e] * 0x1p-32 + (double)l[TE + e] * 0x1p-16 + (double)l[2 * TE + e];
+        l[e] = 0;
+        l[TE + e] = 0;
+        l[2 * TE + e] = 0;
+      }
+    }
+    if (c) {
+      uint64_t fv[NF];
+#pragma unroll
+      for (int f = 0; f < NF; ++f) fv[f] = (uint64_t)__double_as_longlong(sum[f]);
+      flush_entry<NF>(p, st, table, pbase + e / C, (uint64_t)(e % C), c, fv, err);
+    }
+  }
+  __syncthreads();
+}
+
 // NK >= 0 (FAST plans): exactly NK radix-packed int32 key columns, known at
 // compile time (no per-tuple loop bounds and plan-field branches); -1: run time
 template <int MODE, int WK, int NF, bool FAST, int NK = -1>
@@ -230,13 +290,22 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   unsigned char *wt = tabs + (MODE == TM_SHARED ? 0 : (size_t)wid * p.local_bytes);
   uint64_t *tkeys = (uint64_t *)wt;                      // HASHED only
   uint64_t *tf = (uint64_t *)(wt + (MODE == TM_HASHED ? 8 * TE : 0));   // [NF][TE*CW]
-  uint32_t *tcnt = (uint32_t *)((unsigned char *)tf + (size_t)8 * TE * CW * NF);   // [TE*CW]
+  constexpr bool FXM = FAST && (MODE == TM_DIRECT || MODE == TM_SHARED);
+  const bool fx = FXM && p.fx_agg;                       // CTA-uniform
+  uint32_t *tlimb = (uint32_t *)wt;                      // fx: [NF][3][TE] limbs
+  uint32_t *tcnt = (uint32_t *)((unsigned char *)tf + (size_t)(fx ? 12 : 8) * TE * CW * NF);   // [TE*CW]
   for (int e = (MODE == TM_SHARED ? tid : lane); e < TE * CW; e += (MODE == TM_SHARED ? kP1Threads : 32)) {
     if (MODE == TM_HASHED) tkeys[e] = kEmpty;
     tcnt[e] = 0;
+    if (fx) {
 #pragma unroll
-    for (int f = 0; f < NF; ++f) tf[f * TE * CW + e] = f < p.nf ? field_identity(p.field[f].kind) : 0;
+      for (int f = 0; f < 3 * NF; ++f) tlimb[f * TE + e] = 0;
+    } else {
+#pragma unroll
+      for (int f = 0; f < NF; ++f) tf[f * TE * CW + e] = f < p.nf ? field_identity(p.field[f].kind) : 0;
+    }
   }
+  int fx_since = 0;                                      // tuples since the last flush (limb bound)
 
   // rounds (Plan::rounds > 1): this launch scans the sub-range k_task_begin chose
   if (p.rounds > 1) {
@@ -274,7 +343,11 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   int64_t prev_last = (lo > 0 && lo < hi) ? *(const int64_t *)(tup + (lo - 1) * tb + 4 * tsw) : INT64_MIN;
   const int per_warp = (ST + kP1Warps - 1) / kP1Warps;
 
-  auto flush_shared = [&]() { flush_tables<MODE, NF, FAST>(p, st, table, tabs, tf, tcnt, pbase, err); };
+  auto flush_shared = [&]() {
+    if (FXM && fx) flush_fx3<MODE, NF>(p, st, table, tabs, pbase, err);
+    else flush_tables<MODE, NF, FAST>(p, st, table, tabs, tf, tcnt, pbase, err);
+    fx_since = 0;
+  };
   auto flush_hashed = [&]() {      // warp-private table of one pane
     __syncwarp();
     for (int e = lane; e < TE; e += 32) {
@@ -425,7 +498,24 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
                 tf[f * TE * 32 + e] = field_combine(p.field[f].kind, tf[f * TE * 32 + e], fv[f]);
           }
         } else if (MODE == TM_DIRECT || MODE == TM_SHARED) {
-          if (valid) {
+          if (valid && FXM && fx) {
+            const int e = pw * C + (int)key;
+            red_add_u32(&tcnt[e], 1u);
+#pragma unroll
+            for (int f = 0; f < NF; ++f) {
+              const float xf = (float)__longlong_as_double((long long)fv[f]);   // exact: an f32 widened
+              uint64_t X;
+              if (fx48(__float_as_uint(xf), X)) {
+                uint32_t *l = tlimb + 3 * f * TE + e;
+                red_add_u32(l, (uint32_t)X & 0xffffu);
+                red_add_u32(l + TE, (uint32_t)(X >> 16) & 0xffffu);
+                if (X >> 32) red_add_u32(l + 2 * TE, (uint32_t)(X >> 32));
+              } else {
+                atomicAdd((double *)&table[((pbase + pw) & (p.R - 1)) * p.slot_words + fld_off(p, f) + key],
+                          __longlong_as_double((long long)fv[f]));
+              }
+            }
+          } else if (valid) {
             const int e = pw * C + (int)key;
             atomicAdd(&tcnt[e], 1u);
 #pragma unroll
@@ -485,7 +575,9 @@ k_pane_agg(const Plan p, State *__restrict__ st, const unsigned char *__restrict
       issue(k + kStages);
     }
     if (++slot == kStages) { slot = 0; phase ^= 1u; }
-    if (false) {
+    if (FXM && fx) {                                     // limbs take < 2^16 chunks between flushes
+      fx_since += ntup;
+      if (fx_since + ST >= 65535 && pbase >= 0) flush_shared();
     }
   }
   if (pbase >= 0) {

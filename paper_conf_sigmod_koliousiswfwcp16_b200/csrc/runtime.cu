@@ -384,6 +384,7 @@ static saber_status size_plan(saber_query *q) {
       p.local_pl = 1;
       p.local_bytes = ((p.local_entries * eh) + 15) & ~15;
     }
+    p.fx_agg = 0;
     {
       bool fast = p.nf <= 2;
       for (int f = 0; f < p.nf; ++f) fast &= p.field[f].kind == FK_SUM_F && p.field[f].type == T_F32;
@@ -402,6 +403,24 @@ static saber_status size_plan(saber_query *q) {
       else if (p.nkeys > 0)
         fk &= p.fast_path != 0;
       p.fast_keys = (fk || p.fast_path) ? 1 : 0;
+    }
+    // k_pane_agg FX3 tables (atomic DIRECT / SHARED tables of f32 sums): three u32
+    // limbs per sum instead of one fp64 word -- re-size the pane window for them
+    if (p.fast_keys && p.nf >= 1 && p.nf <= 2 && (p.local_mode == 1 || p.local_mode == 3) &&
+        !getenv_flag("SABER_NO_FX")) {
+      bool sums = true;
+      for (int f = 0; f < p.nf; ++f) sums &= p.field[f].kind == FK_SUM_F && p.field[f].type == T_F32;
+      const int edx = 4 + 12 * p.nf;
+      // SHARED: at least one pane of C entries, up to 48 KiB (3 CTAs/SM with the 32 KiB stage ring)
+      const int64_t budget = p.local_mode == 1 ? direct_budget
+                             : std::max<int64_t>(p.local_bytes, std::min<int64_t>(48 * 1024, (int64_t)edx * p.C));
+      const int64_t pl = std::min<int64_t>(1024, budget / (edx * p.C));
+      if (sums && pl >= 1) {
+        p.fx_agg = 1;
+        p.local_pl = (int)pl;
+        p.local_entries = p.local_pl * (int)p.C;
+        p.local_bytes = ((p.local_entries * edx) + 15) & ~15;
+      }
     }
     // phase-2 geometry
     const int smem_budget = 96 * 1024;
@@ -650,6 +669,7 @@ static saber_status alloc_query(saber_query *q) {
     pl.local_pl = p.lane_pl;
     pl.local_entries = p.lane_entries;
     pl.local_bytes = p.lane_bytes;
+    pl.fx_agg = 0;
     CK(set_kernel_attributes(pl));
     const int lbps = p1_blocks_per_sm(pl);
     q->p1_grid_lane = (p.overlap ? std::max(1, lbps - 1) : lbps) * q->nsm;
