@@ -21,6 +21,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -119,6 +120,61 @@ k_join_pairs(const JoinPlan p, JIn v1, JIn v2, int64_t J0, int64_t *__restrict__
         ++out;
       } else {
         ++cnt;
+      }
+    }
+  }
+  if (!EMIT && act) counts[w * p.s + a_loc] = cnt;
+}
+
+// Fast path: every θ term compares two int32 columns (JOIN_r over Syn) and there
+// are at most kJoinFastTerms of them.  Row a's operands live in registers; the
+// chunk of W2 is staged column-wise (one int32 array per term: every lane of a
+// warp reads the same b, a broadcast); the comparison op per term is uniform.
+constexpr int kJoinFastTerms = 8;
+template <bool EMIT>
+__global__ void __launch_bounds__(kJoinThreads)
+k_join_pairs_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, int64_t *__restrict__ counts,
+                 const int64_t *__restrict__ offs, unsigned char *__restrict__ rows) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  int32_t *col = (int32_t *)smem;                              // [npred][kJoinChunk]
+  const int64_t w = blockIdx.x;
+  const int64_t base = (J0 + w) * p.l;
+  const int a_loc = blockIdx.y * kJoinThreads + threadIdx.x;
+  const bool act = a_loc < p.s;
+  const int np = p.npred;
+  const unsigned char *ta = act ? jtuple(v1, base + a_loc) : nullptr;
+  int32_t av[kJoinFastTerms];
+#pragma unroll
+  for (int k = 0; k < kJoinFastTerms; ++k) av[k] = (act && k < np) ? *(const int32_t *)(ta + 4 * p.pred[k].w1) : 0;
+  int64_t cnt = 0, out = 0;
+  if (EMIT && act) out = offs[w * p.s + a_loc];
+  const int orow = 4 * (p.nw1 + p.nw2);
+  for (int64_t c0 = 0; c0 < p.s; c0 += kJoinChunk) {
+    const int nb = (int)((p.s - c0) < kJoinChunk ? (p.s - c0) : kJoinChunk);
+    __syncthreads();
+    for (int x = threadIdx.x; x < nb; x += kJoinThreads) {
+      const unsigned char *tb = jtuple(v2, base + c0 + x);
+#pragma unroll
+      for (int k = 0; k < kJoinFastTerms; ++k)
+        if (k < np) col[k * kJoinChunk + x] = *(const int32_t *)(tb + 4 * p.pred[k].w2);
+    }
+    __syncthreads();
+    if (!act) continue;
+    for (int bi = 0; bi < nb; ++bi) {
+      bool ok = true;
+#pragma unroll
+      for (int k = 0; k < kJoinFastTerms; ++k)
+        if (k < np) ok &= cmp_op(av[k], p.pred[k].op, col[k * kJoinChunk + bi]);
+      if (!EMIT) {
+        cnt += ok;
+      } else if (ok) {
+        if (out < p.rows_cap) {
+          const unsigned char *tb = jtuple(v2, base + c0 + bi);
+          uint32_t *dst = (uint32_t *)(rows + out * orow);
+          for (int c = 0; c < p.nw1; ++c) dst[c] = ((const uint32_t *)ta)[p.pw1[c]];
+          for (int c = 0; c < p.nw2; ++c) dst[p.nw1 + c] = ((const uint32_t *)tb)[p.pw2[c]];
+        }
+        ++out;
       }
     }
   }
@@ -232,6 +288,7 @@ struct saber_join {
   uint64_t epoch = 0;
   std::vector<JSlot> slots;
   int64_t next_task = 0, next_poll = 0;
+  bool fast = false;               // every θ term compares two int32 columns, <= kJoinFastTerms terms
   std::string err;
 };
 
@@ -257,9 +314,12 @@ static saber_status join_task(saber_join *j, const unsigned char *d1, const unsi
   JIn v1{j->carry[0][j->cur], d1, j->cpos, j->tpos, p.tb1, 0};
   JIn v2{j->carry[1][j->cur], d2, j->cpos, j->tpos, p.tb2, 0};
   const size_t smem = (size_t)kJoinThreads * p.tb1 + (size_t)kJoinChunk * p.tb2;
+  const bool fast = j->fast;
+  const size_t fsmem = (size_t)kJoinFastTerms * kJoinChunk * 4;
   if (nwin > 0) {
     const dim3 grid((unsigned)nwin, (unsigned)((p.s + kJoinThreads - 1) / kJoinThreads));
-    k_join_pairs<false><<<grid, kJoinThreads, smem, j->cs>>>(p, v1, v2, j->J0, j->counts, nullptr, nullptr);
+    if (fast) k_join_pairs_i32<false><<<grid, kJoinThreads, fsmem, j->cs>>>(p, v1, v2, j->J0, j->counts, nullptr, nullptr);
+    else k_join_pairs<false><<<grid, kJoinThreads, smem, j->cs>>>(p, v1, v2, j->J0, j->counts, nullptr, nullptr);
     JCK(cudaGetLastError());
     JCK(cudaMemsetAsync(j->ticket, 0, sizeof(int), j->cs));
     ++j->epoch;
@@ -267,7 +327,8 @@ static saber_status join_task(saber_join *j, const unsigned char *d1, const unsi
     k_join_scan<<<148 * 4, kJoinThreads, 0, j->cs>>>(j->counts, nwin * p.s, j->status, j->ticket, j->epoch,
                                                      s.d_total);
     JCK(cudaGetLastError());
-    k_join_pairs<true><<<grid, kJoinThreads, smem, j->cs>>>(p, v1, v2, j->J0, nullptr, j->counts, s.rows);
+    if (fast) k_join_pairs_i32<true><<<grid, kJoinThreads, fsmem, j->cs>>>(p, v1, v2, j->J0, nullptr, j->counts, s.rows);
+    else k_join_pairs<true><<<grid, kJoinThreads, smem, j->cs>>>(p, v1, v2, j->J0, nullptr, j->counts, s.rows);
     JCK(cudaGetLastError());
     k_join_hdr<<<148, 256, 0, j->cs>>>(p, v1, j->J0, nwin, j->counts, s.d_total, (WinHdr *)s.hdr);
     JCK(cudaGetLastError());
@@ -360,6 +421,8 @@ saber_status saber_join_create(const saber_schema *s1, const saber_schema *s2, c
     delete j;
     return jfail(nullptr, SABER_EINVAL, "bad projection column");
   }
+  j->fast = op->npred <= kJoinFastTerms && !std::getenv("SABER_JOIN_GENERIC");
+  for (int k = 0; k < op->npred; ++k) j->fast &= p.pred[k].t1 == T_I32 && p.pred[k].t2 == T_I32;
   if (cfg) j->cfg = *cfg;
   if (j->cfg.task_bytes <= 0) j->cfg.task_bytes = 32ll << 20;
   j->device = (cfg && cfg->device >= 0) ? cfg->device : 0;
