@@ -400,17 +400,27 @@ def run_join(args, rank, world):
     nwin = (n - size) // slide + 1
     tests = nwin * size * size
     tests_per_s = tests / (ms / 1e3)
-    # ALU roofline: a pair test needs at least a compare and a select per
-    # θ term on one INT32 lane; B200: 148 SMs x 128 INT32 lanes per clock
+    # two bounds: ALU -- a pair test needs at least a compare and a select
+    # per θ term on one INT32 lane (B200: 148 SMs x 128 INT32 lanes per clock); HBM -- the
+    # pair rows written.  The roofline reports the binding one (the larger time)
     clk_ghz = MEASURED_SM_GHZ
     peak = 148 * 128 * clk_ghz * 1e9 / (2 * args.join_r)
+    row_bytes = 16
+    hbm_peak, hbm_src = measured_peaks()
+    t_alu = tests / peak
+    t_hbm = pairs * row_bytes / (hbm_peak * 1e9)
     line = {"metric": METRIC, "value": 2 * n / (ms / 1e3), "unit": "tuples/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "i32", "data": "synthetic",
             "config": {"workload": name, "task_tuples": batch, "windows_per_step": nwin, "pairs_out_per_step": pairs},
-            "roofline": {"bound": "alu", "achieved": tests_per_s, "peak": peak, "unit": "pair tests/s",
-                         "frac": tests_per_s / peak, "peak_source": "derived: 148 SMs x 128 INT32 lanes x SM clock / "
-                                                                    "(2 instructions x r terms per pair test)"},
+            "roofline": ({"bound": "alu", "achieved": tests_per_s, "peak": peak, "unit": "pair tests/s",
+                          "frac": tests_per_s / peak,
+                          "peak_source": "derived: 148 SMs x 128 INT32 lanes x SM clock / (2 instructions x r terms "
+                                         "per pair test)"} if t_alu >= t_hbm else
+                         {"bound": "hbm", "achieved": pairs * row_bytes / (ms / 1e3) / 1e9, "peak": hbm_peak,
+                          "unit": "GB/s", "frac": pairs * row_bytes / (ms / 1e3) / 1e9 / hbm_peak,
+                          "peak_source": hbm_src, "note": "pair rows written (16 B each)"}) |
+                        {"pair_tests_per_s": tests_per_s, "alu_bound_ms": t_alu * 1e3, "hbm_bound_ms": t_hbm * 1e3},
             "clocks": clk.summary(), "gpu_launches": 5 * nt}
     if rank == 0:
         print(json.dumps(line), flush=True)

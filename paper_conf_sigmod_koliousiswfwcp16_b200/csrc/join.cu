@@ -144,8 +144,17 @@ k_join_pairs_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, int64_t *__restri
   const int np = p.npred;
   const unsigned char *ta = act ? jtuple(v1, base + a_loc) : nullptr;
   int32_t av[kJoinFastTerms];
+  uint32_t om[kJoinFastTerms];                                 // outcome bits of op: lt | eq << 1 | gt << 2
 #pragma unroll
-  for (int k = 0; k < kJoinFastTerms; ++k) av[k] = (act && k < np) ? *(const int32_t *)(ta + 4 * p.pred[k].w1) : 0;
+  for (int k = 0; k < kJoinFastTerms; ++k) {
+    av[k] = (act && k < np) ? *(const int32_t *)(ta + 4 * p.pred[k].w1) : 0;
+    const int op = k < np ? p.pred[k].op : OP_EQ;
+    om[k] = op == OP_LT ? 1u : op == OP_LE ? 3u : op == OP_GT ? 4u : op == OP_GE ? 6u : op == OP_EQ ? 2u : 5u;
+  }
+  auto term = [&](int k, int32_t b) -> uint32_t {          // a_k op b as one bit, branch-free
+    const int32_t a = av[k];
+    return (om[k] >> (a < b ? 0 : (a == b ? 1 : 2))) & 1u;
+  };
   int64_t cnt = 0, out = 0;
   if (EMIT && act) out = offs[w * p.s + a_loc];
   const int orow = 4 * (p.nw1 + p.nw2);
@@ -160,14 +169,24 @@ k_join_pairs_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, int64_t *__restri
     }
     __syncthreads();
     if (!act) continue;
+    if constexpr (!EMIT) {
+      // count pass: independent iterations, unrolled so the broadcast shared loads overlap
+#pragma unroll 8
+      for (int bi = 0; bi < nb; ++bi) {
+        uint32_t ok = 1u;
+#pragma unroll
+        for (int k = 0; k < kJoinFastTerms; ++k)
+          if (k < np) ok &= term(k, col[k * kJoinChunk + bi]);
+        cnt += ok;
+      }
+    } else {
+#pragma unroll 4
     for (int bi = 0; bi < nb; ++bi) {
-      bool ok = true;
+      uint32_t ok = 1u;
 #pragma unroll
       for (int k = 0; k < kJoinFastTerms; ++k)
-        if (k < np) ok &= cmp_op(av[k], p.pred[k].op, col[k * kJoinChunk + bi]);
-      if (!EMIT) {
-        cnt += ok;
-      } else if (ok) {
+        if (k < np) ok &= term(k, col[k * kJoinChunk + bi]);
+      if (ok) {
         if (out < p.rows_cap) {
           const unsigned char *tb = jtuple(v2, base + c0 + bi);
           uint32_t *dst = (uint32_t *)(rows + out * orow);
@@ -176,6 +195,7 @@ k_join_pairs_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, int64_t *__restri
         }
         ++out;
       }
+    }
     }
   }
   if (!EMIT && act) counts[w * p.s + a_loc] = cnt;
