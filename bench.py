@@ -289,6 +289,20 @@ def cpu_oracle_sample(spec, g, budget_s, threads):
     return value, sample, dt
 
 
+def run_config(args, spec, g, name, world):
+    """The workload's static description, identical for both arms (--impl saber /
+    reference); run-dependent counters are reported outside it."""
+    tb = spec["schema"]["tuple_bytes"]
+    n = g["n"]
+    return {"workload": name, "groups": args.groups if args.config == "C3" else None,
+            "task_bytes": (args.task_mb or workloads.bench_task_mb(args.config, args.groups)) << 20,
+            "tuples_per_gpu": n,
+            "l2": ("flushed: a 512 MiB memset before every step (input < 2x the 126 MB L2)"
+                   if n * tb < (256 << 20) else
+                   f"inputs ({n * tb >> 20} MiB per GPU) exceed the 126 MB L2: no flush needed"),
+            "parallelism": f"dp{world} (stream partitions + halo)"}
+
+
 def run_reference(args, spec, g, name, rank, world):
     if rank != 0:
         return
@@ -302,7 +316,7 @@ def run_reference(args, spec, g, name, rank, world):
     line = {"metric": METRIC, "value": value, "unit": "tuples/s", "impl": "reference", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": None, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": name, "groups": args.groups},
+            "config": run_config(args, spec, g, name, world),
             "cpu_baseline": {"value": value, "unit": "tuples/s", "cores": threads, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": value, "unit": "tuples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -698,13 +712,8 @@ def main():
                 "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
                 "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "input_gbs": total_tuples * tb / (ms_step / 1e3) / 1e9,
-                "config": {"workload": name, "groups": args.groups if args.config == "C3" else None,
-                           "task_bytes": task_bytes, "tuples_per_gpu": n,
-                           "l2": ("flushed: a 512 MiB memset before every step (input < 2x the 126 MB L2)"
-                                  if n * tb < (256 << 20) else
-                                  f"inputs ({n * tb >> 20} MiB per GPU) exceed the 126 MB L2: no flush needed"),
-                           "windows_per_step": out_windows, "rows_per_step": out_rows,
-                           "out_tuples_per_step": out_tuples, "parallelism": f"dp{world} (stream partitions + halo)"},
+                "config": run_config(args, spec, g, name, world),
+                "output_per_step": {"windows": out_windows, "rows": out_rows, "out_tuples": out_tuples},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": launches}
         print(json.dumps(line), flush=True)

@@ -24,8 +24,17 @@
 namespace sb {
 
 constexpr int kSelThreads = 256, kSelWarps = 8;
-constexpr int kSelStageBytes = 32768;
-constexpr int kSelStages = 3;
+#ifndef SB_SEL_STAGE_KB
+#define SB_SEL_STAGE_KB 32
+#endif
+#ifndef SB_SEL_STAGES
+#define SB_SEL_STAGES 3
+#endif
+#ifndef SB_SEL_BPS
+#define SB_SEL_BPS 2
+#endif
+constexpr int kSelStageBytes = SB_SEL_STAGE_KB * 1024;
+constexpr int kSelStages = SB_SEL_STAGES;
 constexpr int kSelMaxIter = kSelStageBytes / 16 / kSelThreads;   // tuples per thread per stage (16-B tuples)
 
 __device__ __forceinline__ int64_t sel_s_int(const unsigned char *t, int word, int type) {
@@ -35,7 +44,7 @@ __device__ __forceinline__ double sel_s_flt(const unsigned char *t, int word, in
   return type == T_F32 ? (double)*(const float *)(t + 4 * word) : *(const double *)(t + 4 * word);
 }
 
-__global__ void __launch_bounds__(kSelThreads, 2)
+__global__ void __launch_bounds__(kSelThreads, SB_SEL_BPS)
 k_select(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ task,
          const unsigned char *__restrict__ carry0, const unsigned char *__restrict__ carry1,
          unsigned char *__restrict__ stage_rows, int64_t *__restrict__ cta_cnt,
