@@ -771,6 +771,9 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     const int ntup = range32 - xs < ST ? range32 - xs : ST;
     int pf = divg(p, R0 + xs);
     const int pl = divg(p, R0 + xs + ntup - 1);
+    // τ of every pane's first tuple in this stage (header ts of count windows, A7)
+    for (int qq = divg(p, R0 + xs + g - 1) + tid; qq * g < R0 + xs + ntup; qq += kP1Threads)
+      if (qq >= minrel) pane_ts[(P0 + qq) & Rm] = lds_s64(sb + (uint32_t)((qq * g - R0 - xs) * tb) + tsoff);
     if (pf < minrel) pf = minrel;
     const int ie = ib + per_warp < ntup ? ib + per_warp : ntup;
     bool first_round = true;
@@ -804,7 +807,6 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
           const int64_t up = i > 0 ? lds_s64(t - tb + tsoff) : prev_last;
           if (valid & (tau < up)) err |= ERR_ORDER;
           if (valid & (tau < 0)) err |= ERR_TS;
-          if (valid && rel == q * g && q >= minrel) pane_ts[(P0 + q) & Rm] = tau;
         }
         const int po = q - prel;
         if (!all_in) valid &= (po >= lo_ofs) & (po < PL);

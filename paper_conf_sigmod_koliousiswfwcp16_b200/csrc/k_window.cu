@@ -798,6 +798,10 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
   int64_t *scnt = (int64_t *)(skeys + ST);
   uint64_t *sf = (uint64_t *)(scnt + ST);
   double *sc = (double *)(sf + (size_t)p.nf * ST);     // TwoSum compensation of FK_SUM_F fields
+  // occupied state slots of the item, in insertion order: keys are never removed
+  // within an item, so windows scan only these instead of all ST slots
+  int *occ = (int *)(sc + (size_t)p.nf * ST);
+  __shared__ int s_nocc;
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
   if (nw <= 0) return;
   const int64_t maxprobe = (int64_t)st->max_probe;
@@ -816,6 +820,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
       scnt[h] = 0;
       FOR_F(f) { sf[f * ST + h] = field_identity(p.field[f].kind); sc[f * ST + h] = 0.0; }
     }
+    if (threadIdx.x == 0) s_nocc = 0;
     __syncthreads();
     auto find = [&](uint64_t k) -> int {
       uint32_t h = (uint32_t)(fmix64(k) >> 32) & (uint32_t)(ST - 1);
@@ -825,6 +830,7 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
         if (cur == k) return (int)h;
         if (cur == kEmpty) {
           uint64_t old = atomicCAS((unsigned long long *)&skeys[h], kEmpty, k);
+          if (old == kEmpty) occ[atomicAdd(&s_nocc, 1)] = (int)h;
           if (old == kEmpty || old == k) return (int)h;
         }
         h = (h + 1) & (uint32_t)(ST - 1);
@@ -864,21 +870,27 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
         for (int64_t q = (j - 1) * p.L; q < j * p.L; ++q) visit_pane(q, -1, false);
       }
       __syncthreads();
-      for (int h = threadIdx.x; h < ST; h += blockDim.x)
+      const int nocc = s_nocc;
+      for (int x = threadIdx.x; x < nocc; x += blockDim.x) {
+        const int h = occ[x];
         if (scnt[h] == 0)
           FOR_F(f)
             if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) { sf[f * ST + h] = 0; sc[f * ST + h] = 0.0; }
+      }
       if (p.has_minmax) {
-        for (int h = threadIdx.x; h < ST; h += blockDim.x)
+        for (int x = threadIdx.x; x < nocc; x += blockDim.x)
           FOR_F(f)
-            if (p.field[f].kind == FK_MIN || p.field[f].kind == FK_MAX) sf[f * ST + h] = field_identity(p.field[f].kind);
+            if (p.field[f].kind == FK_MIN || p.field[f].kind == FK_MAX)
+              sf[f * ST + occ[x]] = field_identity(p.field[f].kind);
         __syncthreads();
         for (int64_t q = j * p.L; q < j * p.L + p.K; ++q) visit_pane(q, 0, true);
       }
       __syncthreads();
       int my = 0;
       uint64_t fv[kMaxField];
-      for (int h = threadIdx.x; h < ST; h += blockDim.x) {
+      const int nocc2 = s_nocc;                         // the min/max visit may have added keys
+      for (int x = threadIdx.x; x < nocc2; x += blockDim.x) {
+        const int h = occ[x];
         if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
         FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
             __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];
@@ -891,7 +903,8 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
         if (threadIdx.x == 0) counts[ci] = total;
       } else {
         int64_t r = counts[ci] + excl;
-        for (int h = threadIdx.x; h < ST; h += blockDim.x) {
+        for (int x = threadIdx.x; x < nocc2; x += blockDim.x) {
+          const int h = occ[x];
           if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
           FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
             __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];

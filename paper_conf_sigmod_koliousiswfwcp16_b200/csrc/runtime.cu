@@ -436,7 +436,7 @@ static saber_status size_plan(saber_query *q) {
       (void)gpb; (void)smem_budget;
     } else {
       p.GS = 256;
-      p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + 2 * p.nf)));   // keys, counts, fields, compensation
+      p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + 2 * p.nf) + 4));   // keys, counts, fields, compensation, occupancy list
       const double A = (double)(p.K + q->win_chunk * p.L) / 2.0;
       const double B = p.key_pack == KP_RADIX ? (double)p.G / (double)p.C : 1e30;
       const double per_slot = std::max(1e-9, std::min(A, B));
@@ -444,7 +444,7 @@ static saber_status size_plan(saber_query *q) {
       if (sb > p.C) sb = p.C;
       p.SB = (int)sb;
       p.S = (int)(p.C / sb);
-      p.p2_smem = p.state_cap * 8 * (2 + 2 * p.nf);
+      p.p2_smem = p.state_cap * (8 * (2 + 2 * p.nf) + 4);
       // radix-packed keys with a declared domain: key-range slabs with a dense
       // shared-memory state (48 KiB) over compacted pane buckets
       if (p.key_pack == KP_RADIX && p.G < (1ll << 31)) {
