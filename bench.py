@@ -66,6 +66,8 @@ def parse():
     ap.add_argument("--hash-capacity", type=int, default=0,
                     help="pane hash-table slots (power of two; 0: the planner's guess).  CM2 defaults to "
                          "2x the expected distinct jobIds per pane (the paper's static hash-table pool, L1293-1295)")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo: multi-rank plumbing check with ranks sharing GPUs (collectives via the host)")
     ap.add_argument("--launcher-check", action="store_true",
                     help="CPU (gloo) check of the multi-rank launch: no GPU work")
     return ap.parse_args()
@@ -454,6 +456,11 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.dist_backend == "gloo":
+        # plumbing check of the multi-rank path on a box with fewer GPUs than ranks:
+        # ranks share the visible GPUs round-robin, collectives go through the host
+        import torch
+        local = local % max(1, torch.cuda.device_count())
     if world != args.gpus:
         print(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}", file=sys.stderr)
         sys.exit(2)
@@ -464,7 +471,10 @@ def main():
     import torch.distributed as dist
     if world > 1:
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.dist_backend == "gloo":
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     if args.impl == "reference":
         run_reference(args, spec, g, name, rank, world)
         if world > 1:
@@ -492,7 +502,7 @@ def main():
     def max_over_ranks(x):
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device=dev if args.dist_backend == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
@@ -530,8 +540,18 @@ def main():
     # partition planning metadata (first window / base index) is fixed by the data;
     # the query objects are created outside the timed region, the halo bytes are
     # exchanged inside it every step.
+    def halo_exchange():
+        if args.dist_backend == "nccl":
+            return exchange_halo(spec, part, begin, n, rank, world)
+        # gloo (plumbing check, small partitions): the window arithmetic on the device
+        # (saber_partition_plan), the bytes through the host
+        from paper_conf_sigmod_koliousiswfwcp16_b200.saber import partition_plan
+        h, fw, bi = exchange_halo(spec, part.cpu(), begin, n, rank, world,
+                                  plan=lambda sp, pt, b, m: partition_plan(sp, part.data_ptr(), b, m))
+        return h.to(dev), fw, bi
+
     if world > 1:
-        _, first_window, base_index = exchange_halo(spec, part, begin, n, rank, world)
+        _, first_window, base_index = halo_exchange()
     else:
         first_window, base_index = 0, begin
     times, stats_acc = [], []
@@ -565,7 +585,7 @@ def main():
             ev0.record(stream)
             pieces = []
             if world > 1:
-                halo, fw, bi = exchange_halo(spec, part, begin, n, rank, world)
+                halo, fw, bi = halo_exchange()
                 assert (fw, bi) == (first_window, base_index)
                 if halo.numel():
                     pieces.append((halo.data_ptr(), halo.numel()))
@@ -646,7 +666,7 @@ def main():
             t0 = time.perf_counter()
             halo_np = None
             if world > 1:
-                halo, _, _ = exchange_halo(spec, part, begin, n, rank, world)
+                halo, _, _ = halo_exchange()
                 halo_np = halo.cpu().numpy() if halo.numel() else None
             got_bytes = 0
             chunks = []
