@@ -643,7 +643,9 @@ def main():
                 "launches_per_step": scan_launches / max(1, len(stats_acc)), "peak_source": peak_src,
                 "scan_grid": stats_acc[-1]["scan_grid"] if stats_acc else None,
                 "window_grid": stats_acc[-1]["window_grid"] if stats_acc else None,
-                "share_of_step": (scan_ms / max(1, len(stats_acc))) / ms_rank if ms_rank else None}
+                "share_of_step": (scan_ms / max(1, len(stats_acc))) / ms_rank if ms_rank else None,
+                "window_ms_per_step": sum(s["assemble_ms"] for s in stats_acc) / max(1, len(stats_acc)),
+                "overlap": bool(stats_acc[-1]["overlap"]) if stats_acc else None}
 
     # ---------------- end-to-end through the C ABI from pinned host memory
     e2e = None

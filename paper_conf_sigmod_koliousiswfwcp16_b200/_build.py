@@ -44,9 +44,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
         objdir = os.path.join(CSRC, "..", "build")
         os.makedirs(objdir, exist_ok=True)
         objs, procs = [], []
-        for f in cus:     # one nvcc per translation unit, in parallel
+        hdrs = [x for x in srcs if not x.endswith(".cu")]
+        for f in cus:     # one nvcc per stale translation unit, in parallel
             o = os.path.join(objdir, f[:-3] + ".o")
             objs.append(o)
+            if not force and not _stale(o, [os.path.join(CSRC, f), *hdrs]):
+                continue
             cmd = [NVCC, *ARCH, *[x for x in FLAGS if x != "-shared"], "-c", "-I", os.path.join(ROOT, "include"),
                    os.path.join(CSRC, f), "-o", o]
             if verbose:

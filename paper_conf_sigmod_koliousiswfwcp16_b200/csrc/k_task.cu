@@ -135,7 +135,8 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
     if (err) st->error |= err;
     st->tile_epoch += 1;
     st->sel_rows = st->row_base;
-    *tile_ctr = 0;
+    tile_ctr[0] = 0;
+    tile_ctr[1] = 0;
     sh[0] = J0; sh[1] = J1; sh[2] = pos0;
   }
   __syncwarp();

@@ -369,26 +369,324 @@ k_win_block(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ t
 }
 
 // ---------------------------------------------------------------------------
+// Row counts of the register variant's windows, before any value is assembled
+// (count-then-write, the shape of PAPER.md §5.4): on the FAST plan a
+// (window, key) row exists iff the key's window count is > 0, i.e. iff one of the
+// window's K panes counted the key.  Per pane, a ballot over its C count words
+// gives a presence bitmap (C/32 words, shared memory); a window's bitmap is the
+// OR of its K pane bitmaps and its row count the popcount.  A CTA takes 256
+// consecutive windows per ticket, scans their row counts, and a decoupled
+// look-back over the (cheap, evenly timed) tickets gives the global offsets; it
+// writes every window header.  The assembly kernel then reads its windows' row
+// offsets from the headers and never waits on another CTA.
+constexpr int kWrWin = 512;          // windows per ticket (two per thread)
+template <int NBW>
+__global__ void __launch_bounds__(kWbThreads)
+k_wb_rows(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table, const int64_t *__restrict__ pane_ts,
+          WinHdr *__restrict__ hdr, uint64_t *__restrict__ status, int *__restrict__ ticket) {
+  hdr += st->hdr_base;
+  __shared__ unsigned s_bm[kWrWin + 64][NBW];   // pane presence bitmaps (K <= 64)
+  __shared__ int s_t;
+  __shared__ int s_ws[8];
+  __shared__ int64_t s_base;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  const int W = (int)p.slot_words, K = (int)p.K;
+  const int64_t Rm = p.R - 1;
+  const uint64_t epoch = (uint64_t)st->tile_epoch;
+  const int64_t nitems = (J1 - J0 + kWrWin - 1) / kWrWin;
+  constexpr int U = 8;                            // panes in flight per warp
+  for (;;) {
+    if (tid == 0) s_t = atomicAdd(ticket, 1);
+    __syncthreads();
+    const int64_t t = s_t;
+    if (t >= nitems) break;
+    const int64_t j0 = J0 + t * kWrWin;
+    const int jn = (int)((J1 - j0) < kWrWin ? (J1 - j0) : kWrWin);
+    const int npanes = jn + K - 1;                    // panes [j0, j0 + npanes) (one-pane slides)
+    for (int x0 = warp * U; x0 < npanes; x0 += (kWbThreads / 32) * U) {
+      int64_t v[U][NBW];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const uint64_t *cw = table + ((j0 + x0 + u) & Rm) * W + lane;
+#pragma unroll
+        for (int z = 0; z < NBW; ++z)
+          v[u][z] = x0 + u < npanes ? (int64_t)__ldcg((const unsigned long long *)cw + z * 32) : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int z = 0; z < NBW; ++z) {
+          const unsigned bal = __ballot_sync(kFull, v[u][z] > 0);
+          if (lane == 0 && x0 + u < npanes) s_bm[x0 + u][z] = bal;
+        }
+    }
+    __syncthreads();
+    int n0 = 0, n1 = 0;
+    const int w0 = 2 * tid;
+#pragma unroll
+    for (int z = 0; z < NBW; ++z) {
+      if (w0 < jn) {
+        unsigned m = 0;
+        for (int k = 1; k < K; ++k) m |= s_bm[w0 + k][z];          // panes shared by both windows
+        n0 += __popc(m | s_bm[w0][z]);
+        if (w0 + 1 < jn) n1 += __popc(m | s_bm[w0 + K][z]);
+      }
+    }
+    const int n = n0 + n1;
+    // block exclusive scan of the row counts
+    int y = n;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int zz = __shfl_up_sync(kFull, y, o);
+      if (lane >= o) y += zz;
+    }
+    if (lane == 31) s_ws[warp] = y;
+    __syncthreads();
+    if (warp == 0) {
+      int v = lane < kWbThreads / 32 ? s_ws[lane] : 0, u = v;
+#pragma unroll
+      for (int o = 1; o < 8; o <<= 1) {
+        const int zz = __shfl_up_sync(kFull, u, o);
+        if (lane >= o) u += zz;
+      }
+      const int total = __shfl_sync(kFull, u, kWbThreads / 32 - 1);
+      if (lane < kWbThreads / 32) s_ws[lane] = u - v;
+      const int64_t excl = lookback_warp(status, t, epoch, (uint64_t)total, st->row_base);
+      if (lane == 0) {
+        s_base = excl;
+        if (t == nitems - 1) {
+          st->sel_rows = excl + (int64_t)total;
+          if (excl + (int64_t)total > p.rows_cap) atomicOr(&st->error, ERR_RESULT);
+        }
+      }
+    }
+    __syncthreads();
+    const int64_t off = s_base + s_ws[warp] + y - n;
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      if (w0 + e >= jn) break;
+      const int64_t j = j0 + w0 + e;
+      WinHdr h;
+      h.window_id = j;
+      h.ts = (p.win_kind == WK_TIME) ? p.T0 + j * p.l : pane_ts[j & Rm];
+      h.row_offset = off + (e ? n0 : 0);
+      h.nrows = e ? n1 : n0;
+      h.flags = 0;
+      hdr[j - J0] = h;
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Register variant of the FAST plan for one-pane slides (L = 1) over C = 32..256
+// dense keys (C3 at G = 64): an item is one K-aligned block of K window starts.
+// Warp w owns key chunk kc = w mod C/32 (lane = key within the chunk) and window
+// group g = w div C/32 (WPT = K/ng consecutive window starts, ng = 256/C groups).
+// The same van Herk / Gil-Werman decomposition as above, done in registers:
+//   V[i] = S[i] ⊕ P[i],  S[i] = ⊕ panes [bK+i, bK+K),  P[i] = ⊕ panes [(b+1)K, (b+1)K+i)
+// each thread walks its WPT panes of block b backwards (local suffixes) and its
+// WPT panes of block b+1 forwards (local prefixes); the group totals go through
+// shared memory, S[i] = local suffix ⊕ totals of the later groups of block b,
+// P[i] = totals of the earlier groups of block b+1 ⊕ local prefix.  Nothing is
+// written back into the staged panes, so the next ticket's bulk copies are issued
+// as soon as every thread has read them and overlap this item's presence ballots,
+// look-back and row writes.  One ballot per (window, key chunk) gives the
+// presence masks; a window's rows are its keys in order (prefix popcounts).
+template <int NF, int WPT>
+__global__ void __launch_bounds__(kWbThreads, 3)
+k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table,
+                const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
+                uint64_t *__restrict__ status, int *__restrict__ ticket, int NB) {
+  (void)NB; (void)status; (void)pane_ts;
+  ticket += 1;                                // [0] is k_wb_rows' ticket
+  hdr += st->hdr_base;
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ uint64_t bar;
+  __shared__ int s_t, s_next;
+  __shared__ unsigned s_mask[64][8];          // presence: [window of the block][key chunk]
+  __shared__ int64_t s_woff[64];              // first row of each window (k_wb_rows)
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t J0 = st->J0, J1 = st->J1;
+  if (J1 <= J0) return;
+  const int W = (int)p.slot_words;            // C·(1+nf) words per pane slot
+  const int C = (int)p.C, K = (int)p.K;
+  const int64_t Rm = p.R - 1;
+  const int nkc = C >> 5, ng = kWbThreads / C;
+  const int kc = warp % nkc, g = warp / nkc;
+  const int key = kc * 32 + lane;
+  const int64_t bfirst = J0 / K;
+  const int64_t nitems = (J1 - 1) / K - bfirst + 1;
+  const int NP = 2 * K - 1;                   // staged panes per item
+  uint64_t *raw = (uint64_t *)smem;           // [NP][W]
+  uint64_t *tot = raw + (size_t)NP * W;       // [2][ng][W]: group totals of blocks b and b+1
+  const int64_t qhi = J1 - 1 + K - 1;         // last pane read by the task's windows
+  const unsigned lt = (1u << lane) - 1u;
+  auto stage = [&](int64_t t) {               // thread 0: bulk copies of item t's panes
+    const int64_t q0 = (bfirst + t) * K;
+    const int64_t sa = q0 > J0 ? q0 : J0;
+    const int64_t se = (q0 + NP) < (qhi + 1) ? (q0 + NP) : (qhi + 1);
+    uint32_t bytes = 0;
+    for (int64_t q = sa; q < se;) {
+      const int64_t run = ((q | Rm) + 1 - q) < (se - q) ? ((q | Rm) + 1 - q) : (se - q);
+      bytes += (uint32_t)(run * W * 8);
+      q += run;
+    }
+    mbar_expect_tx(&bar, bytes);
+    for (int64_t q = sa; q < se;) {
+      const int64_t run = ((q | Rm) + 1 - q) < (se - q) ? ((q | Rm) + 1 - q) : (se - q);
+      for (int64_t d = 0; d < run;) {                      // <= 1 MiB per bulk copy
+        const int64_t n = (run - d) * W * 8 <= (1 << 20) ? (run - d) : ((1 << 20) / (W * 8));
+        bulk_g2s(raw + (q + d - q0) * W, table + ((q + d) & Rm) * W, (uint32_t)(n * W * 8), &bar);
+        d += n;
+      }
+      q += run;
+    }
+  };
+  if (tid == 0) {
+    mbar_init(&bar, 1);
+    fence_mbar_init();
+    s_t = atomicAdd(ticket, 1);
+    if (s_t < nitems) stage(s_t);
+  }
+  __syncthreads();
+  uint32_t phase = 0;
+  for (int64_t t = s_t; t < nitems; ) {
+    const int64_t q0 = (bfirst + t) * K;
+    mbar_wait(&bar, phase);
+    phase ^= 1u;
+    // ---- local suffixes over block b and local prefixes over block b+1
+    const int i0 = g * WPT;
+    int64_t c[WPT];
+    double f[NF][WPT];
+    {
+      int64_t ac = 0;
+      double af[NF];
+#pragma unroll
+      for (int x = 0; x < NF; ++x) af[x] = 0.0;
+#pragma unroll
+      for (int ii = WPT - 1; ii >= 0; --ii) {
+        const uint64_t *r = raw + (i0 + ii) * W + key;
+        ac += (int64_t)r[0];
+        c[ii] = ac;
+#pragma unroll
+        for (int x = 0; x < NF; ++x) {
+          af[x] += __longlong_as_double((long long)r[(1 + x) * C]);
+          f[x][ii] = af[x];
+        }
+      }
+      uint64_t *tb = tot + g * W + key;
+      tb[0] = (uint64_t)ac;
+#pragma unroll
+      for (int x = 0; x < NF; ++x) tb[(1 + x) * C] = (uint64_t)__double_as_longlong(af[x]);
+    }
+    {
+      int64_t ac = 0;
+      double af[NF];
+#pragma unroll
+      for (int x = 0; x < NF; ++x) af[x] = 0.0;
+#pragma unroll
+      for (int ii = 0; ii < WPT; ++ii) {
+        c[ii] += ac;                                        // local prefix: panes before i in the group
+#pragma unroll
+        for (int x = 0; x < NF; ++x) f[x][ii] += af[x];
+        const int qi = K + i0 + ii;
+        if (qi < NP) {
+          const uint64_t *r = raw + qi * W + key;
+          ac += (int64_t)r[0];
+#pragma unroll
+          for (int x = 0; x < NF; ++x) af[x] += __longlong_as_double((long long)r[(1 + x) * C]);
+        }
+      }
+      uint64_t *tb = tot + (ng + g) * W + key;
+      tb[0] = (uint64_t)ac;
+#pragma unroll
+      for (int x = 0; x < NF; ++x) tb[(1 + x) * C] = (uint64_t)__double_as_longlong(af[x]);
+    }
+    __syncthreads();
+    // every thread has read its staged panes: the next ticket's copies go now
+    if (tid == 0) {
+      fence_proxy_async_smem();
+      s_next = atomicAdd(ticket, 1);
+      if (s_next < nitems) stage(s_next);
+    }
+    // ---- window values: S[i] = local suffix ⊕ later groups of b, P[i] = earlier groups of b+1 ⊕ local prefix
+    {
+      int64_t tc = 0;
+      double tf[NF];
+#pragma unroll
+      for (int x = 0; x < NF; ++x) tf[x] = 0.0;
+      for (int h = g + 1; h < ng; ++h) {
+        const uint64_t *tb = tot + h * W + key;
+        tc += (int64_t)tb[0];
+#pragma unroll
+        for (int x = 0; x < NF; ++x) tf[x] += __longlong_as_double((long long)tb[(1 + x) * C]);
+      }
+      for (int h = 0; h < g; ++h) {
+        const uint64_t *tb = tot + (ng + h) * W + key;
+        tc += (int64_t)tb[0];
+#pragma unroll
+        for (int x = 0; x < NF; ++x) tf[x] += __longlong_as_double((long long)tb[(1 + x) * C]);
+      }
+#pragma unroll
+      for (int ii = 0; ii < WPT; ++ii) {
+        c[ii] += tc;
+#pragma unroll
+        for (int x = 0; x < NF; ++x) f[x][ii] += tf[x];
+      }
+    }
+    // ---- presence (no HAVING on the FAST plan: count > 0) of the item's windows
+    const int64_t ja = q0 > J0 ? q0 : J0;
+    const int64_t jb = (q0 + K) < J1 ? (q0 + K) : J1;
+    unsigned pres = 0;
+#pragma unroll
+    for (int ii = 0; ii < WPT; ++ii) {
+      const int64_t j = q0 + i0 + ii;
+      const bool pr = j >= ja && j < jb && c[ii] > 0;
+      pres |= (unsigned)pr << ii;
+      const unsigned bal = __ballot_sync(kFull, pr);
+      if (lane == 0) s_mask[i0 + ii][kc] = bal;
+    }
+    if (tid < K) {                                           // row offsets from k_wb_rows' headers
+      const int64_t j = q0 + tid;
+      s_woff[tid] = (j >= ja && j < jb) ? __ldcg((const long long *)&hdr[j - J0].row_offset) : 0;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int ii = 0; ii < WPT; ++ii) {
+      if (!((pres >> ii) & 1u)) continue;
+      const int i = i0 + ii;
+      int before = 0;
+      for (int z = 0; z < kc; ++z) before += __popc(s_mask[i][z]);
+      const int64_t row = s_woff[i] + before + __popc(s_mask[i][kc] & lt);
+      if (row >= p.rows_cap) continue;
+      if (p.nkeys) ((int32_t *)(rows + p.col_off[0]))[row] = key;
+#pragma unroll
+      for (int a = 0; a < kMaxAgg; ++a) {
+        if (a >= p.nagg) break;
+        const AggOut &o = p.agg[a];
+        double x = 0.0;
+#pragma unroll
+        for (int y = 0; y < NF; ++y)
+          if (y == o.field) x = f[y][ii];
+        uint64_t bits = o.fn == AG_COUNT ? (uint64_t)c[ii] : (uint64_t)__double_as_longlong(x);
+        if (o.fn == AG_AVG) bits = (uint64_t)__double_as_longlong(wb_div(x, (double)c[ii]));
+        ((uint64_t *)(rows + p.col_off[p.nkeys + a]))[row] = bits;
+      }
+    }
+    __syncthreads();
+    t = s_next;
+  }
+}
+
+// ---------------------------------------------------------------------------
 // host side: usable when an item's staged panes + window values fit in shared
 // memory and its windows / rounds fit the per-item arrays
 static int wb_nb(const Plan &p) {
   int nb = (int)((32 * p.L + p.K - 1) / p.K);     // about 32 windows per item
   return nb < 1 ? 1 : nb;
-}
-int wb_smem(const Plan &p) {
-  const int nb = wb_nb(p);
-  return (int)(((nb + 1) * p.K - 1 + (nb == 1 ? 0 : nb * p.K)) * p.slot_words * 8);
-}
-bool wb_usable(const Plan &p) {
-  if (p.key_mode == KM_HASH || p.nagg == 0 || p.K > 64 || (p.slot_words & 1)) return false;   // 16-B bulk copies
-  const int nb = wb_nb(p);
-  // the van Herk phase runs one thread per (block, word) and direction: too few
-  // words leave the CTA idle (C4's 4 keys), those plans keep k_vh_build + k_win_packed
-  if ((nb == 1 ? 2 * p.slot_words : nb * p.slot_words) < 64) return false;
-  const int64_t nwin = (nb * p.K + p.L - 1) / p.L + 1;
-  if (nwin > kWbMaxWin || (nwin * p.C + kWbThreads - 1) / kWbThreads > kWbMaxRounds) return false;
-  if (p.slot_words > kWbMaxWords) return false;
-  return wb_smem(p) <= 96 * 1024;
 }
 static bool wb_fast(const Plan &p) {
   if (p.nhave || p.has_minmax || p.nf > 2 || p.key_mode == KM_HASH) return false;
@@ -398,7 +696,45 @@ static bool wb_fast(const Plan &p) {
     if (p.agg[a].fn != AG_COUNT && p.agg[a].fn != AG_SUM && p.agg[a].fn != AG_AVG) return false;
   return !std::getenv("SABER_NO_WBFAST");
 }
+// register variant: FAST plan, one-pane slides, 32..256 dense keys (power of two),
+// fp64 sums only, K a multiple of the 256/C window groups with <= 16 windows per thread
+static int wbr_wpt(const Plan &p) {
+  if (!wb_fast(p) || p.L != 1 || p.key_mode == KM_HASH || p.C < 32 || p.C > 256 || (p.C & (p.C - 1))) return 0;
+  if (p.slot_words != p.C * (1 + p.nf) || p.nf < 1 || std::getenv("SABER_NO_WBREG")) return 0;
+  for (int f = 0; f < p.nf; ++f)
+    if (p.field[f].kind != FK_SUM_F) return 0;
+  const int64_t ng = kWbThreads / p.C;
+  if (p.K > 64 || p.K % ng) return 0;
+  const int64_t wpt = p.K / ng;
+  return (wpt == 4 || wpt == 8 || wpt == 16) ? (int)wpt : 0;
+}
+static int wbr_smem(const Plan &p) {
+  return (int)(((2 * p.K - 1) + 2 * (kWbThreads / p.C)) * p.slot_words * 8);
+}
+int wb_smem(const Plan &p) {
+  if (wbr_wpt(p)) return wbr_smem(p);
+  const int nb = wb_nb(p);
+  return (int)(((nb + 1) * p.K - 1 + (nb == 1 ? 0 : nb * p.K)) * p.slot_words * 8);
+}
+bool wb_usable(const Plan &p) {
+  if (p.key_mode == KM_HASH || p.nagg == 0 || p.K > 64 || (p.slot_words & 1)) return false;   // 16-B bulk copies
+  if (wbr_wpt(p)) return wbr_smem(p) <= 100 * 1024;
+  const int nb = wb_nb(p);
+  // the van Herk phase runs one thread per (block, word) and direction: too few
+  // words leave the CTA idle (C4's 4 keys), those plans keep k_vh_build + k_win_packed
+  if ((nb == 1 ? 2 * p.slot_words : nb * p.slot_words) < 64) return false;
+  const int64_t nwin = (nb * p.K + p.L - 1) / p.L + 1;
+  if (nwin > kWbMaxWin || (nwin * p.C + kWbThreads - 1) / kWbThreads > kWbMaxRounds) return false;
+  if (p.slot_words > kWbMaxWords) return false;
+  return wb_smem(p) <= 96 * 1024;
+}
 static void *wb_kernel(const Plan &p) {
+  if (const int wpt = wbr_wpt(p)) {
+    if (p.nf == 1) return wpt == 4 ? (void *)k_win_block_reg<1, 4> : wpt == 8 ? (void *)k_win_block_reg<1, 8>
+                                                                              : (void *)k_win_block_reg<1, 16>;
+    return wpt == 4 ? (void *)k_win_block_reg<2, 4> : wpt == 8 ? (void *)k_win_block_reg<2, 8>
+                                                               : (void *)k_win_block_reg<2, 16>;
+  }
   if (wb_fast(p)) return p.nf <= 1 ? (void *)k_win_block<1, true> : (void *)k_win_block<2, true>;
   return p.nf <= 1 ? (void *)k_win_block<1, false> : p.nf <= 2 ? (void *)k_win_block<2, false>
        : p.nf <= 4 ? (void *)k_win_block<4, false> : (void *)k_win_block<8, false>;
@@ -411,8 +747,14 @@ int wb_blocks_per_sm(const Plan &p) {
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, wb_kernel(p), kWbThreads, wb_smem(p));
   return b > 0 ? b : 1;
 }
+bool wb_prepass(const Plan &p) { return wbr_wpt(p) != 0; }
 cudaError_t launch_windows_block(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st) {
   const int nb = wb_nb(p);
+  if (wbr_wpt(p)) {     // row counts, offsets and headers first (k_wb_rows), then the values
+    void (*k)(const Plan, State *, const uint64_t *, const int64_t *, WinHdr *, uint64_t *, int *) =
+        p.C <= 32 ? k_wb_rows<1> : p.C <= 64 ? k_wb_rows<2> : p.C <= 128 ? k_wb_rows<4> : k_wb_rows<8>;
+    k<<<grid, kWbThreads, 0, st>>>(p, q.st, q.table, q.pane_ts, (WinHdr *)s.hdr, q.tile_status, q.tile_ctr);
+  }
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&q.table, (void *)&q.pane_ts, (void *)&s.hdr, (void *)&s.rows,
                   (void *)&q.tile_status, (void *)&q.tile_ctr, (void *)&nb};
   return cudaLaunchKernel(wb_kernel(p), dim3(grid), dim3(kWbThreads), args, (size_t)wb_smem(p), st);

@@ -102,7 +102,7 @@ cudaError_t launch_agg_round(const Plan &p, const QueryDev &q, const SlotDev &s,
     if ((e = launch_windows_fused(p, q, s, p2_grid, st))) return e;
   }
   if ((e = launch_task_end(p, q, s, st))) return e;
-  *launches += p.bucket_mode ? 1 : p.key_mode == KM_HASH ? 4 : p.win_wide && !p.nhave ? 5 : 3;   // k_win_wide: + count + scan
+  *launches += p.bucket_mode ? 1 : p.key_mode == KM_HASH ? 4 : p.win_wide && !p.nhave ? 5 : p.win_block && wb_prepass(p) ? 4 : 3;   // k_win_wide: + count + scan; k_win_block_reg: + k_wb_rows
   if (evs) cudaEventRecord(evs[2], st);
   return cudaGetLastError();
 }
@@ -129,7 +129,7 @@ cudaError_t launch_agg_task_overlap(const Plan &p, const QueryDev &q, const Slot
   }
   if (evs) cudaEventRecord(evs[1], cs);
   if ((e = cudaMemcpyAsync(s.wst, q.st, sizeof(State), cudaMemcpyDeviceToDevice, cs))) return e;
-  if ((e = cudaMemsetAsync(s.ticket, 0, sizeof(int), cs))) return e;
+  if ((e = cudaMemsetAsync(s.ticket, 0, 2 * sizeof(int), cs))) return e;
   if ((e = launch_task_end(p, q, s, cs))) return e;
   if ((e = cudaEventRecord(scan_done, cs))) return e;
   if ((e = cudaStreamWaitEvent(ws, scan_done, 0))) return e;
@@ -140,7 +140,7 @@ cudaError_t launch_agg_task_overlap(const Plan &p, const QueryDev &q, const Slot
   else e = launch_windows_fused(p, qw, s, p2_grid, ws);
   if (e) return e;
   if ((e = launch_win_end(q, s, ws))) return e;
-  *launches += p.win_block ? 3 : p.win_wide && !p.nhave ? 6 : 4;
+  *launches += p.win_block ? (wb_prepass(p) ? 4 : 3) : p.win_wide && !p.nhave ? 6 : 4;
   if (evs) cudaEventRecord(evs[2], ws);
   return cudaGetLastError();
 }

@@ -37,6 +37,7 @@ cudaError_t launch_bucket_scan(const Plan &p, const QueryDev &q, const void *tup
 cudaError_t launch_bucket_windows(const Plan &p, const QueryDev &q, const SlotDev &s, int nsm, cudaStream_t st);
 // k_winblock.cu
 bool wb_usable(const Plan &p);
+bool wb_prepass(const Plan &p);   // k_win_block_reg: k_wb_rows runs first
 cudaError_t wb_set_attributes(const Plan &p);
 int wb_blocks_per_sm(const Plan &p);
 cudaError_t launch_windows_block(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st);

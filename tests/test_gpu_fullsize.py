@@ -229,8 +229,9 @@ def run_stream(S, oracle, spec, g, task_bytes, sample=None, full=False):
 
     stream = torch.cuda.current_stream().cuda_stream
     off, nbytes = 0, part.numel()
+    eff = q.stats()["task_tuples"] * tb             # effective φ (the dispatcher may cut smaller tasks)
     while off < nbytes:
-        nb = min(task_bytes, nbytes - off)
+        nb = min(eff, nbytes - off)
         st = q.submit_device(part.data_ptr() + off, nb, stream)
         if st == S.EAGAIN:
             drain()
