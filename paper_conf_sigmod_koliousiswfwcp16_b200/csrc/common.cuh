@@ -101,6 +101,13 @@ __device__ __forceinline__ bool s_preds(const Plan &p, const unsigned char *t) {
 }
 
 __device__ __forceinline__ int64_t cnt_off(const Plan &p) { return p.key_mode == KM_HASH ? p.C : 0; }
+// pane presence bitmaps (Plan::pane_bm): [R][8] u32 right after the ring's R slots
+__device__ __forceinline__ uint32_t *pane_bm_words(const Plan &p, uint64_t *table) {
+  return (uint32_t *)(table + p.R * p.slot_words);
+}
+__device__ __forceinline__ const uint32_t *pane_bm_words(const Plan &p, const uint64_t *table) {
+  return (const uint32_t *)(table + p.R * p.slot_words);
+}
 __device__ __forceinline__ int64_t fld_off(const Plan &p, int f) { return cnt_off(p) + (int64_t)(1 + f) * p.C; }
 
 // --------------------------------------------------------------------------

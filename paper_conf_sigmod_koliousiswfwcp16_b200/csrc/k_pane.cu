@@ -131,10 +131,12 @@ __device__ __forceinline__ void atom_field(int kind, uint64_t *addr, uint64_t v)
 }
 
 // add one pre-aggregated (pane, key) entry into the device pane ring
-template <int NF>
+template <int NF, bool BM = true>
 __device__ __forceinline__ void flush_entry(const Plan &p, State *st, uint64_t *table, int64_t pane, uint64_t key,
                                             uint32_t c, const uint64_t (&fv)[NF], int &err) {
   uint64_t *base = table + (pane & (p.R - 1)) * p.slot_words;
+  if (BM && p.pane_bm)                          // dense keys only (C <= 256): presence bit of (pane, key)
+    atomicOr(pane_bm_words(p, table) + (pane & (p.R - 1)) * 8 + (key >> 5), 1u << (key & 31));
   int64_t idx;
   if (p.key_mode == KM_HASH) {
     idx = global_insert(p, st, base, key, err);
@@ -639,8 +641,9 @@ __device__ __forceinline__ uint32_t sel4c(const uint4 &v) {
 // scripts/ubench_pane_accum.cu: 0.82 -> 0.30 SM-cycles per update).  A limb
 // receives at most g chunks of <= 0xffff between flushes, so it cannot wrap.
 // Any other value (negative, >= 1, finer than 2^-32, non-finite) is added in
-// fp64 straight into the device pane ring (RED.ADD.F64), so every f32 input is
-// summed; the flush converts the limbs exactly (< 2^53) and adds them.
+// fp64 into a CTA-wide side table (shared CAS loop, a rare path), so every f32
+// input is summed; the flush converts the limbs exactly (< 2^53) and adds the
+// side word.
 __device__ __forceinline__ bool fx32(uint32_t xb, uint32_t &X) {
   const uint32_t ex = (xb >> 23) & 0xffu;
   const uint32_t m = (xb & 0x7fffffu) | 0x800000u;
@@ -660,13 +663,21 @@ __device__ __forceinline__ void red_add_s(uint32_t saddr, uint32_t v) {
 
 // flush of FX tables: sum the copies' count and limbs of each entry, one set of
 // L2 REDs per (pane, key) per CTA (as flush_tables); CTA-collective
+// Panes wholly inside this CTA's tuples (selfzero, CTA-relative pane r with
+// r·g - R0 in [0, range - g]) have no other writer: their slots are written with
+// plain stores, zeros for absent keys included, so k_zero_panes skips them and no
+// RED has to fetch their lines (k_zero_panes initialises only the panes that hold
+// a CTA boundary).  side: per entry, the fp64 sum of the values the limbs cannot
+// hold (added into the ring by the flush, never straight into the table).
 template <int MODE>
 __device__ __forceinline__ void flush_fx(const Plan &p, State *st, uint64_t *table, unsigned char *tabs,
-                                         int64_t pbase, int &err) {
+                                         int64_t pbase, int &err, double *side, int selfzero, int64_t P0, int R0,
+                                         int range, int minrel) {
   const int tid = threadIdx.x;
   const int TE = p.local_entries;
   constexpr int NCOPY = MODE == TM_SHARED ? 1 : kP1Warps;
   const int C = (int)p.C;
+  const int64_t g = p.g, Rm = p.R - 1;
   __syncthreads();
   for (int e = tid; e < TE; e += kP1Threads) {
     uint32_t c = 0;
@@ -682,9 +693,27 @@ __device__ __forceinline__ void flush_fx(const Plan &p, State *st, uint64_t *tab
       lm[2 * e] = 0;
       lm[2 * e + 1] = 0;
     }
-    if (c) {
-      const uint64_t fv[1] = {(uint64_t)__double_as_longlong((double)X * 0x1p-32)};   // exact: X < 2^53
-      flush_entry<1>(p, st, table, pbase + e / C, (uint64_t)(e % C), c, fv, err);
+    const double sx = side[e];
+    side[e] = 0.0;
+    const int64_t pane = pbase + e / C;
+    const int64_t r = pane - P0, t0 = r * g - R0;
+    const bool own = selfzero && r >= minrel && t0 >= 0 && t0 + g <= range;
+    if (p.pane_bm) {                          // 32 consecutive entries: one pane, one 32-key chunk
+      const unsigned bal = __ballot_sync(kFull, c != 0);
+      uint32_t *bw = pane_bm_words(p, table) + (pane & Rm) * 8 + (e % C) / 32;
+      if ((tid & 31) == 0) {
+        if (own) *bw = bal;
+        else if (bal) atomicOr(bw, bal);
+      }
+    }
+    const double sum = (double)X * 0x1p-32 + sx;                                       // limbs exact: X < 2^53
+    if (own) {
+      uint64_t *base = table + (pane & Rm) * p.slot_words;
+      base[e % C] = (uint64_t)c;
+      base[C + e % C] = (uint64_t)__double_as_longlong(sum);
+    } else if (c) {
+      const uint64_t fv[1] = {(uint64_t)__double_as_longlong(sum)};
+      flush_entry<1, false>(p, st, table, pane, (uint64_t)(e % C), c, fv, err);
     }
   }
   __syncthreads();
@@ -693,7 +722,7 @@ __device__ __forceinline__ void flush_fx(const Plan &p, State *st, uint64_t *tab
 template <int MODE, int NF, int KK, int OC, bool FX = false>
 __global__ void __launch_bounds__(kP1Threads, MODE == TM_DIRECT ? SB_P1_DIRECT_BPS : 2)
 k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict__ tup, int64_t n,
-           uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts) {
+           uint64_t *__restrict__ table, int64_t *__restrict__ pane_ts, int selfzero) {
   constexpr bool ONECH = OC != 0;
   static_assert(OC != 2 || NF == 1, "fixed layout: one value column");
   extern __shared__ __align__(128) unsigned char smem[];
@@ -706,6 +735,10 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
   unsigned char *tabs = (unsigned char *)(empty + kStages);
   const int TE = p.local_entries;
   const int CW = MODE == TM_LANE ? 32 : 1;
+  // FX: fp64 side table of values the limbs cannot hold, one word per entry (CTA-wide)
+  double *side = (double *)(tabs + (size_t)(MODE == TM_SHARED ? 1 : kP1Warps) * p.local_bytes);
+  if (FX)
+    for (int e = tid; e < TE; e += kP1Threads) side[e] = 0.0;
   unsigned char *wt = tabs + (MODE == TM_SHARED ? 0 : (size_t)wid * p.local_bytes);
   uint64_t *tf = (uint64_t *)wt;                                    // [NF][TE*CW]
   uint32_t *tcnt = (uint32_t *)(wt + (size_t)8 * TE * CW * NF);     // [TE*CW]
@@ -780,7 +813,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     for (int cur = pf; cur <= pl;) {
       if (prel < 0 || cur < prel || cur >= prel + PL) {
         if (prel >= 0) {
-          if (FX) flush_fx<MODE>(p, st, table, tabs, P0 + prel, err);
+          if (FX) flush_fx<MODE>(p, st, table, tabs, P0 + prel, err, side, selfzero, P0, R0, range32, minrel);
           else flush_tables<MODE, NF, true>(p, st, table, tabs, tf, tcnt, P0 + prel, err);
         }
         prel = cur;
@@ -858,7 +891,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
               red_add_s(lm, X & 0xffffu);
               red_add_s(lm + 4u, X >> 16);
             } else {
-              atomicAdd((double *)&table[((P0 + prel + po) & Rm) * p.slot_words + p.C + key], fv[0]);
+              atomicAdd(&side[e], fv[0]);
             }
           } else {
             const int e = po * C + (int)key;
@@ -885,7 +918,7 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
     if (++slot == kStages) { slot = 0; phase ^= 1u; }
   }
   if (prel >= 0) {
-    if (FX) flush_fx<MODE>(p, st, table, tabs, P0 + prel, err);
+    if (FX) flush_fx<MODE>(p, st, table, tabs, P0 + prel, err, side, selfzero, P0, R0, range32, minrel);
     else flush_tables<MODE, NF, true>(p, st, table, tabs, tf, tcnt, P0 + prel, err);
   }
   if (err) atomicOr(&st->error, err);
@@ -894,8 +927,10 @@ k_pane_cnt(const Plan p, State *__restrict__ st, const unsigned char *__restrict
 // ---------------------------------------------------------------- host side
 int p1_nf_template(int nf) { return nf <= 1 ? 1 : nf <= 2 ? 2 : nf <= 4 ? 4 : 8; }
 
+static bool p1_cnt_fx(const Plan &p);
 int p1_smem_bytes(const Plan &p) {
-  return kStages * kStageBytes + 2 * kStages * 8 + (p.local_mode == TM_SHARED ? 1 : kP1Warps) * p.local_bytes;
+  return kStages * kStageBytes + 2 * kStages * 8 + (p.local_mode == TM_SHARED ? 1 : kP1Warps) * p.local_bytes +
+         (p1_cnt_fx(p) ? (p.local_entries * 8 + 15) / 16 * 16 : 0);     // FX side table
 }
 
 template <int M, int WK, int NK>
@@ -985,6 +1020,13 @@ static void *p1_cnt(const Plan &p) {
   }
 }
 bool p1_is_cnt(const Plan &p) { return p1_cnt(p) != nullptr; }
+// the count kernel p1_cnt picks is an FX instance (flush_fx: side table, plain
+// stores into the panes a CTA owns)
+static bool p1_cnt_fx(const Plan &p) {
+  if (!p1_cnt(p) || (p.local_mode != TM_DIRECT && p.local_mode != TM_SHARED)) return false;
+  const int kk = p.key_mode == KM_GLOBAL ? KK_GLOBAL : KK_RADIX;
+  return syn_layout(p, kk) && fx_ok(p);
+}
 void *p1_kernel(const Plan &p) {
   void *k = p1_cnt(p);
   return k ? k : p1_generic(p);
@@ -1002,16 +1044,37 @@ int p1_blocks_per_sm(const Plan &p) {
   return b > 0 ? b : 1;
 }
 
+// the scan kernel and grid of a task of n tuples; k_pane_cnt initialises the pane
+// slots that lie wholly inside one CTA's tuples itself (*per = its tuples per CTA,
+// 0 for the other kernels)
+static void *p1_choose(const Plan &p, int64_t n, int grid, int *g, int64_t *per) {
+  const int64_t stage_t = kStageBytes / p.tuple_bytes;
+  int64_t need = (n + stage_t - 1) / stage_t;     // at least one stage per CTA
+  *g = (int)(need < grid ? need : grid);
+  if (*g < 1) *g = 1;
+  // the fast count kernel keeps CTA-relative positions and panes in 32 bits
+  void *k = p1_cnt(p);
+  if (!k || (n / *g + stage_t + p.g) >= (1ll << 30)) k = nullptr;
+  // the fixed Syn layout reads 32-B tuples (k_pane_cnt: tb = 32, ST = kStageBytes / 32)
+  const int64_t st_t = kStageBytes / p.tuple_bytes;
+  *per = k && p1_cnt_fx(p) && !p.overlap && !std::getenv("SABER_NO_SELFZERO")
+             ? ((n + *g - 1) / *g + st_t - 1) / st_t * st_t : 0;
+  return k ? k : p1_generic(p);
+}
+int64_t p1_selfzero_per(const Plan &p, int64_t n, int grid, int *g) {
+  int64_t per;
+  p1_choose(p, n, grid, g, &per);
+  return n > 0 ? per : 0;
+}
 cudaError_t launch_pane_agg(const Plan &p, const QueryDev &q, const void *tuples, int64_t n, int grid,
                             cudaStream_t st) {
   if (n <= 0) return cudaSuccess;
-  const int64_t stage_t = kStageBytes / p.tuple_bytes;
-  int64_t need = (n + stage_t - 1) / stage_t;     // at least one stage per CTA
-  int g = (int)(need < grid ? need : grid);
-  void *args[] = {(void *)&p, (void *)&q.st, (void *)&tuples, (void *)&n, (void *)&q.table, (void *)&q.pane_ts};
-  // the fast count kernel keeps CTA-relative positions and panes in 32 bits
-  void *k = p1_cnt(p);
-  if (!k || (n / g + stage_t + p.g) >= (1ll << 30)) k = p1_generic(p);
+  int g;
+  int64_t per;
+  void *k = p1_choose(p, n, grid, &g, &per);
+  int sz = per > 0;
+  void *args[] = {(void *)&p, (void *)&q.st, (void *)&tuples, (void *)&n, (void *)&q.table, (void *)&q.pane_ts,
+                  (void *)&sz};
   return cudaLaunchKernel(k, dim3(g), dim3(kP1Threads), args, (size_t)p1_smem_bytes(p), st);
 }
 

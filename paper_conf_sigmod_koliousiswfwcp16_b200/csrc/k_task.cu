@@ -191,10 +191,34 @@ __global__ void k_task_begin(const Plan p, State *st, const unsigned char *tup, 
 // initialise the pane slots [zero_lo, zero_hi) of the ring: one CTA per slot at a
 // time, one contiguous segment (hash keys, counts, each field) after the other,
 // so no per-word division decides the identity value
-__global__ void __launch_bounds__(256) k_zero_panes(const Plan p, const State *st, uint64_t *table) {
+__global__ void __launch_bounds__(256) k_zero_panes(const Plan p, const State *st, uint64_t *table, int sgrid,
+                                                    int64_t sper) {
   const int64_t lo = st->zero_lo, hi = st->zero_hi;
   if (hi <= lo) return;
   const int64_t W = p.slot_words;
+  if (sper > 0) {
+    // the scan (k_pane_cnt) initialises every pane wholly inside one CTA's tuples;
+    // here only the panes holding a CTA boundary b_c = task_pos + min(c·per, n),
+    // c = 0..sgrid (the task's ends included): floor((b_c-1)/g) and floor(b_c/g)
+    const int64_t pos = st->task_pos, n = st->task_n;
+    for (int64_t x = blockIdx.x; x < 2 * ((int64_t)sgrid + 1); x += gridDim.x) {
+      const int64_t c = x >> 1;
+      const int64_t b = pos + (c * sper < n ? c * sper : n) - (x & 1);
+      if (b < 0) continue;
+      const int64_t pane = b / p.g;
+      if (pane < lo || pane >= hi) continue;
+      const int64_t slot = pane & (p.R - 1);
+      for (int64_t w = threadIdx.x; w < W; w += blockDim.x) table[slot * W + w] = 0;
+      if (p.pane_bm && threadIdx.x < 8) pane_bm_words(p, table)[slot * 8 + threadIdx.x] = 0;
+    }
+    return;
+  }
+  if (p.pane_bm) {                                   // presence bitmaps of the new panes
+    uint32_t *bm = pane_bm_words(p, table);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (hi - lo) * 8;
+         i += (int64_t)gridDim.x * blockDim.x)
+      bm[((lo + (i >> 3)) & (p.R - 1)) * 8 + (i & 7)] = 0;
+  }
   bool flat = p.bucket_mode || (p.key_mode != KM_HASH && !p.has_minmax);
   if (flat && (W & 1) == 0) {
     // every word's identity is 0: 16-byte stores over the ring-contiguous runs
@@ -440,8 +464,10 @@ cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s
                                  s.meta, q.carry[0], q.carry[1], q.tile_ctr, q.win_ts, q.ts_mask, round);
   return cudaGetLastError();
 }
-cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st) {
-  k_zero_panes<<<148 * 4, 256, 0, st>>>(p, q.st, q.table);
+cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st, int64_t n, int scan_grid) {
+  int g = 0;
+  const int64_t per = n > 0 && p.nagg > 0 && !p.bucket_mode ? p1_selfzero_per(p, n, scan_grid, &g) : 0;
+  k_zero_panes<<<148 * 4, 256, 0, st>>>(p, q.st, q.table, g, per);
   return cudaGetLastError();
 }
 cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st) {

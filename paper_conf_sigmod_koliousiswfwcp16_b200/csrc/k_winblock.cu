@@ -405,6 +405,13 @@ k_wb_rows(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ tab
     const int64_t j0 = J0 + t * kWrWin;
     const int jn = (int)((J1 - j0) < kWrWin ? (J1 - j0) : kWrWin);
     const int npanes = jn + K - 1;                    // panes [j0, j0 + npanes) (one-pane slides)
+    if (p.pane_bm) {                                  // the scan's presence bitmaps (8 u32 per pane)
+      const uint32_t *bm = pane_bm_words(p, table);
+      for (int i = tid; i < npanes * NBW; i += kWbThreads) {
+        const int x = i / NBW, z = i - x * NBW;
+        s_bm[x][z] = __ldcg(bm + ((j0 + x) & Rm) * 8 + z);
+      }
+    } else
     for (int x0 = warp * U; x0 < npanes; x0 += (kWbThreads / 32) * U) {
       int64_t v[U][NBW];
 #pragma unroll

@@ -67,6 +67,7 @@ int p2_blocks_per_sm(const Plan &p);
 int sel_blocks_per_sm(const Plan &p);
 int bk_scan_blocks_per_sm(const Plan &p);
 bool wb_usable(const Plan &p);
+bool wb_prepass(const Plan &p);
 bool ww_usable(const Plan &p);
 int ww_blocks_per_sm(const Plan &p);
 bool p1_is_cnt(const Plan &p);

@@ -74,7 +74,16 @@ cudaError_t launch_agg_round(const Plan &p, const QueryDev &q, const SlotDev &s,
                              int win_chunk, cudaStream_t st, cudaEvent_t *evs, int *launches, int round) {
   cudaError_t e;
   if ((e = launch_task_begin(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, st, round))) return e;
-  if ((e = launch_zero_panes(p, q, st))) return e;
+  // a count-window task without tuples (finish() after the last one) closes no
+  // window (they close by position, reading A3) and touches no pane: bookkeeping only
+  if (n == 0 && p.win_kind == WK_COUNT) {
+    if (evs) { cudaEventRecord(evs[0], st); cudaEventRecord(evs[1], st); }
+    if ((e = launch_task_end(p, q, s, st))) return e;
+    *launches = 2;
+    if (evs) cudaEventRecord(evs[2], st);
+    return cudaGetLastError();
+  }
+  if ((e = launch_zero_panes(p, q, st, p.bucket_mode ? 0 : n, p1_grid))) return e;
   *launches = 2;
   if (evs) cudaEventRecord(evs[0], st);
   if (n > 0) {
@@ -120,7 +129,7 @@ cudaError_t launch_agg_task_overlap(const Plan &p, const QueryDev &q, const Slot
                                     cudaEvent_t scan_done, cudaEvent_t *evs, int *launches) {
   cudaError_t e;
   if ((e = launch_task_begin(p, q, s, tuples, n, final_, has_wm, wm, emit_on_finish, cs))) return e;
-  if ((e = launch_zero_panes(p, q, cs))) return e;
+  if ((e = launch_zero_panes(p, q, cs, 0, p1_grid))) return e;
   *launches = 2;
   if (evs) cudaEventRecord(evs[0], cs);
   if (n > 0) {

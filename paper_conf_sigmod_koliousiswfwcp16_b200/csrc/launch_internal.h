@@ -10,7 +10,9 @@ namespace sb {
 // k_task.cu
 cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s, const void *tuples, int64_t n,
                               int final_, int has_wm, int64_t wm, int emit_on_finish, cudaStream_t st, int round = 0);
-cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st);
+cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st, int64_t n, int scan_grid);
+// k_pane_cnt initialises the pane slots wholly inside one CTA's tuples: its tuples per CTA (0: other kernels)
+int64_t p1_selfzero_per(const Plan &p, int64_t n, int grid, int *g);
 cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);
 cudaError_t launch_win_end(const QueryDev &q, const SlotDev &s, cudaStream_t st);
 cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);

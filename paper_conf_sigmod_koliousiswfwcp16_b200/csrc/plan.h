@@ -108,6 +108,9 @@ struct Plan {
   int32_t win_wide, ww_grid;       // many dense keys (256 < C <= 2048): k_win_wide (k_winwide.cu), its grid
   int32_t rounds, pad11;           // kernel rounds per task (State::round_off): time-window aggregation 2, else 1
   int32_t fx_agg, pad12;           // k_pane_agg FX3 tables: sums as three u32 limbs of x·2^32 (DIRECT / SHARED)
+  // pane presence bitmaps (k_win_block_reg plans): 8 u32 per ring slot after the
+  // table (pane_bm_words), bit k set iff the pane counted key k (flush_entry / flush_fx)
+  int32_t pane_bm, pad13;
 };
 
 // Per-query device state, updated only by kernels on the query's stream.

@@ -568,7 +568,7 @@ static saber_status alloc_query(saber_query *q) {
   CK(cudaMalloc(&q->qd.tile_ctr, 64));
   CK(cudaMalloc(&q->d_tmp, 64));
   if (p.nagg > 0) {
-    CK(cudaMalloc(&q->qd.table, (size_t)p.R * p.slot_words * 8));
+    CK(cudaMalloc(&q->qd.table, (size_t)p.R * p.slot_words * 8 + (size_t)p.R * 32));   // + pane bitmaps
     CK(cudaMalloc(&q->qd.pane_ts, (size_t)p.R * 8));
     if (p.key_mode != KM_HASH) {
       CK(cudaMalloc(&q->qd.vh_pre, (size_t)p.R * p.slot_words * 8));
@@ -625,6 +625,10 @@ static saber_status alloc_query(saber_query *q) {
   if (p.nagg > 0 && !p.win_block && ww_usable(p) && !getenv_flag("SABER_NO_WINWIDE")) p.win_wide = 1;
   CK(set_kernel_attributes(p));
   if (p.win_block) p.wb_grid = wb_blocks_per_sm(p) * q->nsm;
+  // k_win_block_reg plans count rows from the scan's pane presence bitmaps
+  if (p.win_block && wb_prepass(p) && p.win_kind == WK_COUNT && p.C % 32 == 0 && p.C <= 256 &&
+      !getenv_flag("SABER_NO_PANE_BM"))
+    p.pane_bm = 1;
   if (p.win_wide) p.ww_grid = ww_blocks_per_sm(p) * q->nsm;
   // overlap the window phase of task i with the scan of task i+1 (dense / global
   // pane tables): the ring must hold the panes of two tasks' windows at once
