@@ -502,7 +502,7 @@ k_wb_rows(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ tab
 // as soon as every thread has read them and overlap this item's presence ballots,
 // look-back and row writes.  One ballot per (window, key chunk) gives the
 // presence masks; a window's rows are its keys in order (prefix popcounts).
-template <int NF, int WPT>
+template <int NF, int CC, int WPT>
 __global__ void __launch_bounds__(kWbThreads, 3)
 k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table,
                 const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
@@ -518,10 +518,9 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t J0 = st->J0, J1 = st->J1;
   if (J1 <= J0) return;
-  const int W = (int)p.slot_words;            // C·(1+nf) words per pane slot
-  const int C = (int)p.C, K = (int)p.K;
+  // compile-time geometry: C = CC keys, ng = 256/C window groups of WPT windows, K = ng·WPT
+  constexpr int C = CC, nkc = CC / 32, ng = kWbThreads / CC, K = ng * WPT, W = CC * (1 + NF);
   const int64_t Rm = p.R - 1;
-  const int nkc = C >> 5, ng = kWbThreads / C;
   const int kc = warp % nkc, g = warp / nkc;
   const int key = kc * 32 + lane;
   const int64_t bfirst = J0 / K;
@@ -562,6 +561,11 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
   uint32_t phase = 0;
   for (int64_t t = s_t; t < nitems; ) {
     const int64_t q0 = (bfirst + t) * K;
+    const int64_t ja = q0 > J0 ? q0 : J0;
+    const int64_t jb = (q0 + K) < J1 ? (q0 + K) : J1;
+    // row offsets of the item's windows (k_wb_rows' headers), in flight during the wait
+    int64_t my_off = 0;
+    if (tid < K && q0 + tid >= ja && q0 + tid < jb) my_off = __ldcg((const long long *)&hdr[q0 + tid - J0].row_offset);
     mbar_wait(&bar, phase);
     phase ^= 1u;
     // ---- local suffixes over block b and local prefixes over block b+1
@@ -645,8 +649,6 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
       }
     }
     // ---- presence (no HAVING on the FAST plan: count > 0) of the item's windows
-    const int64_t ja = q0 > J0 ? q0 : J0;
-    const int64_t jb = (q0 + K) < J1 ? (q0 + K) : J1;
     unsigned pres = 0;
 #pragma unroll
     for (int ii = 0; ii < WPT; ++ii) {
@@ -656,17 +658,15 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
       const unsigned bal = __ballot_sync(kFull, pr);
       if (lane == 0) s_mask[i0 + ii][kc] = bal;
     }
-    if (tid < K) {                                           // row offsets from k_wb_rows' headers
-      const int64_t j = q0 + tid;
-      s_woff[tid] = (j >= ja && j < jb) ? __ldcg((const long long *)&hdr[j - J0].row_offset) : 0;
-    }
+    if (tid < K) s_woff[tid] = my_off;
     __syncthreads();
 #pragma unroll
     for (int ii = 0; ii < WPT; ++ii) {
       if (!((pres >> ii) & 1u)) continue;
       const int i = i0 + ii;
       int before = 0;
-      for (int z = 0; z < kc; ++z) before += __popc(s_mask[i][z]);
+#pragma unroll
+      for (int z = 0; z < nkc - 1; ++z) before += z < kc ? __popc(s_mask[i][z]) : 0;
       const int64_t row = s_woff[i] + before + __popc(s_mask[i][kc] & lt);
       if (row >= p.rows_cap) continue;
       if (p.nkeys) ((int32_t *)(rows + p.col_off[0]))[row] = key;
@@ -735,13 +735,18 @@ bool wb_usable(const Plan &p) {
   if (p.slot_words > kWbMaxWords) return false;
   return wb_smem(p) <= 96 * 1024;
 }
+template <int NF, int CC>
+static void *wbr_kernel(int wpt) {
+  return wpt == 4 ? (void *)k_win_block_reg<NF, CC, 4> : wpt == 8 ? (void *)k_win_block_reg<NF, CC, 8>
+                                                                  : (void *)k_win_block_reg<NF, CC, 16>;
+}
+template <int NF>
+static void *wbr_kernel_c(int c, int wpt) {
+  return c == 32 ? wbr_kernel<NF, 32>(wpt) : c == 64 ? wbr_kernel<NF, 64>(wpt) : c == 128 ? wbr_kernel<NF, 128>(wpt)
+                                                                                 : wbr_kernel<NF, 256>(wpt);
+}
 static void *wb_kernel(const Plan &p) {
-  if (const int wpt = wbr_wpt(p)) {
-    if (p.nf == 1) return wpt == 4 ? (void *)k_win_block_reg<1, 4> : wpt == 8 ? (void *)k_win_block_reg<1, 8>
-                                                                              : (void *)k_win_block_reg<1, 16>;
-    return wpt == 4 ? (void *)k_win_block_reg<2, 4> : wpt == 8 ? (void *)k_win_block_reg<2, 8>
-                                                               : (void *)k_win_block_reg<2, 16>;
-  }
+  if (const int wpt = wbr_wpt(p)) return p.nf == 1 ? wbr_kernel_c<1>((int)p.C, wpt) : wbr_kernel_c<2>((int)p.C, wpt);
   if (wb_fast(p)) return p.nf <= 1 ? (void *)k_win_block<1, true> : (void *)k_win_block<2, true>;
   return p.nf <= 1 ? (void *)k_win_block<1, false> : p.nf <= 2 ? (void *)k_win_block<2, false>
        : p.nf <= 4 ? (void *)k_win_block<4, false> : (void *)k_win_block<8, false>;
