@@ -1027,6 +1027,7 @@ static bool p1_cnt_fx(const Plan &p) {
   const int kk = p.key_mode == KM_GLOBAL ? KK_GLOBAL : KK_RADIX;
   return syn_layout(p, kk) && fx_ok(p);
 }
+bool p1_cnt_fx_plan(const Plan &p) { return p1_cnt_fx(p); }
 void *p1_kernel(const Plan &p) {
   void *k = p1_cnt(p);
   return k ? k : p1_generic(p);

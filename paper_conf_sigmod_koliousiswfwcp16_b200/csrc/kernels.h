@@ -71,6 +71,7 @@ bool wb_prepass(const Plan &p);
 bool ww_usable(const Plan &p);
 int ww_blocks_per_sm(const Plan &p);
 bool p1_is_cnt(const Plan &p);
+bool p1_cnt_fx_plan(const Plan &p);
 int wb_blocks_per_sm(const Plan &p);
 cudaError_t set_kernel_attributes(const Plan &p);
 

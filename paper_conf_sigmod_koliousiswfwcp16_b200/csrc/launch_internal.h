@@ -13,6 +13,7 @@ cudaError_t launch_task_begin(const Plan &p, const QueryDev &q, const SlotDev &s
 cudaError_t launch_zero_panes(const Plan &p, const QueryDev &q, cudaStream_t st, int64_t n, int scan_grid);
 // k_pane_cnt initialises the pane slots wholly inside one CTA's tuples: its tuples per CTA (0: other kernels)
 int64_t p1_selfzero_per(const Plan &p, int64_t n, int grid, int *g);
+bool p1_cnt_fx_plan(const Plan &p);   // the count scan runs k_pane_cnt's FX tables (12 B per entry)
 cudaError_t launch_win_scan(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);
 cudaError_t launch_win_end(const QueryDev &q, const SlotDev &s, cudaStream_t st);
 cudaError_t launch_task_end(const Plan &p, const QueryDev &q, const SlotDev &s, cudaStream_t st);

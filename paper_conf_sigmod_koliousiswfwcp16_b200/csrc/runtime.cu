@@ -410,7 +410,9 @@ static saber_status size_plan(saber_query *q) {
         !getenv_flag("SABER_NO_FX")) {
       bool sums = true;
       for (int f = 0; f < p.nf; ++f) sums &= p.field[f].kind == FK_SUM_F && p.field[f].type == T_F32;
-      const int edx = 4 + 12 * p.nf;
+      // k_pane_cnt's FX tables hold a u32 count and two u32 limbs (12 B per entry, more
+      // panes per flush window); k_pane_agg's FX3 tables three limbs per field
+      const int edx = p1_cnt_fx_plan(p) && !getenv_flag("SABER_FX16") ? 12 : 4 + 12 * p.nf;
       // SHARED: at least one pane of C entries, up to 48 KiB (3 CTAs/SM with the 32 KiB stage ring)
       const int64_t budget = p.local_mode == 1 ? direct_budget
                              : std::max<int64_t>(p.local_bytes, std::min<int64_t>(48 * 1024, (int64_t)edx * p.C));
@@ -437,6 +439,7 @@ static saber_status size_plan(saber_query *q) {
     } else {
       p.GS = 256;
       p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + 2 * p.nf) + 4));   // keys, counts, fields, compensation, occupancy list
+      if (const char *hs = std::getenv("SABER_HASH_STATE")) p.state_cap = (int)floor_pow2(std::max(64, std::atoi(hs)));
       const double A = (double)(p.K + q->win_chunk * p.L) / 2.0;
       const double B = p.key_pack == KP_RADIX ? (double)p.G / (double)p.C : 1e30;
       const double per_slot = std::max(1e-9, std::min(A, B));
