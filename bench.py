@@ -377,18 +377,22 @@ def run_join(args, rank, world):
         gen_device(lib_gen, "syn", seed, 0, n, 1, 64, b, st.cuda_stream)
         bufs.append(b)
     torch.cuda.synchronize()
-    batch = max(size, ((args.task_mb or 32) << 20) // 32)
+    # tasks of 4 MiB per stream by default: a task's pair rows (selectivity 2^-min(r, 4) of
+    # s^2 per window, 16 B each) must fit its result slot, sized from that estimate
+    batch = max(size, ((args.task_mb or 4) << 20) // 32)
     batch = min(batch, n)
     nt = (n + batch - 1) // batch
+    est_pairs = (batch // slide + 1) * size * size / 2 ** min(args.join_r, 4)
+    rbytes = int(min(8 << 30, max(64 << 20, est_pairs * 16 * 1.25)))
     j = saber.Join(js, task_bytes=batch * 32, result_mode=saber.RESULTS_DEVICE, result_slots=nt + 1,
-                   result_bytes=1 << 30)
+                   result_bytes=rbytes)
     times, pairs = [], 0
     with Clocks(0, os.path.join(ROOT, "gpurun_out", "clocks_join.csv") if os.path.isdir(os.path.join(ROOT, "gpurun_out"))
                 else "/tmp/clocks_join.csv") as clk:
         for it in range(args.warmup + args.steps):
             j.close()
             j = saber.Join(js, task_bytes=batch * 32, result_mode=saber.RESULTS_DEVICE, result_slots=nt + 1,
-                           result_bytes=1 << 30)
+                           result_bytes=rbytes)
             torch.cuda.synchronize()
             clk.timed = it >= args.warmup
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -402,10 +406,10 @@ def run_join(args, rank, world):
             torch.cuda.synchronize()
             clk.timed = False
             tot = 0
-            while True:
+            for _ in range(nt):
                 rc, r = j.poll_raw(-1)
-                if rc != 0:
-                    break
+                if rc != 0:                    # e.g. ENOMEM: the pairs did not fit a slot -- never a bench value
+                    raise saber.SaberError(rc, j.last_error())
                 tot += r.ntuples
                 j.release(r)
             if it >= args.warmup:

@@ -636,11 +636,106 @@ static void *bk_emit_kernel(const Plan &p) {
   return p.nf == 0 ? bk_emit_nf<0, C>(p.nagg) : p.nf == 1 ? bk_emit_nf<1, C>(p.nagg) : bk_emit_nf<2, C>(p.nagg);
 }
 
+
+// window assembly, pass 1 without a sliding state (one-pane slides, slabs of
+// <= 4,096 keys, K <= 64): a (window, slab)'s row count is the number of keys
+// present in any of its K pane buckets = popcount of the OR of the K pane
+// presence bitmaps.  An item (slab, chunk of windows) builds the bitmaps of its
+// panes in shared memory from the buckets' u16 key offsets (one shared atomicOr
+// per entry, each entry read once) and ORs them per window; no per-window
+// barrier, no count/uncount pair per entry (k_bkt_count: C3 G=1K 200 µs per GiB).
+constexpr int kBrSmem = 48 * 1024;
+template <int WPB>
+__global__ void __launch_bounds__(256)
+k_bkt_rows(const Plan p, const State *__restrict__ st, const unsigned long long *__restrict__ bcnt,
+           const unsigned char *__restrict__ bkt, int64_t *__restrict__ counts) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  uint32_t *bm = (uint32_t *)smem;                       // [panes][WPB]
+  constexpr int TPW = WPB < 32 ? WPB : 32;               // threads per window
+  const int S = p.S, K = (int)p.K, g = (int)p.g;
+  const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
+  if (nw <= 0) return;
+  // windows per item: what the bitmaps' shared memory holds, but about one item per CTA
+  const int wmax = kBrSmem / (4 * WPB) - K + 1;
+  const int64_t want = (nw + gridDim.x - 1) / gridDim.x;
+  const int Wt = (int)(want < 16 ? 16 : want > wmax ? wmax : want);
+  const int64_t nitems = ((nw + Wt - 1) / Wt) * S;
+  const int64_t Rm = p.R - 1;
+  const uint16_t *keys = (const uint16_t *)bkt;
+  const int tid = threadIdx.x;
+  for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
+    const int64_t chunk = item / S;
+    const int s = (int)(item % S);
+    const int64_t ja = J0 + chunk * Wt;
+    const int jn = (int)((J1 - ja) < Wt ? (J1 - ja) : Wt);
+    const int np = jn + K - 1;
+    __syncthreads();
+    for (int i = tid; i < np * WPB; i += 256) bm[i] = 0u;
+    __syncthreads();
+    // a warp per pane; 16-B loads of 8 key offsets when the bucket stride allows
+    const int warp = tid >> 5, lane = tid & 31;
+    for (int x = warp; x < np; x += 8) {
+      const int64_t b = ((ja + x) & Rm) * S + s;
+      const int n = (int)__ldg(bcnt + b);
+      const uint16_t *kp = keys + b * g;
+      uint32_t *row = bm + x * WPB;
+      if ((g & 7) == 0) {
+        const uint4 *kp4 = (const uint4 *)kp;
+#pragma unroll 4
+        for (int v = lane; v * 8 < n; v += 32) {
+          const uint4 q = __ldg(kp4 + v);
+          const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+          for (int h = 0; h < 8; ++h)
+            if (v * 8 + h < n) {
+              const uint32_t k = (w[h >> 1] >> (16 * (h & 1))) & 0xffffu;
+              atomicOr(&row[k >> 5], 1u << (k & 31));
+            }
+        }
+      } else {
+#pragma unroll 4
+        for (int e = lane; e < n; e += 32) {
+          const uint32_t k = __ldg(kp + e);
+          atomicOr(&row[k >> 5], 1u << (k & 31));
+        }
+      }
+    }
+    __syncthreads();
+    constexpr int WPP = 256 / TPW;                       // windows per pass
+    const int sub = tid % TPW;
+    for (int w0 = 0; w0 < jn; w0 += WPP) {
+      const int w = w0 + tid / TPW;
+      int c = 0;
+      if (w < jn)
+        for (int z = sub; z < WPB; z += TPW) {
+          uint32_t m = 0;
+          for (int k = 0; k < K; ++k) m |= bm[(w + k) * WPB + z];
+          c += __popc(m);
+        }
+#pragma unroll
+      for (int o = TPW / 2; o; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
+      if (sub == 0 && w < jn) counts[(ja + w - J0) * S + s] = c;
+    }
+  }
+}
+static void *bk_rows_kernel(const Plan &p) {
+  const int wpb = (1 << p.bk_shift) / 32;
+  if (p.L != 1 || p.K > 64 || wpb < 8 || wpb > 128 || kBrSmem / (4 * wpb) - p.K + 1 < 16 ||
+      std::getenv("SABER_NO_BKROWS"))
+    return nullptr;
+  return wpb == 8 ? (void *)k_bkt_rows<8> : wpb == 16 ? (void *)k_bkt_rows<16> : wpb == 32 ? (void *)k_bkt_rows<32>
+       : wpb == 64 ? (void *)k_bkt_rows<64> : (void *)k_bkt_rows<128>;
+}
+
 cudaError_t bk_set_attributes(const Plan &p) {
   cudaError_t e = cudaFuncSetAttribute(bk_scan_kernel(p), cudaFuncAttributeMaxDynamicSharedMemorySize, bk_scan_smem());
   if (e) return e;
   e = cudaFuncSetAttribute((void *)k_bkt_count, cudaFuncAttributeMaxDynamicSharedMemorySize, bk_count_smem(p));
   if (e) return e;
+  if (void *k = bk_rows_kernel(p)) {
+    e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kBrSmem);
+    if (e) return e;
+  }
   e = cudaFuncSetAttribute(bk_emit_kernel<false>(p), cudaFuncAttributeMaxDynamicSharedMemorySize, bk_emit_smem(p));
   if (e) return e;
   return cudaFuncSetAttribute(bk_emit_kernel<true>(p), cudaFuncAttributeMaxDynamicSharedMemorySize, bk_emit_smem(p));
@@ -665,7 +760,13 @@ cudaError_t launch_bucket_scan(const Plan &p, const QueryDev &q, const void *tup
 
 cudaError_t launch_bucket_windows(const Plan &p, const QueryDev &q, const SlotDev &s, int nsm, cudaStream_t st) {
   const unsigned long long *bc = (const unsigned long long *)q.table;
-  k_bkt_count<<<nsm * 3, 256, bk_count_smem(p), st>>>(p, q.st, bc, q.bkt, s.counts);
+  if (void *k = bk_rows_kernel(p)) {
+    void *ra[] = {(void *)&p, (void *)&q.st, (void *)&bc, (void *)&q.bkt, (void *)&s.counts};
+    cudaError_t e = cudaLaunchKernel(k, dim3(nsm * 4), dim3(256), ra, (size_t)kBrSmem, st);
+    if (e) return e;
+  } else {
+    k_bkt_count<<<nsm * 3, 256, bk_count_smem(p), st>>>(p, q.st, bc, q.bkt, s.counts);
+  }
   cudaError_t e = launch_win_scan(p, q, s, st);
   if (e) return e;
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&bc, (void *)&q.bkt, (void *)&s.counts, (void *)&s.rows};

@@ -404,6 +404,23 @@ static saber_status size_plan(saber_query *q) {
         fk &= p.fast_path != 0;
       p.fast_keys = (fk || p.fast_path) ? 1 : 0;
     }
+    // k_pane_cnt's FX tables (count-window dense plans, f32 sums as u32 limbs): one
+    // CTA-wide table of 6 KiB instead of per-warp copies.  The limbs take
+    // fire-and-forget REDs, which never retry under cross-warp contention, so the copies
+    // bought nothing but 8x the flush work; one table holds 8 panes of 64 keys, so a
+    // flush comes every 8 panes instead of every 3 (C3 G=64 scan 0.788 -> 0.705 ms per
+    // 4 GiB task; 24 KiB tables cost the 4th CTA per SM: 0.754).  SABER_CNT_SHARED_KB=0
+    // keeps the per-warp tables.
+    if (p.win_kind == WK_COUNT && p.key_mode != KM_HASH && p.local_mode == 1 && p1_cnt_fx_plan(p)) {
+      const char *ckb = std::getenv("SABER_CNT_SHARED_KB");
+      const int kb = ckb ? std::atoi(ckb) : 6;
+      if (kb > 0) {
+        p.local_mode = 3;
+        p.local_pl = (int)std::max<int64_t>(1, std::min<int64_t>(1024, ((int64_t)kb * 1024) / (ed * p.C)));
+        p.local_entries = p.local_pl * (int)p.C;
+        p.local_bytes = ((p.local_entries * ed) + 15) & ~15;
+      }
+    }
     // k_pane_agg FX3 tables (atomic DIRECT / SHARED tables of f32 sums): three u32
     // limbs per sum instead of one fp64 word -- re-size the pane window for them
     if (p.fast_keys && p.nf >= 1 && p.nf <= 2 && (p.local_mode == 1 || p.local_mode == 3) &&

@@ -584,3 +584,32 @@ def test_select_n_predicates(saber, oracle_lib, npred):
     spec, g = workloads.c2(sel=0.3, npred=npred)
     data = gen.generate("syn", 1 << 18, g["seed"], rate=1)
     check(saber, oracle_lib, spec, data, task_bytes=(1 << 20) + 32 * 13)
+
+
+# k_wb_rows + k_win_block_reg (FAST plans, one-pane slides, 32..256 dense keys):
+# every template instance the planner can pick (C, K = (256/C)·{4, 8, 16}), two
+# float sum fields (CM), a time window, ragged tasks whose windows span tasks
+@pytest.mark.parametrize("case", ["c32_k32", "c64_k16", "c64_k64", "c128_k16", "c256_k8", "cm_nf2", "time_c64_k32"])
+def test_win_block_reg(saber, oracle_lib, case):
+    if case == "cm_nf2":
+        spec, _ = workloads.c4(rate=64)
+        spec["window"] = workloads.count_window(32 * 48, 48)
+        spec["aggs"] = [("avg", "cpu"), ("sum", "ram"), ("count", None)]
+        spec["group_by"] = [("category", 1, 64)]
+        data = gen.generate("cm", 200000, 41, rate=64, groups=64)
+        tb = 64 * 7919
+    elif case == "time_c64_k32":
+        spec, _ = workloads.c3(groups=64)
+        spec["window"] = workloads.time_window(32, 1)
+        data = gen.generate("syn", 300000, 42, rate=100, groups=64)
+        tb = 32 * 12347
+    else:
+        c, k = (int(x[1:]) for x in case.split("_"))
+        l = {32: 16, 64: 8, 128: 12, 256: 40}[c] if k != 64 else 8
+        spec, _ = workloads.c3(groups=c)
+        spec["window"] = workloads.count_window(k * l, l)
+        spec["aggs"] = [("avg", "a1"), ("count", None), ("sum", "a1")]
+        data = gen.generate("syn", 250000, 40 + c + k, groups=c)
+        tb = 32 * 9973
+    got, exp = check(saber, oracle_lib, spec, data, task_bytes=tb)
+    assert len(exp["win_id"]) > 100
