@@ -201,6 +201,86 @@ k_join_pairs_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, int64_t *__restri
   if (!EMIT && act) counts[w * p.s + a_loc] = cnt;
 }
 
+
+// Emission of the fast path with coalesced rows: a warp per row a of W1, lanes over
+// the b's of the staged W2 chunk.  Row a's pairs are contiguous in the output, in b
+// order, so a ballot over 32 consecutive b's places a lane's row at a's running
+// offset + the popcount of the lower lanes: the warp writes 32 consecutive rows per
+// step (the thread-per-row pass scattered every store over 32 rows far apart).  The
+// θ columns and the projected words of the chunk are staged column-wise; lane l
+// keeps the running offset of the warp's l-th row.  Same rows, same order as the
+// thread-per-row kernel (pairs in (a, b) order, reading A26).
+constexpr int kJoinEmitWords = 8;           // projected words of S2 staged per chunk
+__global__ void __launch_bounds__(kJoinThreads)
+k_join_emit_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, const int64_t *__restrict__ offs,
+                unsigned char *__restrict__ rows) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  int32_t *col = (int32_t *)smem;                              // [npred][kJoinChunk]
+  uint32_t *pj = (uint32_t *)(col + kJoinFastTerms * kJoinChunk);   // [nw2][kJoinChunk]
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t w = blockIdx.x;
+  const int64_t base = (J0 + w) * p.l;
+  const int a0 = blockIdx.y * kJoinThreads;
+  const int np = p.npred, nw1 = p.nw1, nw2 = p.nw2;
+  const int orow = 4 * (nw1 + nw2);
+  const unsigned lt = (1u << lane) - 1u;
+  uint32_t om[kJoinFastTerms];
+#pragma unroll
+  for (int k = 0; k < kJoinFastTerms; ++k) {
+    const int op = k < np ? p.pred[k].op : OP_EQ;
+    om[k] = op == OP_LT ? 1u : op == OP_LE ? 3u : op == OP_GT ? 4u : op == OP_GE ? 6u : op == OP_EQ ? 2u : 5u;
+  }
+  // lane l: running output row of a = a0 + warp + 8·l
+  const int al = a0 + warp + 8 * lane;
+  int64_t run = (lane < kJoinThreads / 8 && al < p.s) ? offs[w * p.s + al] : 0;
+  for (int64_t c0 = 0; c0 < p.s; c0 += kJoinChunk) {
+    const int nb = (int)((p.s - c0) < kJoinChunk ? (p.s - c0) : kJoinChunk);
+    __syncthreads();
+    for (int x = tid; x < nb; x += kJoinThreads) {
+      const unsigned char *tb = jtuple(v2, base + c0 + x);
+#pragma unroll
+      for (int k = 0; k < kJoinFastTerms; ++k)
+        if (k < np) col[k * kJoinChunk + x] = *(const int32_t *)(tb + 4 * p.pred[k].w2);
+#pragma unroll
+      for (int c = 0; c < kJoinEmitWords; ++c)
+        if (c < nw2) pj[c * kJoinChunk + x] = ((const uint32_t *)tb)[p.pw2[c]];
+    }
+    __syncthreads();
+    for (int i = 0; i < kJoinThreads / 8; ++i) {
+      const int a = a0 + warp + 8 * i;
+      if (a >= p.s) break;                                     // warp-uniform
+      const unsigned char *ta = jtuple(v1, base + a);
+      int32_t av[kJoinFastTerms];
+#pragma unroll
+      for (int k = 0; k < kJoinFastTerms; ++k) av[k] = k < np ? *(const int32_t *)(ta + 4 * p.pred[k].w1) : 0;
+      int64_t out = (int64_t)__shfl_sync(kFull, (unsigned long long)run, i);
+      for (int b0 = 0; b0 < nb; b0 += 32) {
+        const int b = b0 + lane;
+        uint32_t ok = b < nb ? 1u : 0u;
+#pragma unroll
+        for (int k = 0; k < kJoinFastTerms; ++k)
+          if (k < np) {
+            const int32_t y = col[k * kJoinChunk + (b < nb ? b : 0)];
+            ok &= (om[k] >> (av[k] < y ? 0 : (av[k] == y ? 1 : 2))) & 1u;
+          }
+        const unsigned bal = __ballot_sync(kFull, ok);
+        if (ok) {
+          const int64_t r = out + __popc(bal & lt);
+          if (r < p.rows_cap) {
+            uint32_t *dst = (uint32_t *)(rows + r * orow);
+            for (int c = 0; c < nw1; ++c) dst[c] = ((const uint32_t *)ta)[p.pw1[c]];
+#pragma unroll
+            for (int c = 0; c < kJoinEmitWords; ++c)
+              if (c < nw2) dst[nw1 + c] = pj[c * kJoinChunk + b];
+          }
+        }
+        out += __popc(bal);
+      }
+      if (lane == i) run = out;
+    }
+  }
+}
+
 // exclusive scan of n counts in place (tiles by ticket, decoupled look-back); the
 // total goes to *total
 __global__ void __launch_bounds__(kJoinThreads)
@@ -347,7 +427,10 @@ static saber_status join_task(saber_join *j, const unsigned char *d1, const unsi
     k_join_scan<<<148 * 4, kJoinThreads, 0, j->cs>>>(j->counts, nwin * p.s, j->status, j->ticket, j->epoch,
                                                      s.d_total);
     JCK(cudaGetLastError());
-    if (fast) k_join_pairs_i32<true><<<grid, kJoinThreads, fsmem, j->cs>>>(p, v1, v2, j->J0, nullptr, j->counts, s.rows);
+    if (fast && p.nw2 <= kJoinEmitWords && !std::getenv("SABER_JOIN_THREAD_EMIT"))
+      k_join_emit_i32<<<grid, kJoinThreads, fsmem + (size_t)kJoinEmitWords * kJoinChunk * 4, j->cs>>>(
+          p, v1, v2, j->J0, j->counts, s.rows);
+    else if (fast) k_join_pairs_i32<true><<<grid, kJoinThreads, fsmem, j->cs>>>(p, v1, v2, j->J0, nullptr, j->counts, s.rows);
     else k_join_pairs<true><<<grid, kJoinThreads, smem, j->cs>>>(p, v1, v2, j->J0, nullptr, j->counts, s.rows);
     JCK(cudaGetLastError());
     k_join_hdr<<<148, 256, 0, j->cs>>>(p, v1, j->J0, nwin, j->counts, s.d_total, (WinHdr *)s.hdr);
@@ -481,6 +564,8 @@ saber_status saber_join_create(const saber_schema *s1, const saber_schema *s2, c
     const size_t smem = (size_t)kJoinThreads * p.tb1 + (size_t)kJoinChunk * p.tb2;
     JCK(cudaFuncSetAttribute((void *)k_join_pairs<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     JCK(cudaFuncSetAttribute((void *)k_join_pairs<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    JCK(cudaFuncSetAttribute((void *)k_join_emit_i32, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)((kJoinFastTerms + kJoinEmitWords) * kJoinChunk * 4)));
     return SABER_OK;
   };
   if (saber_status st = setup()) {
