@@ -383,7 +383,8 @@ constexpr int kWrWin = 512;          // windows per ticket (two per thread)
 template <int NBW>
 __global__ void __launch_bounds__(kWbThreads)
 k_wb_rows(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table, const int64_t *__restrict__ pane_ts,
-          WinHdr *__restrict__ hdr, uint64_t *__restrict__ status, int *__restrict__ ticket) {
+          WinHdr *__restrict__ hdr, uint64_t *__restrict__ status, int *__restrict__ ticket,
+          int64_t *__restrict__ woffs, int nz) {
   hdr += st->hdr_base;
   __shared__ unsigned s_bm[kWrWin + 64][NBW];   // pane presence bitmaps (K <= 64)
   __shared__ int s_t;
@@ -431,15 +432,19 @@ k_wb_rows(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ tab
     }
     __syncthreads();
     int n0 = 0, n1 = 0;
+    int pc0[NBW], pc1[NBW];                             // rows per 32-key word (key slices)
     const int w0 = 2 * tid;
 #pragma unroll
     for (int z = 0; z < NBW; ++z) {
+      pc0[z] = pc1[z] = 0;
       if (w0 < jn) {
         unsigned m = 0;
         for (int k = 1; k < K; ++k) m |= s_bm[w0 + k][z];          // panes shared by both windows
-        n0 += __popc(m | s_bm[w0][z]);
-        if (w0 + 1 < jn) n1 += __popc(m | s_bm[w0 + K][z]);
+        pc0[z] = __popc(m | s_bm[w0][z]);
+        if (w0 + 1 < jn) pc1[z] = __popc(m | s_bm[w0 + K][z]);
       }
+      n0 += pc0[z];
+      n1 += pc1[z];
     }
     const int n = n0 + n1;
     // block exclusive scan of the row counts
@@ -482,6 +487,15 @@ k_wb_rows(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ tab
       h.nrows = e ? n1 : n0;
       h.flags = 0;
       hdr[j - J0] = h;
+      if (nz > 1) {                                     // first row of every key slice of the window
+        int64_t r = h.row_offset;
+        const int wps = NBW / nz;                       // 32-key words per slice
+#pragma unroll
+        for (int z = 0; z < NBW; ++z) {
+          if (z % wps == 0) woffs[(j - J0) * nz + z / wps] = r;
+          r += e ? pc1[z] : pc0[z];
+        }
+      }
     }
     __syncthreads();
   }
@@ -506,7 +520,8 @@ template <int NF, int CC, int WPT>
 __global__ void __launch_bounds__(kWbThreads, 3)
 k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table,
                 const int64_t *__restrict__ pane_ts, WinHdr *__restrict__ hdr, unsigned char *__restrict__ rows,
-                uint64_t *__restrict__ status, int *__restrict__ ticket, int NB) {
+                uint64_t *__restrict__ status, int *__restrict__ ticket, int NB,
+                const int64_t *__restrict__ woffs) {
   (void)NB; (void)status; (void)pane_ts;
   ticket += 1;                                // [0] is k_wb_rows' ticket
   hdr += st->hdr_base;
@@ -519,21 +534,32 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
   const int64_t J0 = st->J0, J1 = st->J1;
   if (J1 <= J0) return;
   // compile-time geometry: C = CC keys, ng = 256/C window groups of WPT windows, K = ng·WPT
+  // (key slices: C = p.C > CC keys are processed CC at a time, NZ items per block)
   constexpr int C = CC, nkc = CC / 32, ng = kWbThreads / CC, K = ng * WPT, W = CC * (1 + NF);
+  const int NZ = (int)(p.C / CC);
   const int64_t Rm = p.R - 1;
   const int kc = warp % nkc, g = warp / nkc;
-  const int key = kc * 32 + lane;
   const int64_t bfirst = J0 / K;
-  const int64_t nitems = (J1 - 1) / K - bfirst + 1;
+  const int64_t nitems = ((J1 - 1) / K - bfirst + 1) * NZ;
   const int NP = 2 * K - 1;                   // staged panes per item
   uint64_t *raw = (uint64_t *)smem;           // [NP][W]
   uint64_t *tot = raw + (size_t)NP * W;       // [2][ng][W]: group totals of blocks b and b+1
   const int64_t qhi = J1 - 1 + K - 1;         // last pane read by the task's windows
   const unsigned lt = (1u << lane) - 1u;
   auto stage = [&](int64_t t) {               // thread 0: bulk copies of item t's panes
-    const int64_t q0 = (bfirst + t) * K;
+    const int64_t q0 = (bfirst + t / NZ) * K;
     const int64_t sa = q0 > J0 ? q0 : J0;
     const int64_t se = (q0 + NP) < (qhi + 1) ? (q0 + NP) : (qhi + 1);
+    if (NZ > 1) {                             // slice z: CC words of the count and of each field
+      const int z = (int)(t % NZ);
+      mbar_expect_tx(&bar, (uint32_t)((se > sa ? se - sa : 0) * W * 8));
+      for (int64_t q = sa; q < se; ++q)
+#pragma unroll
+        for (int f = 0; f <= NF; ++f)
+          bulk_g2s(raw + (q - q0) * W + f * CC, table + (q & Rm) * p.slot_words + f * p.C + z * CC,
+                   (uint32_t)(CC * 8), &bar);
+      return;
+    }
     uint32_t bytes = 0;
     for (int64_t q = sa; q < se;) {
       const int64_t run = ((q | Rm) + 1 - q) < (se - q) ? ((q | Rm) + 1 - q) : (se - q);
@@ -560,12 +586,17 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
   __syncthreads();
   uint32_t phase = 0;
   for (int64_t t = s_t; t < nitems; ) {
-    const int64_t q0 = (bfirst + t) * K;
+    const int64_t q0 = (bfirst + t / NZ) * K;
+    const int z = (int)(t % NZ);
+    const int key = z * CC + kc * 32 + lane;
     const int64_t ja = q0 > J0 ? q0 : J0;
     const int64_t jb = (q0 + K) < J1 ? (q0 + K) : J1;
-    // row offsets of the item's windows (k_wb_rows' headers), in flight during the wait
+    // row offsets of the item's windows (k_wb_rows: headers, or per (window, slice)), in
+    // flight during the wait
     int64_t my_off = 0;
-    if (tid < K && q0 + tid >= ja && q0 + tid < jb) my_off = __ldcg((const long long *)&hdr[q0 + tid - J0].row_offset);
+    if (tid < K && q0 + tid >= ja && q0 + tid < jb)
+      my_off = NZ > 1 ? __ldcg((const long long *)&woffs[(q0 + tid - J0) * NZ + z])
+                      : __ldcg((const long long *)&hdr[q0 + tid - J0].row_offset);
     mbar_wait(&bar, phase);
     phase ^= 1u;
     // ---- local suffixes over block b and local prefixes over block b+1
@@ -579,7 +610,7 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
       for (int x = 0; x < NF; ++x) af[x] = 0.0;
 #pragma unroll
       for (int ii = WPT - 1; ii >= 0; --ii) {
-        const uint64_t *r = raw + (i0 + ii) * W + key;
+        const uint64_t *r = raw + (i0 + ii) * W + (kc * 32 + lane);
         ac += (int64_t)r[0];
         c[ii] = ac;
 #pragma unroll
@@ -588,7 +619,7 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
           f[x][ii] = af[x];
         }
       }
-      uint64_t *tb = tot + g * W + key;
+      uint64_t *tb = tot + g * W + (kc * 32 + lane);
       tb[0] = (uint64_t)ac;
 #pragma unroll
       for (int x = 0; x < NF; ++x) tb[(1 + x) * C] = (uint64_t)__double_as_longlong(af[x]);
@@ -605,13 +636,13 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
         for (int x = 0; x < NF; ++x) f[x][ii] += af[x];
         const int qi = K + i0 + ii;
         if (qi < NP) {
-          const uint64_t *r = raw + qi * W + key;
+          const uint64_t *r = raw + qi * W + (kc * 32 + lane);
           ac += (int64_t)r[0];
 #pragma unroll
           for (int x = 0; x < NF; ++x) af[x] += __longlong_as_double((long long)r[(1 + x) * C]);
         }
       }
-      uint64_t *tb = tot + (ng + g) * W + key;
+      uint64_t *tb = tot + (ng + g) * W + (kc * 32 + lane);
       tb[0] = (uint64_t)ac;
 #pragma unroll
       for (int x = 0; x < NF; ++x) tb[(1 + x) * C] = (uint64_t)__double_as_longlong(af[x]);
@@ -630,13 +661,13 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
 #pragma unroll
       for (int x = 0; x < NF; ++x) tf[x] = 0.0;
       for (int h = g + 1; h < ng; ++h) {
-        const uint64_t *tb = tot + h * W + key;
+        const uint64_t *tb = tot + h * W + (kc * 32 + lane);
         tc += (int64_t)tb[0];
 #pragma unroll
         for (int x = 0; x < NF; ++x) tf[x] += __longlong_as_double((long long)tb[(1 + x) * C]);
       }
       for (int h = 0; h < g; ++h) {
-        const uint64_t *tb = tot + (ng + h) * W + key;
+        const uint64_t *tb = tot + (ng + h) * W + (kc * 32 + lane);
         tc += (int64_t)tb[0];
 #pragma unroll
         for (int x = 0; x < NF; ++x) tf[x] += __longlong_as_double((long long)tb[(1 + x) * C]);
@@ -705,18 +736,27 @@ static bool wb_fast(const Plan &p) {
 }
 // register variant: FAST plan, one-pane slides, 32..256 dense keys (power of two),
 // fp64 sums only, K a multiple of the 256/C window groups with <= 16 windows per thread
-static int wbr_wpt(const Plan &p) {
+// keys per item: all C, or slices of 64 (C = 128 / 256 when the whole table's
+// windows would need more than 16 per thread, C3 G=256: K = 32)
+static int64_t wbr_cc(const Plan &p) {
   if (!wb_fast(p) || p.L != 1 || p.key_mode == KM_HASH || p.C < 32 || p.C > 256 || (p.C & (p.C - 1))) return 0;
   if (p.slot_words != p.C * (1 + p.nf) || p.nf < 1 || std::getenv("SABER_NO_WBREG")) return 0;
   for (int f = 0; f < p.nf; ++f)
     if (p.field[f].kind != FK_SUM_F) return 0;
-  const int64_t ng = kWbThreads / p.C;
-  if (p.K > 64 || p.K % ng) return 0;
-  const int64_t wpt = p.K / ng;
-  return (wpt == 4 || wpt == 8 || wpt == 16) ? (int)wpt : 0;
+  if (p.K > 64) return 0;
+  auto ok = [&](int64_t cc) { const int64_t ng = kWbThreads / cc, w = p.K / ng;
+                              return p.K % ng == 0 && (w == 4 || w == 8 || w == 16); };
+  if (ok(p.C)) return p.C;
+  if (p.C > 64 && ok(64) && !std::getenv("SABER_NO_WBSLICE")) return 64;
+  return 0;
+}
+static int wbr_wpt(const Plan &p) {
+  const int64_t cc = wbr_cc(p);
+  return cc ? (int)(p.K / (kWbThreads / cc)) : 0;
 }
 static int wbr_smem(const Plan &p) {
-  return (int)(((2 * p.K - 1) + 2 * (kWbThreads / p.C)) * p.slot_words * 8);
+  const int64_t cc = wbr_cc(p);
+  return (int)(((2 * p.K - 1) + 2 * (kWbThreads / cc)) * cc * (1 + p.nf) * 8);
 }
 int wb_smem(const Plan &p) {
   if (wbr_wpt(p)) return wbr_smem(p);
@@ -746,7 +786,10 @@ static void *wbr_kernel_c(int c, int wpt) {
                                                                                  : wbr_kernel<NF, 256>(wpt);
 }
 static void *wb_kernel(const Plan &p) {
-  if (const int wpt = wbr_wpt(p)) return p.nf == 1 ? wbr_kernel_c<1>((int)p.C, wpt) : wbr_kernel_c<2>((int)p.C, wpt);
+  if (const int wpt = wbr_wpt(p)) {
+    const int cc = (int)wbr_cc(p);
+    return p.nf == 1 ? wbr_kernel_c<1>(cc, wpt) : wbr_kernel_c<2>(cc, wpt);
+  }
   if (wb_fast(p)) return p.nf <= 1 ? (void *)k_win_block<1, true> : (void *)k_win_block<2, true>;
   return p.nf <= 1 ? (void *)k_win_block<1, false> : p.nf <= 2 ? (void *)k_win_block<2, false>
        : p.nf <= 4 ? (void *)k_win_block<4, false> : (void *)k_win_block<8, false>;
@@ -762,13 +805,15 @@ int wb_blocks_per_sm(const Plan &p) {
 bool wb_prepass(const Plan &p) { return wbr_wpt(p) != 0; }
 cudaError_t launch_windows_block(const Plan &p, const QueryDev &q, const SlotDev &s, int grid, cudaStream_t st) {
   const int nb = wb_nb(p);
+  int64_t *woffs = s.counts;
   if (wbr_wpt(p)) {     // row counts, offsets and headers first (k_wb_rows), then the values
-    void (*k)(const Plan, State *, const uint64_t *, const int64_t *, WinHdr *, uint64_t *, int *) =
+    void (*k)(const Plan, State *, const uint64_t *, const int64_t *, WinHdr *, uint64_t *, int *, int64_t *, int) =
         p.C <= 32 ? k_wb_rows<1> : p.C <= 64 ? k_wb_rows<2> : p.C <= 128 ? k_wb_rows<4> : k_wb_rows<8>;
-    k<<<grid, kWbThreads, 0, st>>>(p, q.st, q.table, q.pane_ts, (WinHdr *)s.hdr, q.tile_status, q.tile_ctr);
+    const int nz = (int)(p.C / wbr_cc(p));
+    k<<<grid, kWbThreads, 0, st>>>(p, q.st, q.table, q.pane_ts, (WinHdr *)s.hdr, q.tile_status, q.tile_ctr, woffs, nz);
   }
   void *args[] = {(void *)&p, (void *)&q.st, (void *)&q.table, (void *)&q.pane_ts, (void *)&s.hdr, (void *)&s.rows,
-                  (void *)&q.tile_status, (void *)&q.tile_ctr, (void *)&nb};
+                  (void *)&q.tile_status, (void *)&q.tile_ctr, (void *)&nb, (void *)&woffs};
   return cudaLaunchKernel(wb_kernel(p), dim3(grid), dim3(kWbThreads), args, (size_t)wb_smem(p), st);
 }
 

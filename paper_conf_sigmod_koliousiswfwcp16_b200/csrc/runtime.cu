@@ -639,7 +639,10 @@ static saber_status alloc_query(saber_query *q) {
   for (auto &s : q->slots) {
     CK(cudaMalloc(&s.dev.rows, rows_bytes ? rows_bytes : 16));
     CK(cudaMalloc(&s.dev.hdr, (size_t)p.win_cap * sizeof(saber_win_hdr)));
-    CK(cudaMalloc(&s.dev.counts, (size_t)p.win_cap * std::max(1, p.S) * 8));
+    // + per (window, 64-key slice) row offsets of k_win_block_reg (dense C <= 256; win_block
+    // is decided after the slots exist)
+    const int64_t wslices = (p.key_mode != KM_HASH && p.C <= 256) ? std::max<int64_t>(1, p.C / 64) : 1;
+    CK(cudaMalloc(&s.dev.counts, (size_t)p.win_cap * std::max<int64_t>({1, p.S, wslices}) * 8));
     CK(cudaMalloc(&s.dev.meta, sizeof(SlotMeta)));
     CK(cudaMalloc(&s.dev.wst, sizeof(State)));
     CK(cudaMalloc(&s.dev.ticket, 64));

@@ -587,9 +587,11 @@ def test_select_n_predicates(saber, oracle_lib, npred):
 
 
 # k_wb_rows + k_win_block_reg (FAST plans, one-pane slides, 32..256 dense keys):
-# every template instance the planner can pick (C, K = (256/C)·{4, 8, 16}), two
+# every template instance the planner can pick (C, K = (256/C)·{4, 8, 16}; key slices of 64
+# for C = 256, K = 32 and C = 128, K = 64), two
 # float sum fields (CM), a time window, ragged tasks whose windows span tasks
-@pytest.mark.parametrize("case", ["c32_k32", "c64_k16", "c64_k64", "c128_k16", "c256_k8", "cm_nf2", "time_c64_k32"])
+@pytest.mark.parametrize("case", ["c32_k32", "c64_k16", "c64_k64", "c128_k16", "c256_k8", "c256_k32", "c128_k64",
+                                  "cm_nf2", "time_c64_k32"])
 def test_win_block_reg(saber, oracle_lib, case):
     if case == "cm_nf2":
         spec, _ = workloads.c4(rate=64)
