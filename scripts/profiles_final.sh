@@ -23,8 +23,11 @@ full k_pane_cnt_C3_G64 k_pane_cnt 2 --config C3 --groups 64
 full k_win_block_reg_C3_G64 k_win_block_reg 3 --config C3 --groups 64
 full k_wb_rows_C3_G64 k_wb_rows 3 --config C3 --groups 64
 full k_pane_agg_C5a k_pane_agg 2 --config C5a
-full k_select_C2 k_select 2 --config C2
+full k_select_C2 k_select 0 --config C2
+full k_win_block_reg_C3_G256 k_win_block_reg 3 --config C3 --groups 256
+full k_bkt_rows_C3_G1024 k_bkt_rows 2 --config C3 --groups 1024
 bash scripts/bench_all.sh $O/bench_all_configs.jsonl > $O/bench_all_configs.txt 2>&1
 for c in C1 C2 C4 C5a C5b SG1; do timeout 600 python bench.py --no-cpu --steps 3 --warmup 3 --config $c 2>>$O/e2e.err | tail -1; done > $O/bench_e2e_configs.jsonl
 ./build_var/ubr > $O/ubench_read_bw.txt 2>&1
+mkdir -p gpurun_out/sweeps; bash scripts/sweeps.sh > gpurun_out/sweeps/tables.txt 2>&1
 ls $O
