@@ -94,7 +94,8 @@ class Stats(C.Structure):
                 ("overlap", C.c_int32), ("reserved", C.c_int32), ("task_tuples", C.c_int64)]
 
 SCAN_KERNELS = ["k_select", "k_pane_agg", "k_pane_cnt", "k_pane_bucket"]
-WINDOW_KERNELS = ["none", "k_vh_build+k_win_packed/k_win_fused", "k_win_block", "k_bkt_count+k_win_scan+k_bkt_emit",
+WINDOW_KERNELS = ["none", "k_vh_build+k_win_packed/k_win_fused", "k_win_block (or k_wb_rows+k_win_block_reg)",
+                  "k_bkt_rows/k_bkt_count+k_win_scan+k_bkt_emit",
                   "k_win_hash", "k_win_slab", "k_vh_build+k_win_wide"]
 
 
