@@ -550,16 +550,18 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
     const int64_t q0 = (bfirst + t / NZ) * K;
     const int64_t sa = q0 > J0 ? q0 : J0;
     const int64_t se = (q0 + NP) < (qhi + 1) ? (q0 + NP) : (qhi + 1);
-    if (NZ > 1) {                             // slice z: CC words of the count and of each field
-      const int z = (int)(t % NZ);
-      mbar_expect_tx(&bar, (uint32_t)((se > sa ? se - sa : 0) * W * 8));
-      for (int64_t q = sa; q < se; ++q)
+    if (NZ > 1) {                             // slice z: CC words of the count and of each field,
+      const int z = (int)(t % NZ);            // the (NF+1)·panes copies issued by the 32 lanes of warp 0
+      if (lane == 0) mbar_expect_tx(&bar, (uint32_t)((se > sa ? se - sa : 0) * W * 8));
+      __syncwarp();
+      for (int64_t q = sa + lane; q < se; q += 32)
 #pragma unroll
         for (int f = 0; f <= NF; ++f)
           bulk_g2s(raw + (q - q0) * W + f * CC, table + (q & Rm) * p.slot_words + f * p.C + z * CC,
                    (uint32_t)(CC * 8), &bar);
       return;
     }
+    if (lane) return;
     uint32_t bytes = 0;
     for (int64_t q = sa; q < se;) {
       const int64_t run = ((q | Rm) + 1 - q) < (se - q) ? ((q | Rm) + 1 - q) : (se - q);
@@ -581,9 +583,9 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
     mbar_init(&bar, 1);
     fence_mbar_init();
     s_t = atomicAdd(ticket, 1);
-    if (s_t < nitems) stage(s_t);
   }
   __syncthreads();
+  if (warp == 0 && s_t < nitems) stage(s_t);           // warp 0 issues the bulk copies
   uint32_t phase = 0;
   for (int64_t t = s_t; t < nitems; ) {
     const int64_t q0 = (bfirst + t / NZ) * K;
@@ -649,10 +651,12 @@ k_win_block_reg(const Plan p, State *__restrict__ st, const uint64_t *__restrict
     }
     __syncthreads();
     // every thread has read its staged panes: the next ticket's copies go now
-    if (tid == 0) {
+    if (warp == 0) {
       fence_proxy_async_smem();
-      s_next = atomicAdd(ticket, 1);
-      if (s_next < nitems) stage(s_next);
+      int nx = 0;
+      if (lane == 0) s_next = nx = atomicAdd(ticket, 1);
+      nx = __shfl_sync(kFull, nx, 0);
+      if (nx < nitems) stage(nx);
     }
     // ---- window values: S[i] = local suffix ⊕ later groups of b, P[i] = earlier groups of b+1 ⊕ local prefix
     {
