@@ -230,9 +230,20 @@ k_join_emit_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, const int64_t *__r
     const int op = k < np ? p.pred[k].op : OP_EQ;
     om[k] = op == OP_LT ? 1u : op == OP_LE ? 3u : op == OP_GT ? 4u : op == OP_GE ? 6u : op == OP_EQ ? 2u : 5u;
   }
-  // lane l: running output row of a = a0 + warp + 8·l
+  // lane l: running output row, θ operands and projected words of a = a0 + warp + 8·l (held in
+  // registers and broadcast by shuffles: no dependent global load per row)
   const int al = a0 + warp + 8 * lane;
-  int64_t run = (lane < kJoinThreads / 8 && al < p.s) ? offs[w * p.s + al] : 0;
+  const bool lv = lane < kJoinThreads / 8 && al < p.s;
+  int64_t run = lv ? offs[w * p.s + al] : 0;
+  int32_t avl[kJoinFastTerms];
+  uint32_t pwl[kJoinEmitWords];
+  {
+    const unsigned char *tal = lv ? jtuple(v1, base + al) : nullptr;
+#pragma unroll
+    for (int k = 0; k < kJoinFastTerms; ++k) avl[k] = (lv && k < np) ? *(const int32_t *)(tal + 4 * p.pred[k].w1) : 0;
+#pragma unroll
+    for (int c = 0; c < kJoinEmitWords; ++c) pwl[c] = (lv && c < nw1) ? ((const uint32_t *)tal)[p.pw1[c]] : 0u;
+  }
   for (int64_t c0 = 0; c0 < p.s; c0 += kJoinChunk) {
     const int nb = (int)((p.s - c0) < kJoinChunk ? (p.s - c0) : kJoinChunk);
     __syncthreads();
@@ -249,10 +260,12 @@ k_join_emit_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, const int64_t *__r
     for (int i = 0; i < kJoinThreads / 8; ++i) {
       const int a = a0 + warp + 8 * i;
       if (a >= p.s) break;                                     // warp-uniform
-      const unsigned char *ta = jtuple(v1, base + a);
       int32_t av[kJoinFastTerms];
 #pragma unroll
-      for (int k = 0; k < kJoinFastTerms; ++k) av[k] = k < np ? *(const int32_t *)(ta + 4 * p.pred[k].w1) : 0;
+      for (int k = 0; k < kJoinFastTerms; ++k) av[k] = __shfl_sync(kFull, avl[k], i);
+      uint32_t pa[kJoinEmitWords];
+#pragma unroll
+      for (int c = 0; c < kJoinEmitWords; ++c) pa[c] = __shfl_sync(kFull, pwl[c], i);
       int64_t out = (int64_t)__shfl_sync(kFull, (unsigned long long)run, i);
       for (int b0 = 0; b0 < nb; b0 += 32) {
         const int b = b0 + lane;
@@ -268,7 +281,9 @@ k_join_emit_i32(const JoinPlan p, JIn v1, JIn v2, int64_t J0, const int64_t *__r
           const int64_t r = out + __popc(bal & lt);
           if (r < p.rows_cap) {
             uint32_t *dst = (uint32_t *)(rows + r * orow);
-            for (int c = 0; c < nw1; ++c) dst[c] = ((const uint32_t *)ta)[p.pw1[c]];
+#pragma unroll
+            for (int c = 0; c < kJoinEmitWords; ++c)
+              if (c < nw1) dst[c] = pa[c];
 #pragma unroll
             for (int c = 0; c < kJoinEmitWords; ++c)
               if (c < nw2) dst[nw1 + c] = pj[c * kJoinChunk + b];
@@ -427,7 +442,7 @@ static saber_status join_task(saber_join *j, const unsigned char *d1, const unsi
     k_join_scan<<<148 * 4, kJoinThreads, 0, j->cs>>>(j->counts, nwin * p.s, j->status, j->ticket, j->epoch,
                                                      s.d_total);
     JCK(cudaGetLastError());
-    if (fast && p.nw2 <= kJoinEmitWords && !std::getenv("SABER_JOIN_THREAD_EMIT"))
+    if (fast && p.nw2 <= kJoinEmitWords && p.nw1 <= kJoinEmitWords && !std::getenv("SABER_JOIN_THREAD_EMIT"))
       k_join_emit_i32<<<grid, kJoinThreads, fsmem + (size_t)kJoinEmitWords * kJoinChunk * 4, j->cs>>>(
           p, v1, v2, j->J0, j->counts, s.rows);
     else if (fast) k_join_pairs_i32<true><<<grid, kJoinThreads, fsmem, j->cs>>>(p, v1, v2, j->J0, nullptr, j->counts, s.rows);
