@@ -53,19 +53,22 @@ def step():
         HT.append(("submit", (time.perf_counter() - t0) * 1e6))
         if st == saber.EAGAIN:
             st_, r = q.poll_raw(-1)
-            q.release(r)
+            if st_ == 0:
+                q.release(r)
             continue
         assert st == 0, q.last_error()
         off += nb
     t0 = time.perf_counter()
     while q.finish() == saber.EAGAIN:
         st_, r = q.poll_raw(-1)
-        q.release(r)
+        if st_ == 0:
+            q.release(r)
     HT.append(("finish", (time.perf_counter() - t0) * 1e6))
     q.record(s.cuda_stream)
     while q.stats()["tasks_pending"] > 0:
         st_, r = q.poll_raw(-1)
-        q.release(r)
+        if st_ == 0:
+            q.release(r)
     torch.cuda.synchronize()
 
 
