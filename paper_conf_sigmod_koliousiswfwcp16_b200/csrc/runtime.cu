@@ -475,6 +475,7 @@ static saber_status size_plan(saber_query *q) {
       const double B = p.key_pack == KP_RADIX ? (double)p.G / (double)p.C : 1e30;
       const double per_slot = std::max(1e-9, std::min(A, B));
       int64_t sb = floor_pow2(std::max<int64_t>(1, (int64_t)(p.state_cap / (2.0 * per_slot))));
+      if (const char *hsb = std::getenv("SABER_HASH_SB")) sb = floor_pow2(std::max(1, std::atoi(hsb)));
       if (sb > p.C) sb = p.C;
       p.SB = (int)sb;
       p.S = (int)(p.C / sb);
