@@ -785,6 +785,7 @@ k_win_vh(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ pre,
 }
 
 // HASH: block-wide state hash keyed by the group key; slab = home-slot range
+constexpr int kHashMaxChunk = 128;      // windows per item (win_chunk <= 128)
 template <bool EMIT>
 __global__ void __launch_bounds__(256)
 k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ table,
@@ -805,116 +806,141 @@ k_win_hash(const Plan p, State *__restrict__ st, const uint64_t *__restrict__ ta
   const int64_t J0 = st->J0, J1 = st->J1, nw = J1 - J0;
   if (nw <= 0) return;
   const int64_t maxprobe = (int64_t)st->max_probe;
-  const int64_t span = (SB + maxprobe + 1) < p.C ? (SB + maxprobe + 1) : p.C;
   const int64_t nchunks = (nw + W - 1) / W;
   const int64_t nitems = nchunks * S;
   if (threadIdx.x == 0) s_err = 0;
+  // An item is (window chunk, key slab).  If its state overflows (more distinct keys
+  // than ST), the item restarts with its slab split into 2, 4, ... sub-slabs of home
+  // slots, each slid on its own; the count and emit passes overflow on the same key
+  // sets, so both pick the same split (rows of a window stay inside its (window,
+  // slab) range, sub-slab after sub-slab -- row order inside a window is free, A8).
+  __shared__ int s_ovf;
+  __shared__ int64_t s_wrun[kHashMaxChunk];            // rows of earlier sub-slabs per window
   for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
     const int64_t chunk = item / S;
-    const uint32_t slot0 = (uint32_t)((item % S) * SB);
+    const uint32_t slab0 = (uint32_t)((item % S) * SB);
     const int64_t ja = J0 + chunk * W;
     const int64_t jb = ja + W < J1 ? ja + W : J1;
-    __syncthreads();
-    for (int h = threadIdx.x; h < ST; h += blockDim.x) {
-      skeys[h] = kEmpty;
-      scnt[h] = 0;
-      FOR_F(f) { sf[f * ST + h] = field_identity(p.field[f].kind); sc[f * ST + h] = 0.0; }
-    }
-    if (threadIdx.x == 0) s_nocc = 0;
-    __syncthreads();
-    auto find = [&](uint64_t k) -> int {
-      uint32_t h = (uint32_t)(fmix64(k) >> 32) & (uint32_t)(ST - 1);
-      volatile uint64_t *vk = skeys;
-      for (int probe = 0; probe < ST; ++probe) {
-        uint64_t cur = vk[h];
-        if (cur == k) return (int)h;
-        if (cur == kEmpty) {
-          uint64_t old = atomicCAS((unsigned long long *)&skeys[h], kEmpty, k);
-          if (old == kEmpty) occ[atomicAdd(&s_nocc, 1)] = (int)h;
-          if (old == kEmpty || old == k) return (int)h;
-        }
-        h = (h + 1) & (uint32_t)(ST - 1);
-      }
-      s_err = 1;
-      return -1;
-    };
-    // mode 0: add (+1) / subtract (-1) invertible fields; mode 2: min/max only
-    auto visit_pane = [&](int64_t q, int sign, bool minmax) {
-      const uint64_t *b = table + (q & (p.R - 1)) * p.slot_words;
-      for (int64_t o = threadIdx.x; o < span; o += blockDim.x) {
-        const uint32_t h = (slot0 + (uint32_t)o) & Cm;
-        const uint64_t k = b[h];
-        if (k == kEmpty) continue;
-        const uint32_t home = (uint32_t)fmix64(k) & Cm;
-        if (((home - slot0) & Cm) >= (uint32_t)SB) continue;
-        const int s = find(k);
-        if (s < 0) continue;
-        if (!minmax) {
-          atomicAdd((unsigned long long *)&scnt[s], (unsigned long long)(sign * (int64_t)b[p.C + h]));
-        }
-        FOR_F(f) {
-          const int kind = p.field[f].kind;
-          const uint64_t v = b[fld_off(p, f) + h];
-          if (!minmax && kind == FK_SUM_F)
-            dd_atomic_add((double *)&sf[f * ST + s], &sc[f * ST + s], sign * __longlong_as_double((long long)v));
-          else if (!minmax && kind == FK_SUM_I) atomicAdd((unsigned long long *)&sf[f * ST + s], (unsigned long long)(sign * (int64_t)v));
-          else if (minmax && kind == FK_MIN) atomicMin((unsigned long long *)&sf[f * ST + s], (unsigned long long)v);
-          else if (minmax && kind == FK_MAX) atomicMax((unsigned long long *)&sf[f * ST + s], (unsigned long long)v);
-        }
-      }
-    };
-    for (int64_t q = ja * p.L; q < ja * p.L + p.K; ++q) visit_pane(q, +1, false);
-    for (int64_t j = ja; j < jb; ++j) {
-      if (j > ja) {
-        for (int64_t q = (j - 1) * p.L + p.K; q < j * p.L + p.K; ++q) visit_pane(q, +1, false);
-        for (int64_t q = (j - 1) * p.L; q < j * p.L; ++q) visit_pane(q, -1, false);
-      }
-      __syncthreads();
-      const int nocc = s_nocc;
-      for (int x = threadIdx.x; x < nocc; x += blockDim.x) {
-        const int h = occ[x];
-        if (scnt[h] == 0)
-          FOR_F(f)
-            if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) { sf[f * ST + h] = 0; sc[f * ST + h] = 0.0; }
-      }
-      if (p.has_minmax) {
-        for (int x = threadIdx.x; x < nocc; x += blockDim.x)
-          FOR_F(f)
-            if (p.field[f].kind == FK_MIN || p.field[f].kind == FK_MAX)
-              sf[f * ST + occ[x]] = field_identity(p.field[f].kind);
+    for (int nsub = 1;; nsub *= 2) {
+      const int SBs = SB / nsub;
+      bool overflow = false;
+      for (int sub = 0; sub < nsub && !overflow; ++sub) {
+        const uint32_t slot0 = slab0 + (uint32_t)(sub * SBs);
         __syncthreads();
-        for (int64_t q = j * p.L; q < j * p.L + p.K; ++q) visit_pane(q, 0, true);
-      }
-      __syncthreads();
-      int my = 0;
-      uint64_t fv[kMaxField];
-      const int nocc2 = s_nocc;                         // the min/max visit may have added keys
-      for (int x = threadIdx.x; x < nocc2; x += blockDim.x) {
-        const int h = occ[x];
-        if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
-        FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
-            __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];
-        if (having_ok(p, scnt[h], fv)) ++my;
-      }
-      int total;
-      int excl = group_excl_scan(my, 256, scan_sm, total);
-      const int64_t ci = (j - J0) * S + (item % S);
-      if (!EMIT) {
-        if (threadIdx.x == 0) counts[ci] = total;
-      } else {
-        int64_t r = counts[ci] + excl;
-        for (int x = threadIdx.x; x < nocc2; x += blockDim.x) {
-          const int h = occ[x];
-          if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
-          FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
-            __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];
-          if (!having_ok(p, scnt[h], fv)) continue;
-          int64_t kv[kMaxKey];
-          decode_key(p, skeys[h], kv);
-          write_row(p, rows, r++, kv, scnt[h], fv);
+        for (int h = threadIdx.x; h < ST; h += blockDim.x) {
+          skeys[h] = kEmpty;
+          scnt[h] = 0;
+          FOR_F(f) { sf[f * ST + h] = field_identity(p.field[f].kind); sc[f * ST + h] = 0.0; }
+        }
+        if (threadIdx.x == 0) { s_nocc = 0; s_ovf = 0; }
+        for (int x = threadIdx.x; x < (int)(jb - ja); x += blockDim.x)
+          if (sub == 0) s_wrun[x] = 0;
+        __syncthreads();
+        auto find = [&](uint64_t k) -> int {
+          uint32_t h = (uint32_t)(fmix64(k) >> 32) & (uint32_t)(ST - 1);
+          volatile uint64_t *vk = skeys;
+          for (int probe = 0; probe < ST; ++probe) {
+            uint64_t cur = vk[h];
+            if (cur == k) return (int)h;
+            if (cur == kEmpty) {
+              uint64_t old = atomicCAS((unsigned long long *)&skeys[h], kEmpty, k);
+              if (old == kEmpty) occ[atomicAdd(&s_nocc, 1)] = (int)h;
+              if (old == kEmpty || old == k) return (int)h;
+            }
+            h = (h + 1) & (uint32_t)(ST - 1);
+          }
+          s_ovf = 1;
+          return -1;
+        };
+        // mode 0: add (+1) / subtract (-1) invertible fields; mode 2: min/max only
+        auto visit_pane = [&](int64_t q, int sign, bool minmax) {
+          const uint64_t *b = table + (q & (p.R - 1)) * p.slot_words;
+          const int64_t sp = (SBs + maxprobe + 1) < p.C ? (SBs + maxprobe + 1) : p.C;
+          for (int64_t o = threadIdx.x; o < sp; o += blockDim.x) {
+            const uint32_t h = (slot0 + (uint32_t)o) & Cm;
+            const uint64_t k = b[h];
+            if (k == kEmpty) continue;
+            const uint32_t home = (uint32_t)fmix64(k) & Cm;
+            if (((home - slot0) & Cm) >= (uint32_t)SBs) continue;
+            const int s = find(k);
+            if (s < 0) continue;
+            if (!minmax) {
+              atomicAdd((unsigned long long *)&scnt[s], (unsigned long long)(sign * (int64_t)b[p.C + h]));
+            }
+            FOR_F(f) {
+              const int kind = p.field[f].kind;
+              const uint64_t v = b[fld_off(p, f) + h];
+              if (!minmax && kind == FK_SUM_F)
+                dd_atomic_add((double *)&sf[f * ST + s], &sc[f * ST + s], sign * __longlong_as_double((long long)v));
+              else if (!minmax && kind == FK_SUM_I) atomicAdd((unsigned long long *)&sf[f * ST + s], (unsigned long long)(sign * (int64_t)v));
+              else if (minmax && kind == FK_MIN) atomicMin((unsigned long long *)&sf[f * ST + s], (unsigned long long)v);
+              else if (minmax && kind == FK_MAX) atomicMax((unsigned long long *)&sf[f * ST + s], (unsigned long long)v);
+            }
+          }
+        };
+        for (int64_t q = ja * p.L; q < ja * p.L + p.K; ++q) visit_pane(q, +1, false);
+        for (int64_t j = ja; j < jb; ++j) {
+          if (j > ja) {
+            for (int64_t q = (j - 1) * p.L + p.K; q < j * p.L + p.K; ++q) visit_pane(q, +1, false);
+            for (int64_t q = (j - 1) * p.L; q < j * p.L; ++q) visit_pane(q, -1, false);
+          }
+          __syncthreads();
+          if (s_ovf) { overflow = true; break; }          // block-uniform (read after the barrier)
+          const int nocc = s_nocc;
+          for (int x = threadIdx.x; x < nocc; x += blockDim.x) {
+            const int h = occ[x];
+            if (scnt[h] == 0)
+              FOR_F(f)
+                if (p.field[f].kind == FK_SUM_F || p.field[f].kind == FK_SUM_I) { sf[f * ST + h] = 0; sc[f * ST + h] = 0.0; }
+          }
+          if (p.has_minmax) {
+            for (int x = threadIdx.x; x < nocc; x += blockDim.x)
+              FOR_F(f)
+                if (p.field[f].kind == FK_MIN || p.field[f].kind == FK_MAX)
+                  sf[f * ST + occ[x]] = field_identity(p.field[f].kind);
+            __syncthreads();
+            for (int64_t q = j * p.L; q < j * p.L + p.K; ++q) visit_pane(q, 0, true);
+          }
+          __syncthreads();
+          if (s_ovf) { overflow = true; break; }
+          int my = 0;
+          uint64_t fv[kMaxField];
+          const int nocc2 = s_nocc;                         // the min/max visit may have added keys
+          for (int x = threadIdx.x; x < nocc2; x += blockDim.x) {
+            const int h = occ[x];
+            if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
+            FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
+                __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];
+            if (having_ok(p, scnt[h], fv)) ++my;
+          }
+          int total;
+          int excl = group_excl_scan(my, 256, scan_sm, total);
+          const int64_t ci = (j - J0) * S + (item % S);
+          const int wi = (int)(j - ja);
+          if (!EMIT) {
+            if (threadIdx.x == 0) counts[ci] = (sub == 0 ? 0 : counts[ci]) + total;
+          } else {
+            int64_t r = counts[ci] + s_wrun[wi] + excl;
+            for (int x = threadIdx.x; x < nocc2; x += blockDim.x) {
+              const int h = occ[x];
+              if (skeys[h] == kEmpty || scnt[h] <= 0) continue;
+              FOR_F(f) fv[f] = p.field[f].kind == FK_SUM_F ? (uint64_t)__double_as_longlong(
+                __longlong_as_double((long long)sf[f * ST + h]) + sc[f * ST + h]) : sf[f * ST + h];
+              if (!having_ok(p, scnt[h], fv)) continue;
+              int64_t kv[kMaxKey];
+              decode_key(p, skeys[h], kv);
+              write_row(p, rows, r++, kv, scnt[h], fv);
+            }
+          }
+          __syncthreads();
+          if (threadIdx.x == 0) s_wrun[wi] += total;
         }
       }
-      __syncthreads();
+      if (!overflow) break;
+      if (SB / (2 * nsub) < 1) {                          // one home slot and still too many keys
+        if (threadIdx.x == 0) s_err = 1;
+        break;
+      }
     }
   }
   __syncthreads();

@@ -471,7 +471,11 @@ static saber_status size_plan(saber_query *q) {
       p.GS = 256;
       p.state_cap = (int)floor_pow2(smem_budget / (8 * (2 + 2 * p.nf) + 4));   // keys, counts, fields, compensation, occupancy list
       if (const char *hs = std::getenv("SABER_HASH_STATE")) p.state_cap = (int)floor_pow2(std::max(64, std::atoi(hs)));
-      const double A = (double)(p.K + q->win_chunk * p.L) / 2.0;
+      // keys a home slot contributes to an item: one per pane it is occupied in.  Sized for
+      // an eighth of the pane slots occupied (hash capacities are planned at >= 2x a pane's
+      // distinct keys); an item whose state still overflows restarts split into 2, 4, ...
+      // sub-slabs (k_win_hash), so a denser stream costs time, not correctness (CM2: 4 -> 1 slab)
+      const double A = (double)(p.K + q->win_chunk * p.L) / 8.0;
       const double B = p.key_pack == KP_RADIX ? (double)p.G / (double)p.C : 1e30;
       const double per_slot = std::max(1e-9, std::min(A, B));
       int64_t sb = floor_pow2(std::max<int64_t>(1, (int64_t)(p.state_cap / (2.0 * per_slot))));
