@@ -111,7 +111,7 @@ CONFIGS = {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5a": c5a, "C5b": c5b, "SG1"
 
 # Task size φ (MiB) bench.py uses per config (device-resident leg): the B200
 # plateau of DESIGN.md §8, bounded where one task's result rows must fit a slot.
-BENCH_TASK_MB = {"C1": 32, "C2": 1024, "C3": 4096, "C3_G256": 4096, "C3_G1024": 1024, "C3_G4096": 1024,
+BENCH_TASK_MB = {"C1": 32, "C2": 1024, "C3": 4096, "C3_G256": 4096, "C3_G1024": 4096, "C3_G4096": 2048,
                  "C3_G16384": 512, "C3_G65536": 256, "C4": 4096, "C5a": 4096, "C5b": 4096, "SG1": 4096,
                  "CM2": 1024}
 
